@@ -1,0 +1,14 @@
+"""Oracle package -- TEST INFRASTRUCTURE ONLY.
+
+Only ``tests/``, ``__graft_entry__.smoke()`` and ``bench.py``'s ``cpu_baseline`` /
+``--impl reference`` legs may import anything under ``oracle/``.  The product path
+(``paper_conf_ppopp_moscovicicp17_b200``) never imports it, and the oracle never
+imports the product path: they share no code.
+
+* ``oracle.oracle_a`` -- Oracle-A, the plain definition of a batch's results and final
+  set (a sequential Pugh skiplist in C, S1 snapshot-batch semantics).  See
+  ``oracle_a.c``'s header for the cited passages.
+* ``oracle.oracle_b`` -- Oracle-B, the paper's GFSL algorithm step by step (Alg 4.1-4.12)
+  as a sequential single-team Python model over the same chunk layout, pinned by the
+  paper's worked examples.
+"""
