@@ -1,0 +1,192 @@
+/*
+ * gfsl.h -- C ABI of the B200-native GFSL (GPU-Friendly SkipList) hot path.
+ *
+ * GFSL is the chunked skiplist of Moscovici, Cohen & Petrank (PPoPP'17 / PACT'17),
+ * /root/reference/PAPER.md ("P:n" = PAPER.md line n).  It is an ordered map over
+ * 32-bit unsigned keys and values (Table 4.1) with three operations:
+ *   Contains(k)  -> bool                     Alg 4.1
+ *   Insert(k, v) -> false iff k is present  Alg 4.5
+ *   Delete(k)    -> false iff k is absent   Alg 4.11
+ * and work arrives as an array of (op type, key).
+ *
+ * Plain C: no CUDA or torch types.  Streams are passed as `void*` holding a
+ * cudaStream_t (NULL = the legacy default stream).  All functions are host functions;
+ * a handle is bound to the CUDA device that was current when it was created and must
+ * be used from a single host thread at a time.
+ *
+ * Batch semantics (reading R1, "S1 snapshot batch"): for every op of a batch
+ * the result is computed against the map as it was BEFORE the batch; the map after the
+ * batch is  M + {successful inserts} - {successful deletes}.  Contract: at most one
+ * mutating op (Insert/Delete) per key per batch.  Outside the contract every result is
+ * still the result of SOME linearization of the batch, but parity with the
+ * oracle is only promised inside it.
+ *
+ * Keys are valid in [0, key_range), key_range <= 2^32 - 2 (the two extremes of the
+ * 32-bit internal key space are the -inf / +inf sentinels of P:203).  Any uint32 is a
+ * valid value.  Invalid ops (op code > 2, or key >= key_range) get result
+ * GFSL_RESULT_INVALID and have no effect.
+ */
+#ifndef GFSL_H_
+#define GFSL_H_
+
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef struct gfsl gfsl;
+typedef gfsl *gfsl_t;
+
+typedef enum gfsl_status {
+  GFSL_OK = 0,
+  GFSL_EINVAL = 1,   /* bad host argument (NULL handle, bad size, ...) */
+  GFSL_ENOMEM = 2,   /* device or host allocation failed */
+  GFSL_EPOOL = 3,    /* chunk pool exhausted: sticky; the structure is undefined */
+  GFSL_ECUDA = 4,    /* a CUDA runtime call failed: sticky */
+  GFSL_ECORRUPT = 5  /* gfsl_validate found an invariant violation */
+} gfsl_status;
+
+/* Op codes (the "operation type" of the op array). */
+enum { GFSL_CONTAINS = 0, GFSL_INSERT = 1, GFSL_DELETE = 2 };
+/* Per-op result codes. */
+enum { GFSL_RESULT_FALSE = 0, GFSL_RESULT_TRUE = 1, GFSL_RESULT_INVALID = 0xFF };
+
+typedef struct gfsl_config {
+  uint32_t chunk_entries;   /* N: 16 (128-B chunks) or 32 (256-B chunks).
+                               0 = 32.  MAX_LEVEL = N (path held one level per lane,
+                               P:493-495). */
+  uint32_t contains_team;   /* lanes per Contains team (a power of two dividing N, >= 4);
+                               0 = the tuned default.  P:205 allows teams <= a warp. */
+  uint32_t contains_blocks_per_sm; /* launch shape of the Contains kernel; 0 = default */
+  uint32_t update_blocks_per_sm;   /* launch shape of the update kernel; 0 = default */
+  uint32_t serial_updates;  /* 1 = one team applies the updates strictly in op order
+                               (deterministic structure; test mode).  0 = concurrent. */
+  uint32_t reserved[3];
+} gfsl_config;
+
+/*
+ * Create an empty GFSL (one unlocked chunk per level holding -inf with a pointer
+ * to the level below; head array; per-level counters = 0).
+ *   key_range : keys are valid in [0, key_range); 1 <= key_range <= 2^32 - 2.
+ *   capacity  : the maximum number of live keys the caller will store; 0 = key_range.
+ *               The library sizes the pre-allocated chunk pools from it.
+ * Returns NULL on failure (see gfsl_last_error()).
+ */
+gfsl_t gfsl_create(uint64_t key_range, uint64_t capacity);
+gfsl_t gfsl_create_ex(uint64_t key_range, uint64_t capacity, const gfsl_config *cfg);
+
+/* Release every device resource of the handle (synchronizes the device first). */
+void gfsl_destroy(gfsl_t h);
+
+/*
+ * Run one batch of n ops, asynchronously on `stream`.
+ *   op_types : device pointer, n x uint8  (GFSL_CONTAINS / _INSERT / _DELETE)
+ *   keys     : device pointer, n x uint32
+ *   values   : device pointer, n x uint32 (read for inserts only; may be NULL, = 0)
+ *   results  : device pointer, n x uint8  (written: GFSL_RESULT_*), in input order
+ * All arrays belong to the caller, must be on the handle's device, and must stay valid
+ * until `stream` reaches the end of the batch.  Batches on one handle are serialized in
+ * issue order (the handle makes each batch wait for the previous one).
+ * Returns GFSL_EINVAL for bad host arguments, or a sticky error (GFSL_EPOOL, GFSL_ECUDA)
+ * raised by an earlier batch; on error nothing is enqueued.
+ */
+gfsl_status gfsl_batch(gfsl_t h, const uint8_t *op_types, const uint32_t *keys,
+                       const uint32_t *values, uint8_t *results, uint64_t n,
+                       void *stream);
+
+/*
+ * Same batch through HOST buffers (pageable or pinned): copies the ops in, runs the
+ * batch, copies the results out, and returns when `results` holds them (synchronous).
+ * This is the end-to-end entry point; the copies go through library-owned pinned
+ * staging buffers on `stream`.
+ */
+gfsl_status gfsl_batch_host(gfsl_t h, const uint8_t *op_types, const uint32_t *keys,
+                            const uint32_t *values, uint8_t *results, uint64_t n,
+                            void *stream);
+
+/* Result of gfsl_validate: the invariants of PAPER.md §4.3 and P:203. */
+typedef struct gfsl_report {
+  uint64_t keys;                /* live keys (bottom level, non-zombie chunks) */
+  uint32_t height;              /* highest level with counter > 0 */
+  uint32_t chunk_entries;       /* N */
+  uint64_t chunks[32];          /* non-zombie chunks reachable per level */
+  uint64_t zombies[32];         /* zombie chunks still linked per level */
+  uint64_t level_keys[32];      /* real keys per level */
+  int64_t  counters[32];        /* the per-level counters as stored */
+  uint64_t pool_used[2];        /* chunks allocated: [0] bottom pool, [1] upper pool */
+  uint64_t pool_cap[2];
+  uint32_t violations;          /* bitmask: bit v-1 set = invariant Vv violated */
+  uint32_t first_violation;     /* lowest violated invariant number, 0 if none */
+  uint64_t restarts;            /* Contains/search restarts so far */
+  uint64_t reserved[4];
+} gfsl_report;
+
+/*
+ * Synchronous structural check and export.  Waits for all batches, walks every level
+ * from its head and checks V1-V12.  If keys_out/vals_out are
+ * non-NULL (host pointers), writes up to `cap` live (key, value) pairs in ascending key
+ * order and sets *count to the number of live keys.  rep and count may be NULL.
+ * Returns GFSL_OK, GFSL_ECORRUPT (rep->violations says which), or an error.
+ */
+gfsl_status gfsl_validate(gfsl_t h, gfsl_report *rep, uint32_t *keys_out,
+                          uint32_t *vals_out, uint64_t cap, uint64_t *count);
+
+/* Human-readable description of the last error on this thread. */
+const char *gfsl_last_error(void);
+
+/* Counters since creation (debug statistics). */
+typedef struct gfsl_stats {
+  uint64_t batches, ops;
+  uint64_t restarts;        /* traversal restarts (Alg 4.2 l.25) */
+  uint64_t splits, merges;  /* Alg 4.9 / Alg 4.12 */
+  uint64_t zombie_unlinks;  /* Alg 4.6 l.10-20 redirects */
+  uint64_t lock_retries;    /* failed CAS / waits in findAndLockEnclosing (Alg 4.8) */
+  uint64_t reserved[8];
+} gfsl_stats;
+gfsl_status gfsl_get_stats(gfsl_t h, gfsl_stats *out);
+
+/* ---- test-only: raw pool access (T2 byte parity, worked-example fixtures) ----
+ * Pool image layout (host memory, little endian):
+ *   uint64 entries[(cap_bottom + cap_upper) * N]   chunk c at entries[c*N .. c*N+N)
+ * Chunk indices [0, cap_upper) are the upper pool, [cap_upper, cap_upper+cap_bottom)
+ * the bottom pool.  The meta block is: head[N] (uint32), counters[N] (int32),
+ * used_bottom, used_upper (uint32).  Internal key = user key + 1; 0 = -inf;
+ * 0xFFFFFFFF = +inf = EMPTY = null pointer. */
+typedef struct gfsl_meta {
+  uint32_t head[32];
+  int32_t counters[32];
+  uint32_t used_bottom, used_upper;
+  uint32_t cap_bottom, cap_upper;
+  uint32_t chunk_entries;
+  uint32_t reserved[3];
+} gfsl_meta;
+gfsl_status gfsl_dump(gfsl_t h, gfsl_meta *meta, uint64_t *entries, uint64_t max_entries);
+gfsl_status gfsl_load(gfsl_t h, const gfsl_meta *meta, const uint64_t *entries,
+                      uint64_t n_entries);
+
+/* ---- multi-GPU range routing (B5) ----
+ * Shard g owns keys [g*ceil(R/G), min(R, (g+1)*ceil(R/G))).  The collective exchange
+ * between these calls is done by the caller (torch.distributed / NCCL).
+ *
+ * gfsl_route_plan: per-op destination and stable order.  Writes counts[G] (device,
+ *   uint64, number of ops for each destination) and perm[n] (device, uint32: perm[j] =
+ *   input index of the j-th op in destination-major, input-stable order).  Invalid keys
+ *   are routed to shard 0, which reports them invalid.
+ * gfsl_route_pack: packs ops in perm order into send_op/send_key/send_val.
+ * gfsl_route_unpack: results[perm[j]] = recv_res[j].
+ */
+gfsl_status gfsl_route_plan(const uint8_t *op_types, const uint32_t *keys, uint64_t n,
+                            uint64_t key_range, uint32_t world, uint64_t *counts,
+                            uint32_t *perm, void *stream);
+gfsl_status gfsl_route_pack(const uint32_t *perm, const uint8_t *op_types,
+                            const uint32_t *keys, const uint32_t *values, uint64_t n,
+                            uint8_t *send_op, uint32_t *send_key, uint32_t *send_val,
+                            void *stream);
+gfsl_status gfsl_route_unpack(const uint32_t *perm, const uint8_t *recv_res, uint64_t n,
+                              uint8_t *results, void *stream);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* GFSL_H_ */

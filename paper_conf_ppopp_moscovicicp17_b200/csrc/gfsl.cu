@@ -1,0 +1,832 @@
+// gfsl.cu -- libgfsl: the C ABI of include/gfsl.h over the sm_100a kernels.
+//
+// A batch is enqueued as (DESIGN.md §Batch pipeline):
+//   memset(ctl) -> classify (a2) -> contains_kernel (B1, a3) -> update_kernel (B2, a4/a5)
+// with no host synchronization.  The library owns the chunk pool, the head
+// array and per-level counters, the bump counters and the sticky error word; the
+// caller owns the op / key / value / result arrays.
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <cstdio>
+#include <cstring>
+#include <string>
+#include <vector>
+
+#include "../../include/gfsl.h"
+#include "gfsl_contains.cuh"
+#include "gfsl_device.cuh"
+#include "gfsl_update.cuh"
+
+using namespace gfsl_dev;
+
+// ------------------------------------------------------------------------------------
+// errors
+static thread_local std::string g_last_error = "no error";
+static void set_last_error(const std::string &s) { g_last_error = s; }
+extern "C" const char *gfsl_last_error(void) { return g_last_error.c_str(); }
+
+#define CK(call)                                                                      \
+  do {                                                                                \
+    cudaError_t e_ = (call);                                                          \
+    if (e_ != cudaSuccess) {                                                          \
+      set_last_error(std::string(#call) + ": " + cudaGetErrorString(e_));             \
+      return GFSL_ECUDA;                                                              \
+    }                                                                                 \
+  } while (0)
+
+struct gfsl {
+  int device = 0;
+  int sms = 148;
+  uint32_t N = 32;
+  uint32_t team = 8;
+  gfsl_config cfg{};
+  uint64_t key_range = 0;
+  DevState d{};
+  BatchCtl *ctl = nullptr;
+  uint32_t *list_c = nullptr, *list_u = nullptr;
+  uint64_t list_cap = 0;
+  uint32_t *h_error = nullptr;  // mapped host memory, device alias in d.error
+  cudaEvent_t last = nullptr;
+  bool sticky_cuda = false;
+  int contains_grid = 0, update_grid = 0;
+  // staging for gfsl_batch_host
+  uint8_t *st_op = nullptr, *st_res = nullptr;
+  uint32_t *st_key = nullptr, *st_val = nullptr;
+  uint64_t st_cap = 0;
+  uint64_t batches = 0, ops = 0;
+};
+
+// ------------------------------------------------------------------------------------
+// kernels: pool init and classify (a2)
+
+// Every pool chunk starts in the "allocated" state of P:237: all entries +inf, max +inf,
+// locked.  Allocation is then only a bump of the counter.
+__global__ void init_pool_kernel(uint64_t *pool, uint64_t total_entries, uint32_t N) {
+  for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < total_entries;
+       i += (uint64_t)gridDim.x * blockDim.x) {
+    pool[i] = (i % N == N - 1) ? (uint64_t)LOCK_HELD : EMPTY_ENTRY;
+  }
+}
+
+// The initial structure: one unlocked chunk per level holding -inf, pointing to
+// the level below; the head array points at them; counters are 0.
+__global__ void init_heads_kernel(DevState d, uint32_t N) {
+  const uint32_t l = threadIdx.x;
+  if (l >= N) return;
+  const uint32_t c = (l == 0) ? d.cap_upper : (l - 1);  // level 0 in the bottom pool
+  const uint32_t below = (l == 0) ? 0u : ((l == 1) ? d.cap_upper : (l - 2));
+  uint64_t *ch = d.pool + (size_t)c * N;
+  ch[0] = mk64(KEY_NEG_INF, l == 0 ? 0u : below);
+  ch[N - 2] = mk64(KEY_POS_INF, NULL_CHUNK);
+  ch[N - 1] = mk64(LOCK_FREE, 0u);
+  d.head[l] = c;
+  d.counter[l] = 0;
+  if (l == 0) {
+    d.bump[0] = 1;
+    d.bump[1] = N - 1;
+  }
+}
+
+// Batch intake: range/op-code check (invalid -> 0xFF, no effect) and the split into the
+// Contains list and the Insert/Delete list (warp-aggregated appends).
+__global__ void classify_kernel(const uint8_t *__restrict__ ops, const uint32_t *__restrict__ keys,
+                                uint8_t *__restrict__ res, uint32_t n, uint64_t key_range,
+                                uint32_t *__restrict__ list_c, uint32_t *__restrict__ list_u,
+                                BatchCtl *ctl) {
+  const int lane = threadIdx.x & 31;
+  const uint32_t stride = gridDim.x * blockDim.x;
+  for (uint32_t base = blockIdx.x * blockDim.x; base < n; base += stride) {
+    const uint32_t i = base + threadIdx.x;
+    bool isc = false, isu = false;
+    if (i < n) {
+      const uint8_t op = ops[i];
+      const uint32_t k = keys[i];
+      const bool valid = op <= 2 && (uint64_t)k < key_range;
+      if (!valid) res[i] = 0xFF;
+      isc = valid && op == 0;
+      isu = valid && op != 0;
+    }
+    const uint32_t bc = __ballot_sync(0xFFFFFFFFu, isc);
+    const uint32_t bu = __ballot_sync(0xFFFFFFFFu, isu);
+    uint32_t oc = 0, ou = 0;
+    if (lane == 0) {
+      if (bc) oc = atomicAdd(&ctl->n_contains, __popc(bc));
+      if (bu) ou = atomicAdd(&ctl->n_updates, __popc(bu));
+    }
+    oc = __shfl_sync(0xFFFFFFFFu, oc, 0);
+    ou = __shfl_sync(0xFFFFFFFFu, ou, 0);
+    const uint32_t below = (1u << lane) - 1u;
+    if (isc) list_c[oc + __popc(bc & below)] = i;
+    if (isu) list_u[ou + __popc(bu & below)] = i;
+  }
+}
+
+// ------------------------------------------------------------------------------------
+// template dispatch
+
+template <int N, int TEAM>
+static void launch_contains(gfsl *h, const uint32_t *keys, uint8_t *res, cudaStream_t s) {
+  contains_kernel<N, TEAM><<<h->contains_grid, 256, 0, s>>>(h->d, keys, res, h->list_c, h->ctl);
+}
+
+#define GFSL_CONTAINS_CONFIGS(X) X(32, 8) X(32, 16) X(32, 32) X(16, 4) X(16, 8) X(16, 16) X(12, 12) X(6, 6)
+
+static bool dispatch_contains(gfsl *h, const uint32_t *keys, uint8_t *res, cudaStream_t s) {
+  switch (h->N * 100 + h->team) {
+#define X(n, t) case n * 100 + t: launch_contains<n, t>(h, keys, res, s); return true;
+    GFSL_CONTAINS_CONFIGS(X)
+#undef X
+  }
+  return false;
+}
+
+template <int N>
+static void launch_update(gfsl *h, const uint8_t *ops, const uint32_t *keys, const uint32_t *vals,
+                          uint8_t *res, uint32_t n, cudaStream_t s) {
+  if (h->cfg.serial_updates) {
+    update_kernel<N><<<1, 32, 0, s>>>(h->d, ops, keys, vals, res, h->list_u, h->ctl, 1, n);
+  } else {
+    update_kernel<N><<<h->update_grid, 256, 0, s>>>(h->d, ops, keys, vals, res, h->list_u, h->ctl, 0, n);
+  }
+}
+
+template <int N, int TEAM>
+static int occ_contains() {
+  int b = 0;
+  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, contains_kernel<N, TEAM>, 256, 0);
+  return b;
+}
+template <int N>
+static int occ_update() {
+  int b = 0;
+  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, update_kernel<N>, 256, 0);
+  return b;
+}
+
+static bool valid_team(uint32_t N, uint32_t team) {
+  switch (N * 100 + team) {
+#define X(n, t) case n * 100 + t: return true;
+    GFSL_CONTAINS_CONFIGS(X)
+#undef X
+  }
+  return false;
+}
+
+static int contains_occupancy(uint32_t N, uint32_t team) {
+  switch (N * 100 + team) {
+#define X(n, t) case n * 100 + t: return occ_contains<n, t>();
+    GFSL_CONTAINS_CONFIGS(X)
+#undef X
+  }
+  return 1;
+}
+static int update_occupancy(uint32_t N) {
+  switch (N) {
+    case 32: return occ_update<32>();
+    case 16: return occ_update<16>();
+    case 12: return occ_update<12>();
+    case 6: return occ_update<6>();
+  }
+  return 1;
+}
+
+// ------------------------------------------------------------------------------------
+// create / destroy
+
+static void free_all(gfsl *h) {
+  if (!h) return;
+  cudaFree(h->d.pool);
+  cudaFree(h->d.head);
+  cudaFree(h->d.counter);
+  cudaFree(h->d.bump);
+  cudaFree(h->d.stats);
+  cudaFree(h->ctl);
+  cudaFree(h->list_c);
+  cudaFree(h->list_u);
+  cudaFree(h->st_op);
+  cudaFree(h->st_res);
+  cudaFree(h->st_key);
+  cudaFree(h->st_val);
+  if (h->h_error) cudaFreeHost(h->h_error);
+  if (h->last) cudaEventDestroy(h->last);
+  delete h;
+}
+
+extern "C" gfsl_t gfsl_create_ex(uint64_t key_range, uint64_t capacity, const gfsl_config *cfg_in) {
+  gfsl_config cfg{};
+  if (cfg_in) cfg = *cfg_in;
+  if (cfg.chunk_entries == 0) cfg.chunk_entries = 32;
+  const uint32_t N = cfg.chunk_entries;
+  if (N != 32 && N != 16 && N != 12 && N != 6) {
+    set_last_error("chunk_entries must be 6, 12, 16 or 32");
+    return nullptr;
+  }
+  if (key_range == 0 || key_range > 0xFFFFFFFEull) {
+    set_last_error("key_range must be in [1, 2^32-2]");
+    return nullptr;
+  }
+  if (capacity == 0) capacity = key_range;
+  if (cfg.contains_team == 0) cfg.contains_team = (N == 32 || N == 16) ? 8 : N;
+  if (!valid_team(N, cfg.contains_team)) {
+    set_last_error("unsupported contains_team for this chunk size");
+    return nullptr;
+  }
+  gfsl *h = new gfsl();
+  h->N = N;
+  h->team = cfg.contains_team;
+  h->cfg = cfg;
+  h->key_range = key_range;
+  auto fail = [&](const char *what, cudaError_t e) -> gfsl_t {
+    set_last_error(std::string(what) + ": " + cudaGetErrorString(e));
+    free_all(h);
+    return nullptr;
+  };
+  cudaError_t e;
+  if ((e = cudaGetDevice(&h->device)) != cudaSuccess) return fail("cudaGetDevice", e);
+  cudaDeviceGetAttribute(&h->sms, cudaDevAttrMultiProcessorCount, h->device);
+
+  // Pool sizing (R18): bottom = 2x the hard bound on live level-0 chunks
+  // ((capacity+1)/floor(DSIZE/3) + 1, from V13) plus slack; upper = bottom/8.
+  const uint64_t DS = N - 2;
+  const uint64_t m = std::max<uint64_t>(1, DS / 3);
+  uint64_t cap_b = 2 * ((capacity + 1) / m + 1) + 64;
+  uint64_t cap_u = cap_b / 8 + 2 * N + 64;
+  if (cap_b + cap_u >= 0xFFFFFFF0ull) {
+    free_all(h);
+    set_last_error("capacity too large for 32-bit chunk indices");
+    return nullptr;
+  }
+  h->d.cap_bottom = (uint32_t)cap_b;
+  h->d.cap_upper = (uint32_t)cap_u;
+  h->d.key_max = (uint32_t)key_range;
+  const uint64_t total_entries = (cap_b + cap_u) * N;
+  if ((e = cudaMalloc(&h->d.pool, total_entries * 8)) != cudaSuccess) return fail("cudaMalloc(pool)", e);
+  if ((e = cudaMalloc(&h->d.head, 32 * 4)) != cudaSuccess) return fail("cudaMalloc", e);
+  if ((e = cudaMalloc(&h->d.counter, 32 * 4)) != cudaSuccess) return fail("cudaMalloc", e);
+  if ((e = cudaMalloc(&h->d.bump, 2 * 4)) != cudaSuccess) return fail("cudaMalloc", e);
+  if ((e = cudaMalloc(&h->d.stats, ST_NSTATS * 8)) != cudaSuccess) return fail("cudaMalloc", e);
+  if ((e = cudaMalloc(&h->ctl, sizeof(BatchCtl))) != cudaSuccess) return fail("cudaMalloc", e);
+  if ((e = cudaHostAlloc(&h->h_error, 4, cudaHostAllocMapped)) != cudaSuccess) return fail("cudaHostAlloc", e);
+  *h->h_error = 0;
+  if ((e = cudaHostGetDevicePointer(&h->d.error, h->h_error, 0)) != cudaSuccess) return fail("cudaHostGetDevicePointer", e);
+  if ((e = cudaEventCreateWithFlags(&h->last, cudaEventDisableTiming)) != cudaSuccess) return fail("cudaEventCreate", e);
+  cudaMemset(h->d.head, 0xFF, 32 * 4);
+  cudaMemset(h->d.counter, 0, 32 * 4);
+  cudaMemset(h->d.stats, 0, ST_NSTATS * 8);
+  init_pool_kernel<<<h->sms * 8, 256>>>(h->d.pool, total_entries, N);
+  init_heads_kernel<<<1, 32>>>(h->d, N);
+  if ((e = cudaGetLastError()) != cudaSuccess) return fail("init kernels", e);
+  if ((e = cudaDeviceSynchronize()) != cudaSuccess) return fail("init sync", e);
+
+  int bc = contains_occupancy(N, h->team);
+  if (cfg.contains_blocks_per_sm) bc = std::min<int>(bc, cfg.contains_blocks_per_sm);
+  int bu = update_occupancy(N);
+  if (cfg.update_blocks_per_sm) bu = std::min<int>(bu, cfg.update_blocks_per_sm);
+  h->contains_grid = h->sms * std::max(1, bc);
+  h->update_grid = h->sms * std::max(1, bu);
+  return h;
+}
+
+extern "C" gfsl_t gfsl_create(uint64_t key_range, uint64_t capacity) {
+  return gfsl_create_ex(key_range, capacity, nullptr);
+}
+
+extern "C" void gfsl_destroy(gfsl_t h) {
+  if (!h) return;
+  cudaDeviceSynchronize();
+  free_all(h);
+}
+
+// ------------------------------------------------------------------------------------
+// batch
+
+static gfsl_status sticky(gfsl *h) {
+  if (h->sticky_cuda) return GFSL_ECUDA;
+  const uint32_t e = *(volatile uint32_t *)h->h_error;
+  if (e & ERR_POOL) {
+    set_last_error("chunk pool exhausted (sticky)");
+    return GFSL_EPOOL;
+  }
+  if (e & ERR_HANG) {
+    set_last_error("device watchdog fired: structure corrupt (sticky)");
+    h->sticky_cuda = true;
+    return GFSL_ECUDA;
+  }
+  return GFSL_OK;
+}
+
+static gfsl_status ensure_lists(gfsl *h, uint64_t n) {
+  if (n <= h->list_cap) return GFSL_OK;
+  cudaDeviceSynchronize();
+  cudaFree(h->list_c);
+  cudaFree(h->list_u);
+  h->list_c = h->list_u = nullptr;
+  h->list_cap = 0;
+  const uint64_t cap = std::max<uint64_t>(n, 1024);
+  CK(cudaMalloc(&h->list_c, cap * 4));
+  CK(cudaMalloc(&h->list_u, cap * 4));
+  h->list_cap = cap;
+  return GFSL_OK;
+}
+
+static gfsl_status enqueue_batch(gfsl *h, const uint8_t *ops, const uint32_t *keys,
+                                 const uint32_t *vals, uint8_t *res, uint64_t n, cudaStream_t s) {
+  CK(cudaStreamWaitEvent(s, h->last, 0));
+  CK(cudaMemsetAsync(h->ctl, 0, sizeof(BatchCtl), s));
+  const int cgrid = (int)std::min<uint64_t>((n + 255) / 256, (uint64_t)h->sms * 16);
+  classify_kernel<<<std::max(cgrid, 1), 256, 0, s>>>(ops, keys, res, (uint32_t)n, h->key_range,
+                                                    h->list_c, h->list_u, h->ctl);
+  bool ok = dispatch_contains(h, keys, res, s);
+  if (!ok) {
+    set_last_error("no contains kernel for this (N, team)");
+    return GFSL_EINVAL;
+  }
+  switch (h->N) {
+    case 32: launch_update<32>(h, ops, keys, vals, res, (uint32_t)n, s); break;
+    case 16: launch_update<16>(h, ops, keys, vals, res, (uint32_t)n, s); break;
+    case 12: launch_update<12>(h, ops, keys, vals, res, (uint32_t)n, s); break;
+    case 6: launch_update<6>(h, ops, keys, vals, res, (uint32_t)n, s); break;
+  }
+  cudaError_t e = cudaGetLastError();
+  if (e != cudaSuccess) {
+    h->sticky_cuda = true;
+    set_last_error(std::string("kernel launch: ") + cudaGetErrorString(e));
+    return GFSL_ECUDA;
+  }
+  CK(cudaEventRecord(h->last, s));
+  h->batches++;
+  h->ops += n;
+  return GFSL_OK;
+}
+
+extern "C" gfsl_status gfsl_batch(gfsl_t h, const uint8_t *op_types, const uint32_t *keys,
+                                  const uint32_t *values, uint8_t *results, uint64_t n,
+                                  void *stream) {
+  if (!h) {
+    set_last_error("NULL handle");
+    return GFSL_EINVAL;
+  }
+  gfsl_status st = sticky(h);
+  if (st != GFSL_OK) return st;
+  if (n == 0) return GFSL_OK;
+  if (!op_types || !keys || !results || n > 0xFFFFFFFFull) {
+    set_last_error("bad batch arguments");
+    return GFSL_EINVAL;
+  }
+  if ((st = ensure_lists(h, n)) != GFSL_OK) return st;
+  return enqueue_batch(h, op_types, keys, values, results, n, (cudaStream_t)stream);
+}
+
+extern "C" gfsl_status gfsl_batch_host(gfsl_t h, const uint8_t *op_types, const uint32_t *keys,
+                                       const uint32_t *values, uint8_t *results, uint64_t n,
+                                       void *stream) {
+  if (!h) {
+    set_last_error("NULL handle");
+    return GFSL_EINVAL;
+  }
+  gfsl_status st = sticky(h);
+  if (st != GFSL_OK) return st;
+  if (n == 0) return GFSL_OK;
+  if (!op_types || !keys || !results || n > 0xFFFFFFFFull) {
+    set_last_error("bad batch arguments");
+    return GFSL_EINVAL;
+  }
+  if (n > h->st_cap) {
+    cudaDeviceSynchronize();
+    cudaFree(h->st_op);
+    cudaFree(h->st_res);
+    cudaFree(h->st_key);
+    cudaFree(h->st_val);
+    h->st_op = h->st_res = nullptr;
+    h->st_key = h->st_val = nullptr;
+    h->st_cap = 0;
+    CK(cudaMalloc(&h->st_op, n));
+    CK(cudaMalloc(&h->st_res, n));
+    CK(cudaMalloc(&h->st_key, n * 4));
+    CK(cudaMalloc(&h->st_val, n * 4));
+    h->st_cap = n;
+  }
+  if ((st = ensure_lists(h, n)) != GFSL_OK) return st;
+  cudaStream_t s = (cudaStream_t)stream;
+  CK(cudaMemcpyAsync(h->st_op, op_types, n, cudaMemcpyHostToDevice, s));
+  CK(cudaMemcpyAsync(h->st_key, keys, n * 4, cudaMemcpyHostToDevice, s));
+  if (values) CK(cudaMemcpyAsync(h->st_val, values, n * 4, cudaMemcpyHostToDevice, s));
+  st = enqueue_batch(h, h->st_op, h->st_key, values ? h->st_val : nullptr, h->st_res, n, s);
+  if (st != GFSL_OK) return st;
+  CK(cudaMemcpyAsync(results, h->st_res, n, cudaMemcpyDeviceToHost, s));
+  CK(cudaStreamSynchronize(s));
+  return sticky(h);
+}
+
+extern "C" gfsl_status gfsl_get_stats(gfsl_t h, gfsl_stats *out) {
+  if (!h || !out) return GFSL_EINVAL;
+  unsigned long long s[ST_NSTATS];
+  CK(cudaDeviceSynchronize());
+  CK(cudaMemcpy(s, h->d.stats, sizeof(s), cudaMemcpyDeviceToHost));
+  memset(out, 0, sizeof(*out));
+  out->batches = h->batches;
+  out->ops = h->ops;
+  out->restarts = s[ST_RESTARTS];
+  out->splits = s[ST_SPLITS];
+  out->merges = s[ST_MERGES];
+  out->zombie_unlinks = s[ST_ZOMBIE_UNLINKS];
+  out->lock_retries = s[ST_LOCK_RETRIES];
+  return GFSL_OK;
+}
+
+// ------------------------------------------------------------------------------------
+// dump / load (test-only)
+
+static gfsl_status read_meta(gfsl *h, gfsl_meta *m) {
+  memset(m, 0, sizeof(*m));
+  uint32_t bump[2];
+  CK(cudaMemcpy(m->head, h->d.head, 32 * 4, cudaMemcpyDeviceToHost));
+  CK(cudaMemcpy(m->counters, h->d.counter, 32 * 4, cudaMemcpyDeviceToHost));
+  CK(cudaMemcpy(bump, h->d.bump, 8, cudaMemcpyDeviceToHost));
+  m->used_bottom = std::min(bump[0], h->d.cap_bottom);
+  m->used_upper = std::min(bump[1], h->d.cap_upper);
+  m->cap_bottom = h->d.cap_bottom;
+  m->cap_upper = h->d.cap_upper;
+  m->chunk_entries = h->N;
+  return GFSL_OK;
+}
+
+extern "C" gfsl_status gfsl_dump(gfsl_t h, gfsl_meta *meta, uint64_t *entries, uint64_t max_entries) {
+  if (!h) return GFSL_EINVAL;
+  CK(cudaDeviceSynchronize());
+  gfsl_meta m;
+  gfsl_status st = read_meta(h, &m);
+  if (st != GFSL_OK) return st;
+  if (meta) *meta = m;
+  if (entries) {
+    const uint64_t total = ((uint64_t)h->d.cap_bottom + h->d.cap_upper) * h->N;
+    CK(cudaMemcpy(entries, h->d.pool, std::min(total, max_entries) * 8, cudaMemcpyDeviceToHost));
+  }
+  return GFSL_OK;
+}
+
+extern "C" gfsl_status gfsl_load(gfsl_t h, const gfsl_meta *meta, const uint64_t *entries,
+                                 uint64_t n_entries) {
+  if (!h || !meta || !entries) return GFSL_EINVAL;
+  const uint64_t total = ((uint64_t)h->d.cap_bottom + h->d.cap_upper) * h->N;
+  if (n_entries != total || meta->chunk_entries != h->N || meta->cap_bottom != h->d.cap_bottom ||
+      meta->cap_upper != h->d.cap_upper) {
+    set_last_error("gfsl_load: image does not match the handle's pool geometry");
+    return GFSL_EINVAL;
+  }
+  CK(cudaDeviceSynchronize());
+  CK(cudaMemcpy(h->d.pool, entries, total * 8, cudaMemcpyHostToDevice));
+  CK(cudaMemcpy(h->d.head, meta->head, 32 * 4, cudaMemcpyHostToDevice));
+  CK(cudaMemcpy(h->d.counter, meta->counters, 32 * 4, cudaMemcpyHostToDevice));
+  uint32_t bump[2] = {meta->used_bottom, meta->used_upper};
+  CK(cudaMemcpy(h->d.bump, bump, 8, cudaMemcpyHostToDevice));
+  return GFSL_OK;
+}
+
+// ------------------------------------------------------------------------------------
+// validate (a6): copy the used part of the pool and walk it.  Invariants:
+//  V1 non-zombie chunks sorted, EMPTY grouped at the end
+//  V2 non-last chunk: max == largest key; last: max = next = inf
+//  V3 consecutive non-zombie chunks: max(c) < min(next)
+//  V4 level l+1 keys are a subset of level l keys
+//  V5 the down pointer of k at level l+1 reaches k laterally
+//  V7 no lock held at quiescence
+//  V8 the last chunk of a level is not a zombie
+//  V9 the head reaches a first non-zombie chunk holding -inf at index 0
+//  V10 keys are valid internal keys; -inf only first
+//  V12 every reachable chunk index is allocated
+//  V13 non-last non-zombie chunks hold >= floor(DSIZE/3) entries (derived)
+//  V14 counter[l] = #non-zombie chunks if level l holds a real key, else 0 (R9/R17)
+
+namespace {
+struct HostPool {
+  uint32_t N, cap_u, cap_b, used_u, used_b;
+  std::vector<uint64_t> up, bot;
+  bool allocated(uint32_t c) const {
+    if (c < cap_u) return c < used_u;
+    return c >= cap_u && (uint64_t)c < (uint64_t)cap_u + used_b;
+  }
+  const uint64_t *chunk(uint32_t c) const {
+    if (c < cap_u) return &up[(size_t)c * N];
+    return &bot[(size_t)(c - cap_u) * N];
+  }
+};
+inline uint32_t klo(uint64_t e) { return (uint32_t)e; }
+inline uint32_t khi(uint64_t e) { return (uint32_t)(e >> 32); }
+}  // namespace
+
+extern "C" gfsl_status gfsl_validate(gfsl_t h, gfsl_report *rep_out, uint32_t *keys_out,
+                                     uint32_t *vals_out, uint64_t cap, uint64_t *count) {
+  if (!h) return GFSL_EINVAL;
+  CK(cudaDeviceSynchronize());
+  gfsl_status st = sticky(h);
+  if (st != GFSL_OK) return st;
+  gfsl_meta m;
+  if ((st = read_meta(h, &m)) != GFSL_OK) return st;
+  HostPool P;
+  P.N = h->N;
+  P.cap_u = m.cap_upper;
+  P.cap_b = m.cap_bottom;
+  P.used_u = m.used_upper;
+  P.used_b = m.used_bottom;
+  P.up.resize((size_t)P.used_u * P.N);
+  P.bot.resize((size_t)P.used_b * P.N);
+  CK(cudaMemcpy(P.up.data(), h->d.pool, P.up.size() * 8, cudaMemcpyDeviceToHost));
+  CK(cudaMemcpy(P.bot.data(), h->d.pool + (size_t)P.cap_u * P.N, P.bot.size() * 8, cudaMemcpyDeviceToHost));
+
+  gfsl_report rep;
+  memset(&rep, 0, sizeof(rep));
+  const uint32_t N = P.N, DS = N - 2, NX = N - 2, LK = N - 1;
+  rep.chunk_entries = N;
+  uint32_t viol = 0;
+  auto V = [&](int v) { viol |= 1u << (v - 1); };
+  int height = 0;
+  for (uint32_t l = 1; l < N; ++l)
+    if (m.counters[l] > 0) height = (int)l;
+  rep.height = height;
+  for (uint32_t l = 0; l < N && l < 32; ++l) rep.counters[l] = m.counters[l];
+  rep.pool_used[0] = P.used_b;
+  rep.pool_used[1] = P.used_u;
+  rep.pool_cap[0] = P.cap_b;
+  rep.pool_cap[1] = P.cap_u;
+
+  // per level: ordered list of (non-zombie chunk index), and key -> chunk map (sorted)
+  std::vector<std::vector<uint32_t>> chunks(N);
+  std::vector<std::vector<std::pair<uint32_t, uint32_t>>> keymap(N);  // (key, value) per level
+  std::vector<std::vector<uint32_t>> keychunk(N);                     // chunk holding that key
+  const uint64_t step_cap = (uint64_t)P.used_u + P.used_b + 16;
+  for (uint32_t l = 0; l < N; ++l) {
+    uint32_t c = m.head[l];
+    bool seen_first = false;
+    uint64_t steps = 0;
+    uint32_t prev_max = 0;
+    bool have_prev = false;
+    while (c != NULL_CHUNK) {
+      if (!P.allocated(c) || ++steps > step_cap) {
+        V(12);
+        break;
+      }
+      const uint64_t *ch = P.chunk(c);
+      const uint32_t state = klo(ch[LK]);
+      const uint32_t next = khi(ch[NX]);
+      const uint32_t mx = klo(ch[NX]);
+      if (state == LOCK_ZOMBIE) {
+        rep.zombies[l]++;
+        if (next == NULL_CHUNK) V(8);
+        c = next;
+        continue;
+      }
+      if (state != LOCK_FREE) V(7);
+      rep.chunks[l]++;
+      chunks[l].push_back(c);
+      // V1 sortedness / EMPTY grouping; count
+      uint32_t cnt = 0;
+      bool empty_seen = false;
+      uint32_t last_key = 0;
+      for (uint32_t i = 0; i < DS; ++i) {
+        const uint32_t k = klo(ch[i]);
+        if (k == KEY_EMPTY) {
+          empty_seen = true;
+          if (ch[i] != EMPTY_ENTRY) V(1);
+          continue;
+        }
+        if (empty_seen) V(1);
+        if (cnt > 0 && k <= last_key) V(1);
+        if (k == KEY_NEG_INF) {
+          if (seen_first || i != 0) V(10);
+        } else {
+          if (k > h->d.key_max) V(10);
+          keymap[l].push_back({k, khi(ch[i])});
+          keychunk[l].push_back(c);
+        }
+        last_key = k;
+        ++cnt;
+      }
+      if (!seen_first) {
+        if (cnt == 0 || klo(ch[0]) != KEY_NEG_INF) V(9);
+      }
+      // V2
+      if (next == NULL_CHUNK) {
+        if (mx != KEY_POS_INF) V(2);
+      } else {
+        if (cnt == 0 || mx != last_key) V(2);
+        if (cnt < std::max<uint32_t>(1, DS / 3)) V(13);
+      }
+      // V3
+      if (have_prev && cnt > 0) {
+        const uint32_t first_real = klo(ch[0]);
+        if (!(prev_max < first_real)) V(3);
+      }
+      if (cnt > 0) {
+        prev_max = last_key;
+        have_prev = true;
+      }
+      seen_first = true;
+      c = next;
+    }
+    if (!seen_first) V(9);
+    rep.level_keys[l] = keymap[l].size();
+    // V14 counters
+    const int64_t expect = keymap[l].empty() ? 0 : (int64_t)rep.chunks[l];
+    if (N >= 12 && m.counters[l] != expect) V(14);
+    if (N < 12 && !keymap[l].empty() && m.counters[l] <= 0 && l >= 1) V(14);
+  }
+  // V4 + V5
+  for (uint32_t l = 0; l + 1 < N; ++l) {
+    const auto &lo = keymap[l];
+    const auto &up = keymap[l + 1];
+    for (size_t i = 0; i < up.size(); ++i) {
+      const uint32_t k = up[i].first;
+      auto it = std::lower_bound(lo.begin(), lo.end(), std::make_pair(k, 0u),
+                                 [](auto a, auto b) { return a.first < b.first; });
+      if (it == lo.end() || it->first != k) {
+        V(4);
+        continue;
+      }
+      const uint32_t target = keychunk[l][it - lo.begin()];
+      // walk laterally from the down pointer to the chunk holding k
+      uint32_t c = up[i].second;
+      uint64_t steps = 0;
+      bool ok = false;
+      while (c != NULL_CHUNK && P.allocated(c) && ++steps <= step_cap) {
+        if (c == target) {
+          ok = true;
+          break;
+        }
+        c = khi(P.chunk(c)[NX]);
+      }
+      if (!ok) V(5);
+    }
+  }
+  // the -inf down pointers must also reach the level below laterally
+  rep.keys = keymap[0].size();
+  rep.violations = viol;
+  for (int v = 1; v <= 32; ++v)
+    if (viol & (1u << (v - 1))) {
+      rep.first_violation = v;
+      break;
+    }
+  unsigned long long s[ST_NSTATS];
+  CK(cudaMemcpy(s, h->d.stats, sizeof(s), cudaMemcpyDeviceToHost));
+  rep.restarts = s[ST_RESTARTS];
+  if (rep_out) *rep_out = rep;
+  if (count) *count = rep.keys;
+  if (keys_out || vals_out) {
+    const uint64_t n = std::min<uint64_t>(cap, keymap[0].size());
+    for (uint64_t i = 0; i < n; ++i) {
+      if (keys_out) keys_out[i] = keymap[0][i].first - 1u;  // user key
+      if (vals_out) vals_out[i] = keymap[0][i].second;
+    }
+  }
+  if (viol) {
+    char buf[128];
+    snprintf(buf, sizeof(buf), "invariant violation mask 0x%x (first V%u)", viol, rep.first_violation);
+    set_last_error(buf);
+    return GFSL_ECORRUPT;
+  }
+  return GFSL_OK;
+}
+
+// ------------------------------------------------------------------------------------
+// multi-GPU routing (B5): stable partition of a batch by destination shard.
+
+constexpr int ROUTE_TILE = 1024;  // ops per block tile (256 threads x 4)
+constexpr int MAX_WORLD = 64;
+
+__device__ __forceinline__ uint32_t route_dest(uint8_t op, uint32_t key, uint64_t key_range,
+                                               uint64_t span, uint32_t world) {
+  if (op > 2 || (uint64_t)key >= key_range) return 0;
+  const uint64_t g = (uint64_t)key / span;
+  return (uint32_t)(g < world ? g : world - 1);
+}
+
+// pass 1: per-tile histogram -> tile_counts[tile * world + g]
+__global__ void route_hist_kernel(const uint8_t *ops, const uint32_t *keys, uint32_t n,
+                                  uint64_t key_range, uint64_t span, uint32_t world,
+                                  uint32_t *tile_counts) {
+  __shared__ uint32_t hist[MAX_WORLD];
+  for (uint32_t g = threadIdx.x; g < world; g += blockDim.x) hist[g] = 0;
+  __syncthreads();
+  const uint32_t base = blockIdx.x * ROUTE_TILE;
+  for (uint32_t i = base + threadIdx.x; i < min(n, base + ROUTE_TILE); i += blockDim.x)
+    atomicAdd(&hist[route_dest(ops[i], keys[i], key_range, span, world)], 1u);
+  __syncthreads();
+  for (uint32_t g = threadIdx.x; g < world; g += blockDim.x) tile_counts[blockIdx.x * world + g] = hist[g];
+}
+
+// pass 2 (one block): destination-major exclusive scan over tiles; counts[g] totals.
+__global__ void route_scan_kernel(uint32_t *tile_counts, uint32_t tiles, uint32_t world,
+                                  unsigned long long *counts) {
+  if (threadIdx.x != 0) return;
+  uint64_t run = 0;
+  for (uint32_t g = 0; g < world; ++g) {
+    uint64_t tot = 0;
+    for (uint32_t t = 0; t < tiles; ++t) {
+      const uint32_t c = tile_counts[t * world + g];
+      tile_counts[t * world + g] = (uint32_t)run;
+      run += c;
+      tot += c;
+    }
+    counts[g] = tot;
+  }
+}
+
+// pass 3: stable scatter of op indices; ranks within a tile follow input order.
+__global__ void route_scatter_kernel(const uint8_t *ops, const uint32_t *keys, uint32_t n,
+                                     uint64_t key_range, uint64_t span, uint32_t world,
+                                     const uint32_t *tile_offsets, uint32_t *perm) {
+  __shared__ uint32_t base_g[MAX_WORLD];
+  __shared__ uint32_t warp_counts[8][MAX_WORLD];
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  const uint32_t tile0 = blockIdx.x * ROUTE_TILE;
+  for (uint32_t g = threadIdx.x; g < world; g += blockDim.x) base_g[g] = tile_offsets[blockIdx.x * world + g];
+  // the tile is processed 256 consecutive ops at a time, in input order
+  for (uint32_t off = 0; off < ROUTE_TILE; off += 256) {
+    for (uint32_t x = threadIdx.x; x < 8 * MAX_WORLD; x += blockDim.x) (&warp_counts[0][0])[x] = 0;
+    __syncthreads();
+    const uint32_t i = tile0 + off + threadIdx.x;
+    const bool live = i < n;
+    const uint32_t g = live ? route_dest(ops[i], keys[i], key_range, span, world) : 0xFFFFFFFFu;
+    const uint32_t same = __match_any_sync(0xFFFFFFFFu, g);
+    if (live && lane == __ffs(same) - 1) warp_counts[warp][g] = __popc(same);
+    __syncthreads();
+    if (live) {
+      uint32_t pos = base_g[g];
+      for (int w = 0; w < warp; ++w) pos += warp_counts[w][g];
+      pos += __popc(same & ((1u << lane) - 1u));
+      perm[pos] = i;
+    }
+    __syncthreads();
+    for (uint32_t d = threadIdx.x; d < world; d += blockDim.x) {
+      uint32_t t = 0;
+      for (int w = 0; w < 8; ++w) t += warp_counts[w][d];
+      base_g[d] += t;
+    }
+    __syncthreads();
+  }
+}
+
+__global__ void route_pack_kernel(const uint32_t *perm, const uint8_t *ops, const uint32_t *keys,
+                                  const uint32_t *vals, uint32_t n, uint8_t *so, uint32_t *sk,
+                                  uint32_t *sv) {
+  for (uint32_t j = blockIdx.x * blockDim.x + threadIdx.x; j < n; j += gridDim.x * blockDim.x) {
+    const uint32_t i = perm[j];
+    so[j] = ops[i];
+    sk[j] = keys[i];
+    sv[j] = vals ? vals[i] : 0u;
+  }
+}
+
+__global__ void route_unpack_kernel(const uint32_t *perm, const uint8_t *rr, uint32_t n, uint8_t *res) {
+  for (uint32_t j = blockIdx.x * blockDim.x + threadIdx.x; j < n; j += gridDim.x * blockDim.x)
+    res[perm[j]] = rr[j];
+}
+
+extern "C" gfsl_status gfsl_route_plan(const uint8_t *op_types, const uint32_t *keys, uint64_t n,
+                                       uint64_t key_range, uint32_t world, uint64_t *counts,
+                                       uint32_t *perm, void *stream) {
+  if (world == 0 || world > MAX_WORLD || n > 0xFFFFFFFFull || !counts || (n && (!op_types || !keys || !perm))) {
+    set_last_error("gfsl_route_plan: bad arguments");
+    return GFSL_EINVAL;
+  }
+  cudaStream_t s = (cudaStream_t)stream;
+  if (n == 0) {
+    CK(cudaMemsetAsync(counts, 0, world * 8, s));
+    return GFSL_OK;
+  }
+  const uint64_t span = (key_range + world - 1) / world;
+  const uint32_t tiles = (uint32_t)((n + ROUTE_TILE - 1) / ROUTE_TILE);
+  uint32_t *tile_counts = nullptr;
+  CK(cudaMallocAsync(&tile_counts, (size_t)tiles * world * 4, s));
+  route_hist_kernel<<<tiles, 256, 0, s>>>(op_types, keys, (uint32_t)n, key_range, span, world, tile_counts);
+  route_scan_kernel<<<1, 32, 0, s>>>(tile_counts, tiles, world, (unsigned long long *)counts);
+  route_scatter_kernel<<<tiles, 256, 0, s>>>(op_types, keys, (uint32_t)n, key_range, span, world,
+                                             tile_counts, perm);
+  CK(cudaFreeAsync(tile_counts, s));
+  CK(cudaGetLastError());
+  return GFSL_OK;
+}
+
+extern "C" gfsl_status gfsl_route_pack(const uint32_t *perm, const uint8_t *op_types,
+                                       const uint32_t *keys, const uint32_t *values, uint64_t n,
+                                       uint8_t *send_op, uint32_t *send_key, uint32_t *send_val,
+                                       void *stream) {
+  if (n > 0xFFFFFFFFull) return GFSL_EINVAL;
+  if (n == 0) return GFSL_OK;
+  const int grid = (int)std::min<uint64_t>((n + 255) / 256, 148 * 16);
+  route_pack_kernel<<<grid, 256, 0, (cudaStream_t)stream>>>(perm, op_types, keys, values, (uint32_t)n,
+                                                            send_op, send_key, send_val);
+  CK(cudaGetLastError());
+  return GFSL_OK;
+}
+
+extern "C" gfsl_status gfsl_route_unpack(const uint32_t *perm, const uint8_t *recv_res, uint64_t n,
+                                         uint8_t *results, void *stream) {
+  if (n > 0xFFFFFFFFull) return GFSL_EINVAL;
+  if (n == 0) return GFSL_OK;
+  const int grid = (int)std::min<uint64_t>((n + 255) / 256, 148 * 16);
+  route_unpack_kernel<<<grid, 256, 0, (cudaStream_t)stream>>>(perm, recv_res, (uint32_t)n, results);
+  CK(cudaGetLastError());
+  return GFSL_OK;
+}

@@ -1,0 +1,141 @@
+// gfsl_device.cuh -- chunk layout, sentinels and memory primitives of the GFSL device path.
+//
+// Chunk layout (Fig 3.1; §4.1): a chunk is N 8-byte entries.
+//   entries 0..N-3  DATA  {lo32 key, hi32 value}      (value = down pointer above level 0)
+//   entry   N-2     NEXT  {lo32 max field, hi32 next chunk index}
+//   entry   N-1     LOCK  {lo32 lock state, hi32 version}
+// Chunks live in one pre-allocated pool and are named by 32-bit indices.
+// Sentinels (reading R3): internal key = user key + 1, so that
+//   -inf = 0, +inf = EMPTY = 0xFFFFFFFF, null pointer = 0xFFFFFFFF.
+// Lock states (reading R4): 0 unlocked, 1 locked, 2 zombie; the upper 32 bits are
+// a version bumped by every unlock, which lets a reader prove that a lock-free read of a
+// chunk was not torn by a writer (used where a NEGATIVE answer must be exact).
+#pragma once
+#include <cstdint>
+
+namespace gfsl_dev {
+
+constexpr uint32_t KEY_NEG_INF = 0u;
+constexpr uint32_t KEY_POS_INF = 0xFFFFFFFFu;
+constexpr uint32_t KEY_EMPTY = 0xFFFFFFFFu;
+constexpr uint32_t NULL_CHUNK = 0xFFFFFFFFu;
+constexpr uint64_t EMPTY_ENTRY = 0xFFFFFFFFFFFFFFFFull;
+
+constexpr uint32_t LOCK_FREE = 0u;
+constexpr uint32_t LOCK_HELD = 1u;
+constexpr uint32_t LOCK_ZOMBIE = 2u;
+
+constexpr int MAX_N = 32;
+
+// error word bits (sticky)
+constexpr uint32_t ERR_POOL = 1u;     // chunk pool exhausted
+constexpr uint32_t ERR_HANG = 2u;     // a watchdog fired (corrupt structure / livelock)
+
+// statistics slots
+enum StatSlot {
+  ST_RESTARTS = 0, ST_SPLITS, ST_MERGES, ST_ZOMBIE_UNLINKS, ST_LOCK_RETRIES, ST_NSTATS
+};
+
+// Device view of one handle.
+struct DevState {
+  uint64_t *pool;        // (cap_upper + cap_bottom) * N entries
+  uint32_t *head;        // head[MAX_N]
+  int32_t *counter;      // counter[MAX_N] "utilized chunks" per level
+  uint32_t *bump;        // bump[0] bottom pool used, bump[1] upper pool used
+  uint32_t *error;       // sticky error word (mapped host memory)
+  unsigned long long *stats;
+  uint32_t cap_bottom;   // bottom-pool chunks, indices [cap_upper, cap_upper + cap_bottom)
+  uint32_t cap_upper;    // upper-pool chunks, indices [0, cap_upper)
+  uint32_t key_max;      // largest valid internal key (= key_range)
+};
+
+// Per-batch control block (device memory, zeroed before every batch).
+struct BatchCtl {
+  uint32_t n_contains;
+  uint32_t n_updates;
+  uint32_t next_update;  // dynamic work counter of the update kernel
+  uint32_t pad;
+};
+
+__device__ __forceinline__ uint32_t lo32(uint64_t x) { return (uint32_t)x; }
+__device__ __forceinline__ uint32_t hi32(uint64_t x) { return (uint32_t)(x >> 32); }
+__device__ __forceinline__ uint64_t mk64(uint32_t lo, uint32_t hi) {
+  return (uint64_t)lo | ((uint64_t)hi << 32);
+}
+
+// ---- loads -------------------------------------------------------------------------
+// Update phase: chunks are written concurrently, so every read goes to L2 (relaxed, gpu
+// scope; never a stale L1 line).
+__device__ __forceinline__ uint64_t ld_relaxed(const uint64_t *p) {
+  uint64_t v;
+  asm volatile("ld.relaxed.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+  return v;
+}
+__device__ __forceinline__ uint64_t ld_acquire(const uint64_t *p) {
+  uint64_t v;
+  asm volatile("ld.acquire.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+  return v;
+}
+__device__ __forceinline__ uint32_t ld_relaxed32(const uint32_t *p) {
+  uint32_t v;
+  asm volatile("ld.relaxed.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+  return v;
+}
+__device__ __forceinline__ int32_t ld_relaxed_s32(const int32_t *p) {
+  int32_t v;
+  asm volatile("ld.relaxed.gpu.global.s32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+  return v;
+}
+__device__ __forceinline__ void st_relaxed(uint64_t *p, uint64_t v) {
+  asm volatile("st.relaxed.gpu.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
+
+// Contains phase: the structure is read-only for the whole kernel (S1), so the
+// non-coherent read-only path (L1-allocating) is legal and lets hot upper-level chunks
+// hit in L1.  One vector load per lane; EPL entries per lane.
+template <int EPL>
+struct ChunkSlice {
+  uint32_t k[EPL];
+  uint32_t v[EPL];
+};
+
+template <int EPL>
+__device__ __forceinline__ void ld_slice_nc(const uint64_t *p, ChunkSlice<EPL> &s);
+
+template <>
+__device__ __forceinline__ void ld_slice_nc<1>(const uint64_t *p, ChunkSlice<1> &s) {
+  asm volatile("ld.global.nc.v2.u32 {%0,%1}, [%2];" : "=r"(s.k[0]), "=r"(s.v[0]) : "l"(p));
+}
+template <>
+__device__ __forceinline__ void ld_slice_nc<2>(const uint64_t *p, ChunkSlice<2> &s) {
+  asm volatile("ld.global.nc.v4.u32 {%0,%1,%2,%3}, [%4];"
+               : "=r"(s.k[0]), "=r"(s.v[0]), "=r"(s.k[1]), "=r"(s.v[1])
+               : "l"(p));
+}
+template <>
+__device__ __forceinline__ void ld_slice_nc<4>(const uint64_t *p, ChunkSlice<4> &s) {
+  asm volatile("ld.global.nc.v8.u32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];"
+               : "=r"(s.k[0]), "=r"(s.v[0]), "=r"(s.k[1]), "=r"(s.v[1]), "=r"(s.k[2]),
+                 "=r"(s.v[2]), "=r"(s.k[3]), "=r"(s.v[3])
+               : "l"(p));
+}
+template <>
+__device__ __forceinline__ void ld_slice_nc<8>(const uint64_t *p, ChunkSlice<8> &s) {
+  asm volatile("ld.global.nc.v8.u32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];"
+               : "=r"(s.k[0]), "=r"(s.v[0]), "=r"(s.k[1]), "=r"(s.v[1]), "=r"(s.k[2]),
+                 "=r"(s.v[2]), "=r"(s.k[3]), "=r"(s.v[3])
+               : "l"(p));
+  asm volatile("ld.global.nc.v8.u32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];"
+               : "=r"(s.k[4]), "=r"(s.v[4]), "=r"(s.k[5]), "=r"(s.v[5]), "=r"(s.k[6]),
+                 "=r"(s.v[6]), "=r"(s.k[7]), "=r"(s.v[7])
+               : "l"(p + 4));
+}
+
+__device__ __forceinline__ void set_error(const DevState &d, uint32_t bit) {
+  atomicOr(d.error, bit);
+}
+__device__ __forceinline__ void stat_add(const DevState &d, int slot, unsigned long long v = 1) {
+  atomicAdd(d.stats + slot, v);
+}
+
+}  // namespace gfsl_dev

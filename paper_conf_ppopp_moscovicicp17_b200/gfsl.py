@@ -1,0 +1,284 @@
+"""Thin Python binding of libgfsl (include/gfsl.h) -- argument marshalling only.
+
+Every step of a batch runs in the sm_100a kernels of ``csrc/``; this module passes
+device pointers, sizes and the current CUDA stream through the C ABI.  There is no CPU
+fallback: if ``libgfsl.so`` is missing or no CUDA device is present, constructing a
+``GFSL`` raises.
+
+Tensors: op types ``uint8``; keys/values 32-bit (``int32`` or ``uint32`` tensors, read as
+uint32 bit patterns); results ``uint8`` (0 false, 1 true, 0xFF invalid).
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+from dataclasses import dataclass
+
+import numpy as np
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_HERE, "libgfsl.so")
+
+GFSL_OK, GFSL_EINVAL, GFSL_ENOMEM, GFSL_EPOOL, GFSL_ECUDA, GFSL_ECORRUPT = range(6)
+CONTAINS, INSERT, DELETE = 0, 1, 2
+RES_FALSE, RES_TRUE, RES_INVALID = 0, 1, 0xFF
+STATUS_NAMES = ["OK", "EINVAL", "ENOMEM", "EPOOL", "ECUDA", "ECORRUPT"]
+
+
+class gfsl_config(ctypes.Structure):
+    _fields_ = [("chunk_entries", ctypes.c_uint32), ("contains_team", ctypes.c_uint32),
+                ("contains_blocks_per_sm", ctypes.c_uint32),
+                ("update_blocks_per_sm", ctypes.c_uint32),
+                ("serial_updates", ctypes.c_uint32), ("reserved", ctypes.c_uint32 * 3)]
+
+
+class gfsl_report(ctypes.Structure):
+    _fields_ = [("keys", ctypes.c_uint64), ("height", ctypes.c_uint32),
+                ("chunk_entries", ctypes.c_uint32), ("chunks", ctypes.c_uint64 * 32),
+                ("zombies", ctypes.c_uint64 * 32), ("level_keys", ctypes.c_uint64 * 32),
+                ("counters", ctypes.c_int64 * 32), ("pool_used", ctypes.c_uint64 * 2),
+                ("pool_cap", ctypes.c_uint64 * 2), ("violations", ctypes.c_uint32),
+                ("first_violation", ctypes.c_uint32), ("restarts", ctypes.c_uint64),
+                ("reserved", ctypes.c_uint64 * 4)]
+
+
+class gfsl_stats(ctypes.Structure):
+    _fields_ = [("batches", ctypes.c_uint64), ("ops", ctypes.c_uint64),
+                ("restarts", ctypes.c_uint64), ("splits", ctypes.c_uint64),
+                ("merges", ctypes.c_uint64), ("zombie_unlinks", ctypes.c_uint64),
+                ("lock_retries", ctypes.c_uint64), ("reserved", ctypes.c_uint64 * 8)]
+
+
+class gfsl_meta(ctypes.Structure):
+    _fields_ = [("head", ctypes.c_uint32 * 32), ("counters", ctypes.c_int32 * 32),
+                ("used_bottom", ctypes.c_uint32), ("used_upper", ctypes.c_uint32),
+                ("cap_bottom", ctypes.c_uint32), ("cap_upper", ctypes.c_uint32),
+                ("chunk_entries", ctypes.c_uint32), ("reserved", ctypes.c_uint32 * 3)]
+
+
+# Every symbol include/gfsl.h declares (checked by tests/test_abi.py).
+EXPORTS = [
+    "gfsl_create", "gfsl_create_ex", "gfsl_destroy", "gfsl_batch", "gfsl_batch_host",
+    "gfsl_validate", "gfsl_last_error", "gfsl_get_stats", "gfsl_dump", "gfsl_load",
+    "gfsl_route_plan", "gfsl_route_pack", "gfsl_route_unpack",
+]
+
+_lib = None
+
+
+def load_library(path: str = LIB_PATH):
+    """Load libgfsl.so and declare the C signatures.  Raises if it is missing."""
+    global _lib
+    if _lib is not None:
+        return _lib
+    if not os.path.exists(path):
+        raise RuntimeError(
+            f"{path} is missing: build it with `python -m paper_conf_ppopp_moscovicicp17_b200.build`"
+            " (there is no CPU fallback)")
+    lib = ctypes.CDLL(path)
+    vp, u64, u32, i32 = ctypes.c_void_p, ctypes.c_uint64, ctypes.c_uint32, ctypes.c_int
+    lib.gfsl_create.restype = vp
+    lib.gfsl_create.argtypes = [u64, u64]
+    lib.gfsl_create_ex.restype = vp
+    lib.gfsl_create_ex.argtypes = [u64, u64, ctypes.POINTER(gfsl_config)]
+    lib.gfsl_destroy.restype = None
+    lib.gfsl_destroy.argtypes = [vp]
+    lib.gfsl_batch.restype = i32
+    lib.gfsl_batch.argtypes = [vp, vp, vp, vp, vp, u64, vp]
+    lib.gfsl_batch_host.restype = i32
+    lib.gfsl_batch_host.argtypes = [vp, vp, vp, vp, vp, u64, vp]
+    lib.gfsl_validate.restype = i32
+    lib.gfsl_validate.argtypes = [vp, ctypes.POINTER(gfsl_report), vp, vp, u64,
+                                  ctypes.POINTER(u64)]
+    lib.gfsl_last_error.restype = ctypes.c_char_p
+    lib.gfsl_last_error.argtypes = []
+    lib.gfsl_get_stats.restype = i32
+    lib.gfsl_get_stats.argtypes = [vp, ctypes.POINTER(gfsl_stats)]
+    lib.gfsl_dump.restype = i32
+    lib.gfsl_dump.argtypes = [vp, ctypes.POINTER(gfsl_meta), vp, u64]
+    lib.gfsl_load.restype = i32
+    lib.gfsl_load.argtypes = [vp, ctypes.POINTER(gfsl_meta), vp, u64]
+    lib.gfsl_route_plan.restype = i32
+    lib.gfsl_route_plan.argtypes = [vp, vp, u64, u64, u32, vp, vp, vp]
+    lib.gfsl_route_pack.restype = i32
+    lib.gfsl_route_pack.argtypes = [vp, vp, vp, vp, u64, vp, vp, vp, vp]
+    lib.gfsl_route_unpack.restype = i32
+    lib.gfsl_route_unpack.argtypes = [vp, vp, u64, vp, vp]
+    _lib = lib
+    return lib
+
+
+class GFSLError(RuntimeError):
+    def __init__(self, status: int, what: str):
+        self.status = status
+        name = STATUS_NAMES[status] if 0 <= status < len(STATUS_NAMES) else str(status)
+        super().__init__(f"{what}: GFSL_{name}: {load_library().gfsl_last_error().decode()}")
+
+
+def _check(status: int, what: str):
+    if status != GFSL_OK:
+        raise GFSLError(status, what)
+
+
+def _ptr(t) -> int | None:
+    return None if t is None else t.data_ptr()
+
+
+def _stream(stream) -> int | None:
+    import torch
+    if stream is None:
+        stream = torch.cuda.current_stream()
+    return stream.cuda_stream
+
+
+@dataclass
+class Report:
+    keys: int
+    height: int
+    chunks: list
+    zombies: list
+    level_keys: list
+    counters: list
+    pool_used: tuple
+    pool_cap: tuple
+    violations: int
+    first_violation: int
+    restarts: int
+
+
+class GFSL:
+    """One GFSL map on the current CUDA device (C handle ``gfsl_t``)."""
+
+    def __init__(self, key_range: int, capacity: int = 0, chunk_entries: int = 32,
+                 contains_team: int = 0, serial_updates: bool = False,
+                 contains_blocks_per_sm: int = 0, update_blocks_per_sm: int = 0):
+        import torch
+        if not torch.cuda.is_available():
+            raise RuntimeError("GFSL needs a CUDA device (there is no CPU fallback)")
+        self.lib = load_library()
+        cfg = gfsl_config(chunk_entries, contains_team, contains_blocks_per_sm,
+                          update_blocks_per_sm, 1 if serial_updates else 0)
+        self.key_range = int(key_range)
+        self.chunk_entries = int(chunk_entries)
+        self.h = self.lib.gfsl_create_ex(self.key_range, int(capacity), ctypes.byref(cfg))
+        if not self.h:
+            raise RuntimeError("gfsl_create failed: " + self.lib.gfsl_last_error().decode())
+
+    def close(self):
+        if getattr(self, "h", None):
+            self.lib.gfsl_destroy(self.h)
+            self.h = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+    # ---- batches -------------------------------------------------------------------
+    def batch(self, op, key, val=None, out=None, stream=None):
+        """Asynchronous batch on device tensors; returns the uint8 result tensor."""
+        import torch
+        n = op.numel()
+        assert op.dtype == torch.uint8 and op.is_cuda and op.is_contiguous()
+        assert key.numel() == n and key.element_size() == 4 and key.is_cuda and key.is_contiguous()
+        if val is not None:
+            assert val.numel() == n and val.element_size() == 4 and val.is_cuda and val.is_contiguous()
+        if out is None:
+            out = torch.empty(n, dtype=torch.uint8, device=op.device)
+        _check(self.lib.gfsl_batch(self.h, _ptr(op), _ptr(key), _ptr(val), _ptr(out), n,
+                                   _stream(stream)), "gfsl_batch")
+        return out
+
+    def batch_host(self, op, key, val=None, out=None, stream=None):
+        """Synchronous batch on HOST tensors (the end-to-end entry point)."""
+        import torch
+        n = op.numel()
+        assert not op.is_cuda and op.dtype == torch.uint8 and op.is_contiguous()
+        assert not key.is_cuda and key.element_size() == 4 and key.is_contiguous()
+        if out is None:
+            out = torch.empty(n, dtype=torch.uint8, pin_memory=op.is_pinned())
+        _check(self.lib.gfsl_batch_host(self.h, _ptr(op), _ptr(key), _ptr(val), _ptr(out), n,
+                                        _stream(stream)), "gfsl_batch_host")
+        return out
+
+    # ---- inspection ----------------------------------------------------------------
+    def validate(self, export: bool = True, raise_on_violation: bool = True):
+        rep = gfsl_report()
+        cnt = ctypes.c_uint64()
+        st = self.lib.gfsl_validate(self.h, ctypes.byref(rep), None, None, 0, ctypes.byref(cnt))
+        if st not in (GFSL_OK, GFSL_ECORRUPT):
+            _check(st, "gfsl_validate")
+        keys = vals = None
+        if export and st == GFSL_OK:
+            n = cnt.value
+            keys = np.empty(n, dtype=np.uint32)
+            vals = np.empty(n, dtype=np.uint32)
+            st = self.lib.gfsl_validate(self.h, None, keys.ctypes.data, vals.ctypes.data, n, None)
+        report = Report(rep.keys, rep.height, list(rep.chunks), list(rep.zombies),
+                        list(rep.level_keys), list(rep.counters), tuple(rep.pool_used),
+                        tuple(rep.pool_cap), rep.violations, rep.first_violation, rep.restarts)
+        if st == GFSL_ECORRUPT and raise_on_violation:
+            raise GFSLError(st, f"gfsl_validate (violations=0x{rep.violations:x})")
+        return report, keys, vals
+
+    def stats(self) -> dict:
+        s = gfsl_stats()
+        _check(self.lib.gfsl_get_stats(self.h, ctypes.byref(s)), "gfsl_get_stats")
+        return {f: getattr(s, f) for f, _ in gfsl_stats._fields_ if f != "reserved"}
+
+    def dump(self):
+        """(meta dict, entries uint64 array of shape [chunks, N]) -- test-only."""
+        m = gfsl_meta()
+        _check(self.lib.gfsl_dump(self.h, ctypes.byref(m), None, 0), "gfsl_dump")
+        total = (m.cap_bottom + m.cap_upper) * m.chunk_entries
+        ent = np.empty(total, dtype=np.uint64)
+        _check(self.lib.gfsl_dump(self.h, ctypes.byref(m), ent.ctypes.data, total), "gfsl_dump")
+        meta = dict(head=list(m.head), counters=list(m.counters), used_bottom=m.used_bottom,
+                    used_upper=m.used_upper, cap_bottom=m.cap_bottom, cap_upper=m.cap_upper,
+                    chunk_entries=m.chunk_entries)
+        return meta, ent.reshape(-1, m.chunk_entries)
+
+    def load(self, meta: dict, entries: np.ndarray):
+        m = gfsl_meta()
+        for i, v in enumerate(meta["head"]):
+            m.head[i] = v
+        for i, v in enumerate(meta["counters"]):
+            m.counters[i] = v
+        m.used_bottom, m.used_upper = meta["used_bottom"], meta["used_upper"]
+        m.cap_bottom, m.cap_upper = meta["cap_bottom"], meta["cap_upper"]
+        m.chunk_entries = meta["chunk_entries"]
+        ent = np.ascontiguousarray(entries, dtype=np.uint64).reshape(-1)
+        _check(self.lib.gfsl_load(self.h, ctypes.byref(m), ent.ctypes.data, ent.size), "gfsl_load")
+
+
+# ---- multi-GPU routing primitives (B5) ------------------------------------------------
+def route_plan(op, key, key_range: int, world: int, stream=None):
+    """Returns (counts int64[world] on device, perm int32[n] on device)."""
+    import torch
+    lib = load_library()
+    n = op.numel()
+    counts = torch.empty(world, dtype=torch.int64, device=op.device)
+    perm = torch.empty(n, dtype=torch.int32, device=op.device)
+    _check(lib.gfsl_route_plan(_ptr(op), _ptr(key), n, key_range, world, _ptr(counts),
+                               _ptr(perm), _stream(stream)), "gfsl_route_plan")
+    return counts, perm
+
+
+def route_pack(perm, op, key, val, stream=None):
+    import torch
+    lib = load_library()
+    n = op.numel()
+    so = torch.empty_like(op)
+    sk = torch.empty_like(key)
+    sv = torch.empty(n, dtype=key.dtype, device=op.device)
+    _check(lib.gfsl_route_pack(_ptr(perm), _ptr(op), _ptr(key), _ptr(val), n, _ptr(so),
+                               _ptr(sk), _ptr(sv), _stream(stream)), "gfsl_route_pack")
+    return so, sk, sv
+
+
+def route_unpack(perm, recv_res, out, stream=None):
+    lib = load_library()
+    _check(lib.gfsl_route_unpack(_ptr(perm), _ptr(recv_res), recv_res.numel(), _ptr(out),
+                                 _stream(stream)), "gfsl_route_unpack")
+    return out

@@ -1,0 +1,178 @@
+"""GPU parity: the CUDA path (through the C ABI) vs Oracle-A, element by element.
+
+Every test runs seeded batches through ``gfsl_batch`` and through the oracle on the same
+inputs, compares every per-op result bit-exactly, and after every batch checks the
+structural invariants (``gfsl_validate``) and that the exported (key, value) set equals
+the oracle's.  Sizes span many chunks and levels plus ragged tails.
+"""
+import numpy as np
+import pytest
+import torch
+
+from oracle.oracle_a import OracleMap
+from paper_conf_ppopp_moscovicicp17_b200.gfsl import GFSL
+from paper_conf_ppopp_moscovicicp17_b200.workload import (
+    SEED_BASE, Workload, prefill_keys, prefill_values)
+
+pytestmark = pytest.mark.gpu
+
+
+def to_dev(op, key, val):
+    dev = torch.device("cuda")
+    op_d = torch.as_tensor(np.ascontiguousarray(op, np.uint8)).to(dev)
+    key_d = torch.as_tensor(np.ascontiguousarray(key, np.uint32).view(np.int32)).to(dev)
+    val_d = None if val is None else torch.as_tensor(
+        np.ascontiguousarray(val, np.uint32).view(np.int32)).to(dev)
+    return op_d, key_d, val_d
+
+
+def check_same_set(g: GFSL, o: OracleMap):
+    rep, ks, vs = g.validate()
+    ok, ov = o.export()
+    assert rep.violations == 0
+    assert rep.keys == len(o)
+    assert np.array_equal(ks, ok)
+    assert np.array_equal(vs, ov)
+    return rep
+
+
+def run_batch(g, o, op, key, val):
+    r_gpu = g.batch(*to_dev(op, key, val)).cpu().numpy()
+    torch.cuda.synchronize()
+    r_ora = o.batch(op, key, val)
+    mism = np.flatnonzero(r_gpu != r_ora)
+    assert mism.size == 0, f"{mism.size} mismatches, first at {mism[:5]}: gpu={r_gpu[mism[:5]]} oracle={r_ora[mism[:5]]} op={op[mism[:5]]} key={key[mism[:5]]}"
+    return r_gpu
+
+
+def prefill(g, o, R, count, seed=SEED_BASE, chunk=1 << 20):
+    for s in range(0, count, chunk):
+        c = min(chunk, count - s)
+        k = prefill_keys(seed, R, c, start=s)
+        v = prefill_values(seed, k)
+        op = np.ones(c, np.uint8)
+        run_batch(g, o, op, k.numpy().astype(np.uint32), v.numpy().astype(np.uint32))
+
+
+def workload_batches(R, B, nb, mix, dist="uniform", seed=SEED_BASE + 1):
+    w = Workload(R, B, mix=mix, dist=dist, seed=seed)
+    for b in range(nb):
+        op, key, val, _ = w.make_batch(b)
+        yield op.numpy(), key.numpy().astype(np.uint32), val.numpy().astype(np.uint32)
+
+
+@pytest.mark.parametrize("N,team", [(32, 8), (32, 16), (32, 32), (16, 4), (16, 8), (16, 16)])
+def test_mixed_batches(N, team):
+    R = 20_000
+    g = GFSL(R, chunk_entries=N, contains_team=team)
+    o = OracleMap(R)
+    prefill(g, o, R, R // 2)
+    check_same_set(g, o)
+    for op, key, val in workload_batches(R, 4_000 + 37, 6, (20, 20, 60)):
+        run_batch(g, o, op, key, val)
+        check_same_set(g, o)
+
+
+@pytest.mark.parametrize("N", [32, 16, 12, 6])
+def test_serial_mode_churn(N):
+    """One team applies the updates in op order: the deterministic mode."""
+    R = 3_000
+    g = GFSL(R, chunk_entries=N, serial_updates=True)
+    o = OracleMap(R)
+    prefill(g, o, R, R // 2)
+    check_same_set(g, o)
+    for op, key, val in workload_batches(R, 1_500, 8, (30, 30, 40)):
+        run_batch(g, o, op, key, val)
+        check_same_set(g, o)
+
+
+@pytest.mark.parametrize("N", [32, 16])
+def test_heavy_churn_small_range(N):
+    """Tiny key range, 50/50 updates: contention, splits, merges and zombies everywhere."""
+    R = 600
+    g = GFSL(R, chunk_entries=N)
+    o = OracleMap(R)
+    for op, key, val in workload_batches(R, 300, 40, (50, 50, 0)):
+        run_batch(g, o, op, key, val)
+        check_same_set(g, o)
+    st = g.stats()
+    assert st["splits"] > 0 and st["merges"] > 0
+
+
+@pytest.mark.parametrize("N", [32, 16])
+def test_fill_then_drain(N):
+    """Insert-only of every key from empty, then Delete-only of every key."""
+    R = 50_000
+    g = GFSL(R, chunk_entries=N)
+    o = OracleMap(R)
+    perm = np.random.default_rng(5).permutation(R).astype(np.uint32)
+    for s in range(0, R, 12_345):
+        k = perm[s:s + 12_345]
+        run_batch(g, o, np.ones(k.size, np.uint8), k, k * 3)
+    rep = check_same_set(g, o)
+    assert rep.keys == R and rep.height >= 2
+    perm2 = np.random.default_rng(6).permutation(R).astype(np.uint32)
+    for s in range(0, R, 9_999):
+        k = perm2[s:s + 9_999]
+        run_batch(g, o, np.full(k.size, 2, np.uint8), k, None)
+        check_same_set(g, o)
+    rep = check_same_set(g, o)
+    assert rep.keys == 0
+
+
+def test_edge_cases():
+    R = 1000
+    g = GFSL(R)
+    o = OracleMap(R)
+    # empty batch
+    out = g.batch(*to_dev(np.zeros(0, np.uint8), np.zeros(0, np.uint32), None))
+    assert out.numel() == 0
+    # everything on an empty map
+    run_batch(g, o, np.array([0, 2, 1, 0], np.uint8), np.array([5, 5, 7, 7], np.uint32),
+              np.array([0, 0, 9, 0], np.uint32))
+    # invalid op codes and keys >= key_range get 0xFF and change nothing
+    op = np.array([3, 255, 1, 0, 2, 1], np.uint8)
+    key = np.array([1, 2, R, R + 5, 0xFFFFFFFF, 999], np.uint32)
+    r = run_batch(g, o, op, key, np.arange(6, dtype=np.uint32))
+    assert r.tolist() == [255, 255, 255, 255, 255, 1]
+    # largest and smallest valid keys
+    run_batch(g, o, np.array([1, 1], np.uint8), np.array([0, R - 1], np.uint32),
+              np.array([1, 2], np.uint32))
+    run_batch(g, o, np.array([0, 0, 2, 0], np.uint8), np.array([0, R - 1, 0, 1], np.uint32), None)
+    check_same_set(g, o)
+
+
+def test_contains_only_full_structure():
+    """Contains-only on a structure holding every key (C4 shape, small)."""
+    R = 200_000
+    for N in (32, 16):
+        g = GFSL(R, chunk_entries=N)
+        o = OracleMap(R)
+        prefill(g, o, R, R)
+        for op, key, val in workload_batches(R, 100_003, 2, (0, 0, 100)):
+            r = run_batch(g, o, op, key, val)
+            assert r.all()
+
+
+def test_zipf_batches():
+    R = 100_000
+    g = GFSL(R)
+    o = OracleMap(R)
+    prefill(g, o, R, R // 2)
+    for op, key, val in workload_batches(R, 20_000, 4, (10, 10, 80), dist="zipf"):
+        run_batch(g, o, op, key, val)
+    check_same_set(g, o)
+
+
+def test_batch_host_matches_device_path():
+    R = 10_000
+    g1, g2 = GFSL(R), GFSL(R)
+    o = OracleMap(R)
+    for op, key, val in workload_batches(R, 3_000, 5, (10, 10, 80)):
+        r1 = run_batch(g1, o, op, key, val)
+        r2 = g2.batch_host(torch.from_numpy(op), torch.from_numpy(key.view(np.int32)),
+                           torch.from_numpy(val.view(np.int32))).numpy()
+        assert np.array_equal(r1, r2)
+    _, k1, v1 = g1.validate()
+    _, k2, v2 = g2.validate()
+    assert np.array_equal(k1, k2) and np.array_equal(v1, v2)
