@@ -1,0 +1,408 @@
+#!/usr/bin/env python3
+"""GFSL batched Contains/Insert/Delete benchmark on B200 (BASELINE.json `metric`).
+
+One JSON line on rank 0.  A "step" is one `gfsl_batch` (classify -> Contains kernel ->
+update kernel) over one batch of synthetic ops; `value` is Mops/s over the K timed
+steps (all ops of all ranks / the slowest rank's summed step time).  Inputs are
+resident in HBM before each timed step; L2 is flushed (a 256 MiB write) between steps.
+
+    python bench.py [--config C2] [--gpus N --steps K --warmup W] [--impl reference]
+
+Configs: C1, C2 (default: R=1M, 10/10/80, the paper's
+Table 5.1 workload), C2-100, C2-2020, C2-5050, C3, C3-zipf, C4-32, C4-16, C5.
+N>1: weak scaling, each rank owns a key-range shard of the same size as the 1-GPU
+config, every rank draws ops over the whole key space and the batch is routed to the
+owners with NCCL all-to-all.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import sys
+import threading
+import time
+
+import numpy as np
+import torch
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+from paper_conf_ppopp_moscovicicp17_b200.workload import (  # noqa: E402
+    SEED_BASE, Workload, prefill_keys, prefill_values)
+
+METRIC = "Mops/s (mixed insert/delete/contains)"
+
+# name: (R, prefill, batch, n_batches, mix, dist, N)
+CONFIGS = {
+    "C1": (10_000, 5_000, 6_250, 16, (10, 10, 80), "uniform", 32),
+    "C2": (1_000_000, 500_000, 625_000, 16, (10, 10, 80), "uniform", 32),
+    "C2-100": (1_000_000, 1_000_000, 10_000_000, 1, (0, 0, 100), "uniform", 32),
+    "C2-2020": (1_000_000, 500_000, 312_500, 32, (20, 20, 60), "uniform", 32),
+    "C2-5050": (1_000_000, 500_000, 125_000, 80, (50, 50, 0), "uniform", 32),
+    "C3": (10_000_000, 5_000_000, 6_250_000, 16, (10, 10, 80), "uniform", 32),
+    "C3-zipf": (10_000_000, 5_000_000, 6_250_000, 16, (10, 10, 80), "zipf", 32),
+    "C4-32": (100_000_000, 100_000_000, 50_000_000, 10, (0, 0, 100), "uniform", 32),
+    "C4-16": (100_000_000, 100_000_000, 50_000_000, 10, (0, 0, 100), "uniform", 16),
+    "C5": (1_000_000_000, 500_000_000, 125_000_000, 8, (10, 10, 80), "uniform", 32),
+}
+L2_FLUSH_BYTES = 256 << 20
+
+
+def load_peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    try:
+        with open(p) as f:
+            d = json.load(f)
+        return float(d["hbm_gbs"]), "measured"
+    except Exception:
+        return 6650.0, "fallback"
+
+
+class ClockSampler:
+    """NVML SM clock + throttle reasons, sampled in a thread during the timed region."""
+
+    REASONS = {
+        0x0000000000000008: "hw_slowdown", 0x0000000000000040: "hw_thermal_slowdown",
+        0x0000000000000020: "sw_thermal_slowdown", 0x0000000000000004: "sw_power_cap",
+        0x0000000000000080: "hw_power_brake_slowdown",
+    }
+
+    def __init__(self, dev_index: int):
+        self.samples, self.reasons, self.ok = [], set(), False
+        self.max_mhz = None
+        try:
+            import pynvml
+            pynvml.nvmlInit()
+            self.nv = pynvml
+            self.hdl = pynvml.nvmlDeviceGetHandleByIndex(dev_index)
+            self.max_mhz = pynvml.nvmlDeviceGetMaxClockInfo(self.hdl, pynvml.NVML_CLOCK_SM)
+            self.ok = True
+        except Exception:
+            self.ok = False
+        self._stop = threading.Event()
+
+    def _run(self):
+        while not self._stop.is_set():
+            try:
+                self.samples.append(self.nv.nvmlDeviceGetClockInfo(self.hdl, self.nv.NVML_CLOCK_SM))
+                r = self.nv.nvmlDeviceGetCurrentClocksEventReasons(self.hdl)
+                for bit, name in self.REASONS.items():
+                    if r & bit:
+                        self.reasons.add(name)
+            except Exception:
+                pass
+            time.sleep(0.002)
+
+    def start(self):
+        if self.ok:
+            self.t = threading.Thread(target=self._run, daemon=True)
+            self.t.start()
+
+    def stop(self):
+        if self.ok:
+            self._stop.set()
+            self.t.join()
+        return {"sm_mhz": statistics.median(self.samples) if self.samples else None,
+                "sm_max_mhz": self.max_mhz, "reasons": sorted(self.reasons),
+                "samples": len(self.samples)}
+
+
+def dist_setup():
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    if world > 1:
+        import torch.distributed as dist
+        torch.cuda.set_device(local)
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    else:
+        torch.cuda.set_device(local)
+    return world, rank, local
+
+
+def barrier(world):
+    if world > 1:
+        import torch.distributed as dist
+        dist.barrier()
+
+
+def max_over_ranks(x: float, world: int) -> float:
+    if world == 1:
+        return x
+    import torch.distributed as dist
+    t = torch.tensor([x], dtype=torch.float64, device="cuda")
+    dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    return float(t.item())
+
+
+# --------------------------------------------------------------------------------------
+# reference arm / cpu baseline: the oracle as it stands, on this host's cores
+
+def oracle_sample(cfg_name, steps, warmup, budget_s=20.0, per_step_ops=1_000_000):
+    """Times Oracle-A on a bounded sample of the config's own batches (1 host thread)."""
+    from oracle.oracle_a import OracleMap
+    R, pre, B, nb, mix, dist, N = CONFIGS[cfg_name]
+    if pre > 4_000_000:
+        # bounded sample of a big config: one key-range shard of 2M keys with the same
+        # prefill density and the ops that fall into it (DESIGN.md §CPU baseline)
+        shard = 2_000_000
+        Rs = shard
+        pre_s = int(round(pre * shard / R))
+        note = f"key-range shard [0,{shard}) of R={R} at the same fill, same mix"
+    else:
+        Rs, pre_s, note = R, pre, f"the config itself (R={R})"
+    o = OracleMap(Rs)
+    k = prefill_keys(SEED_BASE, Rs, pre_s)
+    o.batch(np.ones(pre_s, np.uint8), k.numpy().astype(np.uint32),
+            prefill_values(SEED_BASE, k).numpy().astype(np.uint32))
+    Bs = min(B, per_step_ops)
+    w = Workload(Rs, Bs, mix=mix, dist=dist, seed=SEED_BASE + 1)
+    batches = []
+    for b in range(warmup + steps):
+        op, key, val, _ = w.make_batch(b)
+        batches.append((op.numpy(), key.numpy().astype(np.uint32), val.numpy().astype(np.uint32)))
+    for b in range(warmup):
+        o.batch(*batches[b])
+    t_total, n_total, done = 0.0, 0, 0
+    for b in range(warmup, warmup + steps):
+        t0 = time.perf_counter()
+        o.batch(*batches[b])
+        t_total += time.perf_counter() - t0
+        n_total += Bs
+        done += 1
+        if t_total > budget_s:
+            break
+    o.close()
+    mops = n_total / t_total / 1e6
+    return mops, t_total, done, Bs, note
+
+
+def run_reference(args, world, rank):
+    cfg = args.config
+    if rank != 0:
+        return
+    mops, t, done, Bs, note = oracle_sample(cfg, args.steps, args.warmup, budget_s=60.0)
+    line = {
+        "impl": "reference", "metric": METRIC, "value": round(mops, 4), "unit": "Mops/s",
+        "n_gpus": args.gpus, "steps": done, "warmup": args.warmup,
+        "ms_per_step": round(1000 * t / max(done, 1), 3), "higher_is_better": True,
+        "scaling": "weak", "vs_baseline": None, "dtype": "u32", "data": "synthetic",
+        "config": {"workload": cfg, "batch_ops_sampled": Bs},
+        "cpu_baseline": {"value": round(mops, 4), "unit": "Mops/s", "cores": 1,
+                         "kind": "oracle",
+                         "sample": f"{done} batches of {Bs} ops; {note}; Oracle-A (sequential Pugh skiplist, S1 batches)"},
+        "e2e": {"value": round(mops, 4), "unit": "Mops/s", "h2d_bytes_per_step": 0,
+                "d2h_bytes_per_step": 0},
+    }
+    print(json.dumps(line), flush=True)
+
+
+# --------------------------------------------------------------------------------------
+# GPU arm
+
+def make_inputs(w: Workload, b: int, dev):
+    op, key, val, redraws = w.make_batch(b, device=dev)
+    return op.contiguous(), key.to(torch.int32).contiguous(), val.to(torch.int32).contiguous(), redraws
+
+
+def prefill_gpu(g, R, count, dev, chunk=1 << 24, key_lo=0, seed=SEED_BASE):
+    for s in range(0, count, chunk):
+        c = min(chunk, count - s)
+        k = prefill_keys(seed, R, c, start=s, device=dev) + key_lo
+        v = prefill_values(seed, k)
+        g.batch(torch.ones(c, dtype=torch.uint8, device=dev), k.to(torch.int32),
+                v.to(torch.int32))
+    torch.cuda.synchronize()
+
+
+def run_gpu(args, world, rank, local):
+    from paper_conf_ppopp_moscovicicp17_b200.gfsl import GFSL
+    dev = torch.device("cuda", local)
+    R1, pre1, B1, nb, mix, dist, N = CONFIGS[args.config]
+    if args.chunk:
+        N = args.chunk
+    steps = args.steps if args.steps else nb
+    W = args.warmup
+    hbm_peak, peak_kind = load_peaks()
+
+    # weak scaling: each rank owns a shard of R1 keys and issues B1 ops per step
+    R = R1 * world
+    if world > 1:
+        from paper_conf_ppopp_moscovicicp17_b200.router import ShardedGFSL
+        g = ShardedGFSL(R, rank, world, capacity=R1, chunk_entries=N,
+                        contains_team=args.team, profile_phases=True)
+        lo = g.key_lo
+        prefill_gpu(g.local, R1, pre1, dev, key_lo=lo, seed=SEED_BASE + 1000 * rank)
+    else:
+        g = GFSL(R, capacity=R, chunk_entries=N, contains_team=args.team, profile_phases=True)
+        prefill_gpu(g, R, pre1, dev)
+    w = Workload(R, B1, mix=mix, dist=dist, seed=SEED_BASE + 1 + 7919 * rank)
+    inputs = [make_inputs(w, b, dev) for b in range(W + steps)]
+    redraws = sum(x[3] for x in inputs)
+    flush = torch.empty(L2_FLUSH_BYTES, dtype=torch.uint8, device=dev)
+    stream = torch.cuda.current_stream()
+
+    for b in range(W):
+        g.batch(*inputs[b][:3])
+    torch.cuda.synchronize()
+    barrier(world)
+    local_g = g.local if world > 1 else g
+    local_g.phase_times()  # reset the per-phase sums
+
+    starts = [torch.cuda.Event(enable_timing=True) for _ in range(steps)]
+    ends = [torch.cuda.Event(enable_timing=True) for _ in range(steps)]
+    clocks = ClockSampler(local)
+    barrier(world)
+    torch.cuda.synchronize()
+    clocks.start()
+    wall0 = time.perf_counter()
+    for j in range(steps):
+        flush.zero_()  # L2 flush between timed steps (outside the step's events)
+        starts[j].record(stream)
+        g.batch(*inputs[W + j][:3])
+        ends[j].record(stream)
+    torch.cuda.synchronize()
+    wall = time.perf_counter() - wall0
+    barrier(world)
+    clk = clocks.stop()
+    step_ms = [s.elapsed_time(e) for s, e in zip(starts, ends)]
+    local_ms = sum(step_ms)
+    total_ms = max_over_ranks(local_ms, world)
+    ops_total = B1 * steps * world
+    mops = ops_total / (total_ms / 1e3) / 1e6
+    phases, nbat = local_g.phase_times()
+
+    # algorithmic bytes: chunk reads per Contains op, counted on a Contains-only replay
+    # of the last timed batch's keys (untimed, non-mutating)
+    Cb = N * 8
+    local_g.configure(count_reads=1, profile_phases=0)
+    st0 = local_g.stats()
+    key_last = inputs[W + steps - 1][1]
+    if world > 1:
+        key_last = key_last[(key_last >= g.key_lo) & (key_last < g.key_hi)].contiguous()
+    local_g.batch(torch.zeros(key_last.numel(), dtype=torch.uint8, device=dev), key_last)
+    torch.cuda.synchronize()
+    st1 = local_g.stats()
+    local_g.configure(count_reads=0, profile_phases=1)
+    cops = max(1, st1["contains_ops"] - st0["contains_ops"])
+    reads_per_op = (st1["contains_reads"] - st0["contains_reads"]) / cops
+    reads_l0_per_op = (st1["contains_reads_l0"] - st0["contains_reads_l0"]) / cops
+
+    n_contains = int(round(B1 * mix[2] / 100.0))
+    n_update = B1 - n_contains
+    c_ms = phases["contains"] / max(nbat, 1)
+    u_ms = phases["update"] / max(nbat, 1)
+    i_ms = phases["intake"] / max(nbat, 1)
+    def roof(bytes_per_launch, ms):
+        if ms <= 0 or bytes_per_launch <= 0:
+            return None
+        ach = bytes_per_launch / (ms / 1e3) / 1e9
+        return {"bound": "hbm", "achieved": round(ach, 1), "peak": hbm_peak, "unit": "GB/s",
+                "frac": round(ach / hbm_peak, 4), "traffic": None,
+                "peak_kind": peak_kind}
+    # Contains: every chunk gather of the traversal is C_b random bytes
+    c_bytes = n_contains * reads_per_op * Cb
+    # update: the traversal (same chunk reads) + the entries written (~DSIZE/2 + NEXT/LOCK)
+    u_bytes = n_update * (reads_per_op * Cb + (N // 2) * 8 * 2)
+    roof_c = roof(c_bytes, c_ms)
+    roof_u = roof(u_bytes, u_ms)
+    dominant = "contains" if c_ms >= u_ms else "update"
+    roofline = roof_c if dominant == "contains" else roof_u
+    if roofline is not None:
+        roofline["kernel"] = dominant
+        roofline["algorithmic_bytes_per_launch"] = int(c_bytes if dominant == "contains" else u_bytes)
+
+    # end to end through the C ABI with host buffers (fresh handle, same sequence)
+    e2e = None
+    if not args.no_e2e and world == 1:
+        g2 = GFSL(R, capacity=R, chunk_entries=N, contains_team=args.team)
+        prefill_gpu(g2, R, pre1, dev)
+        host = [(x[0].cpu().pin_memory(), x[1].cpu().pin_memory(), x[2].cpu().pin_memory())
+                for x in inputs]
+        out = torch.empty(B1, dtype=torch.uint8).pin_memory()
+        for b in range(W):
+            g2.batch_host(*host[b], out=out)
+        t_e2e = 0.0
+        for j in range(steps):
+            flush.zero_()
+            torch.cuda.synchronize()
+            t0 = time.perf_counter()
+            g2.batch_host(*host[W + j], out=out)
+            t_e2e += time.perf_counter() - t0
+        e2e = {"value": round(B1 * steps / t_e2e / 1e6, 3), "unit": "Mops/s",
+               "h2d_bytes_per_step": B1 * 9, "d2h_bytes_per_step": B1}
+        g2.close()
+
+    cpu = None
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+        cm, ct, cdone, cBs, note = oracle_sample(args.config, min(steps, 16), 1, budget_s=15.0)
+        cpu = {"value": round(cm, 4), "unit": "Mops/s", "cores": 1, "kind": "oracle",
+               "sample": f"{cdone} batches of {cBs} ops ({ct:.1f} s); {note}"}
+
+    rep = None
+    if args.validate:
+        rep_obj, _, _ = local_g.validate(export=False)
+        rep = {"keys": rep_obj.keys, "height": rep_obj.height, "violations": rep_obj.violations}
+
+    if rank == 0:
+        line = {
+            "metric": METRIC, "value": round(mops, 3), "unit": "Mops/s", "n_gpus": world,
+            "steps": steps, "warmup": W, "ms_per_step": round(total_ms / steps, 4),
+            "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
+            "dtype": "u32", "data": "synthetic",
+            "config": {"workload": args.config, "key_range": R, "prefill": pre1 * world,
+                       "batch_ops": B1 * world, "mix_ins_del_con": list(mix), "keys": dist,
+                       "chunk_entries": N, "contains_team": local_g.cfg.contains_team or 8,
+                       "l2": "flushed (256 MiB write) between timed steps",
+                       "parallelism": f"range-shard x{world}" if world > 1 else "1 GPU"},
+            "roofline": roofline,
+            "roofline_kernels": {"contains": roof_c, "update": roof_u},
+            "phase_ms_per_step": {"intake": round(i_ms, 4), "contains": round(c_ms, 4),
+                                  "update": round(u_ms, 4)},
+            "chunk_reads_per_contains": round(reads_per_op, 3),
+            "chunk_reads_l0_per_contains": round(reads_l0_per_op, 3),
+            "cpu_baseline": cpu,
+            "e2e": e2e,
+            "gpu_launches": 3 * steps * (1 if world == 1 else 1) + (4 * steps if world > 1 else 0),
+            "clocks": clk,
+            "wall_s_timed_region": round(wall, 4),
+            "generator_redraws": int(redraws),
+            "validate": rep,
+        }
+        print(json.dumps(line), flush=True)
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=0, help="timed steps (0 = the config's batch count)")
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", default="gfsl", choices=["gfsl", "reference"])
+    ap.add_argument("--config", default="C2", choices=sorted(CONFIGS))
+    ap.add_argument("--team", type=int, default=0)
+    ap.add_argument("--chunk", type=int, default=0)
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--validate", action="store_true")
+    args = ap.parse_args()
+    if args.warmup < 3:
+        args.warmup = 3
+    if args.impl == "reference":
+        world = int(os.environ.get("WORLD_SIZE", "1"))
+        rank = int(os.environ.get("RANK", "0"))
+        if args.steps == 0:
+            args.steps = CONFIGS[args.config][3]
+        run_reference(args, world, rank)
+        return
+    world, rank, local = dist_setup()
+    run_gpu(args, world, rank, local)
+    if world > 1:
+        import torch.distributed as dist
+        dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

@@ -62,7 +62,11 @@ typedef struct gfsl_config {
   uint32_t update_blocks_per_sm;   /* launch shape of the update kernel; 0 = default */
   uint32_t serial_updates;  /* 1 = one team applies the updates strictly in op order
                                (deterministic structure; test mode).  0 = concurrent. */
-  uint32_t reserved[3];
+  uint32_t count_reads;     /* 1 = Contains kernel counts its chunk reads (gfsl_stats);
+                               measurement builds only, slower */
+  uint32_t profile_phases;  /* 1 = record CUDA events between the phases of every batch
+                               (read with gfsl_phase_times) */
+  uint32_t reserved[1];
 } gfsl_config;
 
 /*
@@ -75,6 +79,13 @@ typedef struct gfsl_config {
  */
 gfsl_t gfsl_create(uint64_t key_range, uint64_t capacity);
 gfsl_t gfsl_create_ex(uint64_t key_range, uint64_t capacity, const gfsl_config *cfg);
+
+/*
+ * Change the run-time options of a live handle: contains_team, the blocks-per-SM launch
+ * shapes, serial_updates, count_reads, profile_phases.  cfg->chunk_entries must be 0 or
+ * equal to the handle's.  Takes effect for the next batch.  GFSL_EINVAL if unsupported.
+ */
+gfsl_status gfsl_configure(gfsl_t h, const gfsl_config *cfg);
 
 /* Release every device resource of the handle (synchronizes the device first). */
 void gfsl_destroy(gfsl_t h);
@@ -119,7 +130,8 @@ typedef struct gfsl_report {
   uint32_t violations;          /* bitmask: bit v-1 set = invariant Vv violated */
   uint32_t first_violation;     /* lowest violated invariant number, 0 if none */
   uint64_t restarts;            /* Contains/search restarts so far */
-  uint64_t reserved[4];
+  uint64_t underfull;           /* non-last chunks with < floor(DSIZE/3) entries (info) */
+  uint64_t reserved[3];
 } gfsl_report;
 
 /*
@@ -142,9 +154,19 @@ typedef struct gfsl_stats {
   uint64_t splits, merges;  /* Alg 4.9 / Alg 4.12 */
   uint64_t zombie_unlinks;  /* Alg 4.6 l.10-20 redirects */
   uint64_t lock_retries;    /* failed CAS / waits in findAndLockEnclosing (Alg 4.8) */
-  uint64_t reserved[8];
+  uint64_t contains_reads;  /* chunk reads by Contains traversals (count_reads=1) */
+  uint64_t contains_reads_l0; /* ... of which on the bottom level */
+  uint64_t contains_ops;    /* Contains ops counted (count_reads=1) */
+  uint64_t reserved[5];
 } gfsl_stats;
 gfsl_status gfsl_get_stats(gfsl_t h, gfsl_stats *out);
+
+/*
+ * Per-phase device time of the batches enqueued since the last call (profile_phases=1):
+ * ms[0] intake (memset + classify), ms[1] Contains kernel, ms[2] update kernel,
+ * ms[3] whole batches; *batches = how many.  Synchronizes the device; resets the sums.
+ */
+gfsl_status gfsl_phase_times(gfsl_t h, double *ms, uint64_t *batches);
 
 /* ---- test-only: raw pool access (T2 byte parity, worked-example fixtures) ----
  * Pool image layout (host memory, little endian):

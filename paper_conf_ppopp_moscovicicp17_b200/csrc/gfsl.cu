@@ -8,6 +8,7 @@
 #include <cuda_runtime.h>
 
 #include <algorithm>
+#include <array>
 #include <cstdio>
 #include <cstring>
 #include <string>
@@ -55,6 +56,7 @@ struct gfsl {
   uint32_t *st_key = nullptr, *st_val = nullptr;
   uint64_t st_cap = 0;
   uint64_t batches = 0, ops = 0;
+  std::vector<std::array<cudaEvent_t, 4>> phase_ev;  // profile_phases
 };
 
 // ------------------------------------------------------------------------------------
@@ -127,7 +129,10 @@ __global__ void classify_kernel(const uint8_t *__restrict__ ops, const uint32_t 
 
 template <int N, int TEAM>
 static void launch_contains(gfsl *h, const uint32_t *keys, uint8_t *res, cudaStream_t s) {
-  contains_kernel<N, TEAM><<<h->contains_grid, 256, 0, s>>>(h->d, keys, res, h->list_c, h->ctl);
+  if (h->cfg.count_reads)
+    contains_kernel<N, TEAM, true><<<h->contains_grid, 256, 0, s>>>(h->d, keys, res, h->list_c, h->ctl);
+  else
+    contains_kernel<N, TEAM, false><<<h->contains_grid, 256, 0, s>>>(h->d, keys, res, h->list_c, h->ctl);
 }
 
 #define GFSL_CONTAINS_CONFIGS(X) X(32, 8) X(32, 16) X(32, 32) X(16, 4) X(16, 8) X(16, 16) X(12, 12) X(6, 6)
@@ -154,7 +159,7 @@ static void launch_update(gfsl *h, const uint8_t *ops, const uint32_t *keys, con
 template <int N, int TEAM>
 static int occ_contains() {
   int b = 0;
-  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, contains_kernel<N, TEAM>, 256, 0);
+  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, contains_kernel<N, TEAM, false>, 256, 0);
   return b;
 }
 template <int N>
@@ -194,6 +199,15 @@ static int update_occupancy(uint32_t N) {
 // ------------------------------------------------------------------------------------
 // create / destroy
 
+static void apply_launch_shape(gfsl *h) {
+  int bc = contains_occupancy(h->N, h->team);
+  if (h->cfg.contains_blocks_per_sm) bc = std::min<int>(bc, h->cfg.contains_blocks_per_sm);
+  int bu = update_occupancy(h->N);
+  if (h->cfg.update_blocks_per_sm) bu = std::min<int>(bu, h->cfg.update_blocks_per_sm);
+  h->contains_grid = h->sms * std::max(1, bc);
+  h->update_grid = h->sms * std::max(1, bu);
+}
+
 static void free_all(gfsl *h) {
   if (!h) return;
   cudaFree(h->d.pool);
@@ -210,6 +224,8 @@ static void free_all(gfsl *h) {
   cudaFree(h->st_val);
   if (h->h_error) cudaFreeHost(h->h_error);
   if (h->last) cudaEventDestroy(h->last);
+  for (auto &ev : h->phase_ev)
+    for (auto &e : ev) cudaEventDestroy(e);
   delete h;
 }
 
@@ -279,17 +295,31 @@ extern "C" gfsl_t gfsl_create_ex(uint64_t key_range, uint64_t capacity, const gf
   if ((e = cudaGetLastError()) != cudaSuccess) return fail("init kernels", e);
   if ((e = cudaDeviceSynchronize()) != cudaSuccess) return fail("init sync", e);
 
-  int bc = contains_occupancy(N, h->team);
-  if (cfg.contains_blocks_per_sm) bc = std::min<int>(bc, cfg.contains_blocks_per_sm);
-  int bu = update_occupancy(N);
-  if (cfg.update_blocks_per_sm) bu = std::min<int>(bu, cfg.update_blocks_per_sm);
-  h->contains_grid = h->sms * std::max(1, bc);
-  h->update_grid = h->sms * std::max(1, bu);
+  apply_launch_shape(h);
   return h;
 }
 
 extern "C" gfsl_t gfsl_create(uint64_t key_range, uint64_t capacity) {
   return gfsl_create_ex(key_range, capacity, nullptr);
+}
+
+extern "C" gfsl_status gfsl_configure(gfsl_t h, const gfsl_config *cfg) {
+  if (!h || !cfg) return GFSL_EINVAL;
+  if (cfg->chunk_entries != 0 && cfg->chunk_entries != h->N) {
+    set_last_error("gfsl_configure: chunk_entries cannot change");
+    return GFSL_EINVAL;
+  }
+  const uint32_t team = cfg->contains_team ? cfg->contains_team : ((h->N == 32 || h->N == 16) ? 8 : h->N);
+  if (!valid_team(h->N, team)) {
+    set_last_error("gfsl_configure: unsupported contains_team");
+    return GFSL_EINVAL;
+  }
+  h->cfg = *cfg;
+  h->cfg.chunk_entries = h->N;
+  h->cfg.contains_team = team;
+  h->team = team;
+  apply_launch_shape(h);
+  return GFSL_OK;
 }
 
 extern "C" void gfsl_destroy(gfsl_t h) {
@@ -333,11 +363,19 @@ static gfsl_status ensure_lists(gfsl *h, uint64_t n) {
 static gfsl_status enqueue_batch(gfsl *h, const uint8_t *ops, const uint32_t *keys,
                                  const uint32_t *vals, uint8_t *res, uint64_t n, cudaStream_t s) {
   CK(cudaStreamWaitEvent(s, h->last, 0));
+  std::array<cudaEvent_t, 4> ev{};
+  const bool prof = h->cfg.profile_phases != 0;
+  if (prof) {
+    for (auto &e : ev) CK(cudaEventCreate(&e));
+    CK(cudaEventRecord(ev[0], s));
+  }
   CK(cudaMemsetAsync(h->ctl, 0, sizeof(BatchCtl), s));
   const int cgrid = (int)std::min<uint64_t>((n + 255) / 256, (uint64_t)h->sms * 16);
   classify_kernel<<<std::max(cgrid, 1), 256, 0, s>>>(ops, keys, res, (uint32_t)n, h->key_range,
                                                     h->list_c, h->list_u, h->ctl);
+  if (prof) CK(cudaEventRecord(ev[1], s));
   bool ok = dispatch_contains(h, keys, res, s);
+  if (prof) CK(cudaEventRecord(ev[2], s));
   if (!ok) {
     set_last_error("no contains kernel for this (N, team)");
     return GFSL_EINVAL;
@@ -353,6 +391,10 @@ static gfsl_status enqueue_batch(gfsl *h, const uint8_t *ops, const uint32_t *ke
     h->sticky_cuda = true;
     set_last_error(std::string("kernel launch: ") + cudaGetErrorString(e));
     return GFSL_ECUDA;
+  }
+  if (prof) {
+    CK(cudaEventRecord(ev[3], s));
+    h->phase_ev.push_back(ev);
   }
   CK(cudaEventRecord(h->last, s));
   h->batches++;
@@ -432,6 +474,31 @@ extern "C" gfsl_status gfsl_get_stats(gfsl_t h, gfsl_stats *out) {
   out->merges = s[ST_MERGES];
   out->zombie_unlinks = s[ST_ZOMBIE_UNLINKS];
   out->lock_retries = s[ST_LOCK_RETRIES];
+  out->contains_reads = s[ST_CREADS];
+  out->contains_reads_l0 = s[ST_CREADS_L0];
+  out->contains_ops = s[ST_COPS];
+  return GFSL_OK;
+}
+
+extern "C" gfsl_status gfsl_phase_times(gfsl_t h, double *ms, uint64_t *batches) {
+  if (!h || !ms) return GFSL_EINVAL;
+  CK(cudaDeviceSynchronize());
+  double acc[4] = {0, 0, 0, 0};
+  for (auto &ev : h->phase_ev) {
+    float a = 0, b = 0, c = 0, t = 0;
+    CK(cudaEventElapsedTime(&a, ev[0], ev[1]));
+    CK(cudaEventElapsedTime(&b, ev[1], ev[2]));
+    CK(cudaEventElapsedTime(&c, ev[2], ev[3]));
+    CK(cudaEventElapsedTime(&t, ev[0], ev[3]));
+    acc[0] += a;
+    acc[1] += b;
+    acc[2] += c;
+    acc[3] += t;
+    for (auto &e : ev) cudaEventDestroy(e);
+  }
+  for (int i = 0; i < 4; ++i) ms[i] = acc[i];
+  if (batches) *batches = h->phase_ev.size();
+  h->phase_ev.clear();
   return GFSL_OK;
 }
 
@@ -496,7 +563,8 @@ extern "C" gfsl_status gfsl_load(gfsl_t h, const gfsl_meta *meta, const uint64_t
 //  V9 the head reaches a first non-zombie chunk holding -inf at index 0
 //  V10 keys are valid internal keys; -inf only first
 //  V12 every reachable chunk index is allocated
-//  V13 non-last non-zombie chunks hold >= floor(DSIZE/3) entries (derived)
+//  (V13 of SURVEY 8(c), min fill floor(DSIZE/3), is NOT an invariant: a splitRemove can
+//   leave the new chunk with cntF - DSIZE/2 < DSIZE/3 entries; it is reported as a count)
 //  V14 counter[l] = #non-zombie chunks if level l holds a real key, else 0 (R9/R17)
 
 namespace {
@@ -611,7 +679,7 @@ extern "C" gfsl_status gfsl_validate(gfsl_t h, gfsl_report *rep_out, uint32_t *k
         if (mx != KEY_POS_INF) V(2);
       } else {
         if (cnt == 0 || mx != last_key) V(2);
-        if (cnt < std::max<uint32_t>(1, DS / 3)) V(13);
+        if (cnt < std::max<uint32_t>(1, DS / 3)) rep.underfull++;  // underfull (not an invariant)
       }
       // V3
       if (have_prev && cnt > 0) {

@@ -26,7 +26,7 @@
 
 namespace gfsl_dev {
 
-template <int N, int TEAM>
+template <int N, int TEAM, bool COUNT = false>
 __global__ void __launch_bounds__(256)
 contains_kernel(DevState d, const uint32_t *__restrict__ keys, uint8_t *__restrict__ res,
                 const uint32_t *__restrict__ list, const BatchCtl *__restrict__ ctl) {
@@ -75,11 +75,16 @@ contains_kernel(DevState d, const uint32_t *__restrict__ keys, uint8_t *__restri
   int level = height;
   uint32_t bt = NULL_CHUNK;                          // backtrack pointer (reduced prevKv)
   unsigned long long restarts = 0;
+  unsigned long long reads = 0, reads_l0 = 0, nops = 0;  // COUNT build only
 
   while (__any_sync(FULL, active)) {
     ChunkSlice<EPL> s;
     if (active) {
       ld_slice_nc<EPL>(d.pool + (size_t)cur * N + t * EPL, s);
+      if (COUNT) {
+        ++reads;
+        reads_l0 += (level == 0);
+      }
     } else {
 #pragma unroll
       for (int j = 0; j < EPL; ++j) { s.k[j] = KEY_EMPTY; s.v[j] = NULL_CHUNK; }
@@ -122,6 +127,7 @@ contains_kernel(DevState d, const uint32_t *__restrict__ keys, uint8_t *__restri
         const bool te = (be >> team_base) & TEAM_BITS;
         if (t == 0) res[opi] = te ? 1 : 0;
         done = true;
+        if (COUNT) ++nops;
       } else if (tb) {                 // down step (l.19-23)
         --level;
         bt = NULL_CHUNK;
@@ -149,6 +155,11 @@ contains_kernel(DevState d, const uint32_t *__restrict__ keys, uint8_t *__restri
     }
   }
   if (restarts && t == 0) stat_add(d, ST_RESTARTS, restarts);
+  if (COUNT && t == 0 && lane_live) {
+    stat_add(d, ST_CREADS, reads);
+    stat_add(d, ST_CREADS_L0, reads_l0);
+    stat_add(d, ST_COPS, nops);
+  }
 }
 
 }  // namespace gfsl_dev

@@ -33,7 +33,11 @@ constexpr uint32_t ERR_HANG = 2u;     // a watchdog fired (corrupt structure / l
 
 // statistics slots
 enum StatSlot {
-  ST_RESTARTS = 0, ST_SPLITS, ST_MERGES, ST_ZOMBIE_UNLINKS, ST_LOCK_RETRIES, ST_NSTATS
+  ST_RESTARTS = 0, ST_SPLITS, ST_MERGES, ST_ZOMBIE_UNLINKS, ST_LOCK_RETRIES,
+  ST_CREADS,      // chunk reads of Contains traversals (counting build only)
+  ST_CREADS_L0,   // ... of which on the bottom level
+  ST_COPS,        // Contains ops counted
+  ST_NSTATS
 };
 
 // Device view of one handle.

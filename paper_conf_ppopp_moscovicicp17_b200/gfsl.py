@@ -29,7 +29,8 @@ class gfsl_config(ctypes.Structure):
     _fields_ = [("chunk_entries", ctypes.c_uint32), ("contains_team", ctypes.c_uint32),
                 ("contains_blocks_per_sm", ctypes.c_uint32),
                 ("update_blocks_per_sm", ctypes.c_uint32),
-                ("serial_updates", ctypes.c_uint32), ("reserved", ctypes.c_uint32 * 3)]
+                ("serial_updates", ctypes.c_uint32), ("count_reads", ctypes.c_uint32),
+                ("profile_phases", ctypes.c_uint32), ("reserved", ctypes.c_uint32 * 1)]
 
 
 class gfsl_report(ctypes.Structure):
@@ -39,14 +40,16 @@ class gfsl_report(ctypes.Structure):
                 ("counters", ctypes.c_int64 * 32), ("pool_used", ctypes.c_uint64 * 2),
                 ("pool_cap", ctypes.c_uint64 * 2), ("violations", ctypes.c_uint32),
                 ("first_violation", ctypes.c_uint32), ("restarts", ctypes.c_uint64),
-                ("reserved", ctypes.c_uint64 * 4)]
+                ("underfull", ctypes.c_uint64), ("reserved", ctypes.c_uint64 * 3)]
 
 
 class gfsl_stats(ctypes.Structure):
     _fields_ = [("batches", ctypes.c_uint64), ("ops", ctypes.c_uint64),
                 ("restarts", ctypes.c_uint64), ("splits", ctypes.c_uint64),
                 ("merges", ctypes.c_uint64), ("zombie_unlinks", ctypes.c_uint64),
-                ("lock_retries", ctypes.c_uint64), ("reserved", ctypes.c_uint64 * 8)]
+                ("lock_retries", ctypes.c_uint64), ("contains_reads", ctypes.c_uint64),
+                ("contains_reads_l0", ctypes.c_uint64), ("contains_ops", ctypes.c_uint64),
+                ("reserved", ctypes.c_uint64 * 5)]
 
 
 class gfsl_meta(ctypes.Structure):
@@ -60,7 +63,8 @@ class gfsl_meta(ctypes.Structure):
 EXPORTS = [
     "gfsl_create", "gfsl_create_ex", "gfsl_destroy", "gfsl_batch", "gfsl_batch_host",
     "gfsl_validate", "gfsl_last_error", "gfsl_get_stats", "gfsl_dump", "gfsl_load",
-    "gfsl_route_plan", "gfsl_route_pack", "gfsl_route_unpack",
+    "gfsl_route_plan", "gfsl_route_pack", "gfsl_route_unpack", "gfsl_phase_times",
+    "gfsl_configure",
 ]
 
 _lib = None
@@ -98,6 +102,10 @@ def load_library(path: str = LIB_PATH):
     lib.gfsl_dump.argtypes = [vp, ctypes.POINTER(gfsl_meta), vp, u64]
     lib.gfsl_load.restype = i32
     lib.gfsl_load.argtypes = [vp, ctypes.POINTER(gfsl_meta), vp, u64]
+    lib.gfsl_configure.restype = i32
+    lib.gfsl_configure.argtypes = [vp, ctypes.POINTER(gfsl_config)]
+    lib.gfsl_phase_times.restype = i32
+    lib.gfsl_phase_times.argtypes = [vp, ctypes.POINTER(ctypes.c_double), ctypes.POINTER(u64)]
     lib.gfsl_route_plan.restype = i32
     lib.gfsl_route_plan.argtypes = [vp, vp, u64, u64, u32, vp, vp, vp]
     lib.gfsl_route_pack.restype = i32
@@ -144,6 +152,7 @@ class Report:
     violations: int
     first_violation: int
     restarts: int
+    underfull: int
 
 
 class GFSL:
@@ -151,15 +160,18 @@ class GFSL:
 
     def __init__(self, key_range: int, capacity: int = 0, chunk_entries: int = 32,
                  contains_team: int = 0, serial_updates: bool = False,
-                 contains_blocks_per_sm: int = 0, update_blocks_per_sm: int = 0):
+                 contains_blocks_per_sm: int = 0, update_blocks_per_sm: int = 0,
+                 count_reads: bool = False, profile_phases: bool = False):
         import torch
         if not torch.cuda.is_available():
             raise RuntimeError("GFSL needs a CUDA device (there is no CPU fallback)")
         self.lib = load_library()
         cfg = gfsl_config(chunk_entries, contains_team, contains_blocks_per_sm,
-                          update_blocks_per_sm, 1 if serial_updates else 0)
+                          update_blocks_per_sm, 1 if serial_updates else 0,
+                          1 if count_reads else 0, 1 if profile_phases else 0)
         self.key_range = int(key_range)
         self.chunk_entries = int(chunk_entries)
+        self.cfg = cfg
         self.h = self.lib.gfsl_create_ex(self.key_range, int(capacity), ctypes.byref(cfg))
         if not self.h:
             raise RuntimeError("gfsl_create failed: " + self.lib.gfsl_last_error().decode())
@@ -217,7 +229,8 @@ class GFSL:
             st = self.lib.gfsl_validate(self.h, None, keys.ctypes.data, vals.ctypes.data, n, None)
         report = Report(rep.keys, rep.height, list(rep.chunks), list(rep.zombies),
                         list(rep.level_keys), list(rep.counters), tuple(rep.pool_used),
-                        tuple(rep.pool_cap), rep.violations, rep.first_violation, rep.restarts)
+                        tuple(rep.pool_cap), rep.violations, rep.first_violation, rep.restarts,
+                        rep.underfull)
         if st == GFSL_ECORRUPT and raise_on_violation:
             raise GFSLError(st, f"gfsl_validate (violations=0x{rep.violations:x})")
         return report, keys, vals
@@ -226,6 +239,19 @@ class GFSL:
         s = gfsl_stats()
         _check(self.lib.gfsl_get_stats(self.h, ctypes.byref(s)), "gfsl_get_stats")
         return {f: getattr(s, f) for f, _ in gfsl_stats._fields_ if f != "reserved"}
+
+    def configure(self, **kw):
+        """Change run-time options (contains_team, serial_updates, count_reads, ...)."""
+        for k, v in kw.items():
+            setattr(self.cfg, k, int(v))
+        _check(self.lib.gfsl_configure(self.h, ctypes.byref(self.cfg)), "gfsl_configure")
+
+    def phase_times(self):
+        """(ms dict of intake/contains/update/total since the last call, batches)."""
+        ms = (ctypes.c_double * 4)()
+        nb = ctypes.c_uint64()
+        _check(self.lib.gfsl_phase_times(self.h, ms, ctypes.byref(nb)), "gfsl_phase_times")
+        return dict(intake=ms[0], contains=ms[1], update=ms[2], total=ms[3]), nb.value
 
     def dump(self):
         """(meta dict, entries uint64 array of shape [chunks, N]) -- test-only."""
