@@ -355,7 +355,7 @@ def run_gpu(args, world, rank, local):
             "dtype": "u32", "data": "synthetic",
             "config": {"workload": args.config, "key_range": R, "prefill": pre1 * world,
                        "batch_ops": B1 * world, "mix_ins_del_con": list(mix), "keys": dist,
-                       "chunk_entries": N, "contains_team": local_g.cfg.contains_team or 8,
+                       "chunk_entries": N, "contains_team": local_g.cfg.contains_team or (4 if N == 32 else 2),
                        "l2": "flushed (256 MiB write) between timed steps",
                        "parallelism": f"range-shard x{world}" if world > 1 else "1 GPU"},
             "roofline": roofline,

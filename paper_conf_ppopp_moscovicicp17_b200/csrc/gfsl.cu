@@ -15,7 +15,7 @@
 #include <vector>
 
 #include "../../include/gfsl.h"
-#include "gfsl_contains.cuh"
+#include "gfsl_search.cuh"
 #include "gfsl_device.cuh"
 #include "gfsl_update.cuh"
 
@@ -45,7 +45,9 @@ struct gfsl {
   uint64_t key_range = 0;
   DevState d{};
   BatchCtl *ctl = nullptr;
-  uint32_t *list_c = nullptr, *list_u = nullptr;
+  uint2 *list_c = nullptr, *list_u = nullptr;
+  uint32_t *plan_path = nullptr, *mut_list = nullptr;
+  uint8_t *plan_top = nullptr;
   uint64_t list_cap = 0;
   uint32_t *h_error = nullptr;  // mapped host memory, device alias in d.error
   cudaEvent_t last = nullptr;
@@ -94,13 +96,14 @@ __global__ void init_heads_kernel(DevState d, uint32_t N) {
 // Contains list and the Insert/Delete list (warp-aggregated appends).
 __global__ void classify_kernel(const uint8_t *__restrict__ ops, const uint32_t *__restrict__ keys,
                                 uint8_t *__restrict__ res, uint32_t n, uint64_t key_range,
-                                uint32_t *__restrict__ list_c, uint32_t *__restrict__ list_u,
+                                uint2 *__restrict__ list_c, uint2 *__restrict__ list_u,
                                 BatchCtl *ctl) {
   const int lane = threadIdx.x & 31;
   const uint32_t stride = gridDim.x * blockDim.x;
   for (uint32_t base = blockIdx.x * blockDim.x; base < n; base += stride) {
     const uint32_t i = base + threadIdx.x;
     bool isc = false, isu = false;
+    uint2 e = make_uint2(0, 0);
     if (i < n) {
       const uint8_t op = ops[i];
       const uint32_t k = keys[i];
@@ -108,6 +111,7 @@ __global__ void classify_kernel(const uint8_t *__restrict__ ops, const uint32_t 
       if (!valid) res[i] = 0xFF;
       isc = valid && op == 0;
       isu = valid && op != 0;
+      e = make_uint2(i | (op == 2 ? DELETE_FLAG : 0u), k + 1u);  // internal key (R3)
     }
     const uint32_t bc = __ballot_sync(0xFFFFFFFFu, isc);
     const uint32_t bu = __ballot_sync(0xFFFFFFFFu, isu);
@@ -119,27 +123,85 @@ __global__ void classify_kernel(const uint8_t *__restrict__ ops, const uint32_t 
     oc = __shfl_sync(0xFFFFFFFFu, oc, 0);
     ou = __shfl_sync(0xFFFFFFFFu, ou, 0);
     const uint32_t below = (1u << lane) - 1u;
-    if (isc) list_c[oc + __popc(bc & below)] = i;
-    if (isu) list_u[ou + __popc(bu & below)] = i;
+    if (isc) list_c[oc + __popc(bc & below)] = e;
+    if (isu) list_u[ou + __popc(bu & below)] = e;
+  }
+}
+
+// Serial (test) mode: the same split, in op-index order (one block, tile by tile).
+__global__ void classify_ordered_kernel(const uint8_t *__restrict__ ops, const uint32_t *__restrict__ keys,
+                                        uint8_t *__restrict__ res, uint32_t n, uint64_t key_range,
+                                        uint2 *__restrict__ list_c, uint2 *__restrict__ list_u,
+                                        BatchCtl *ctl) {
+  __shared__ uint32_t wc[8], wu[8];
+  __shared__ uint32_t base_c, base_u;
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  if (threadIdx.x == 0) base_c = base_u = 0;
+  __syncthreads();
+  for (uint32_t base = 0; base < n; base += blockDim.x) {
+    const uint32_t i = base + threadIdx.x;
+    bool isc = false, isu = false;
+    uint2 e = make_uint2(0, 0);
+    if (i < n) {
+      const uint8_t op = ops[i];
+      const bool valid = op <= 2 && (uint64_t)keys[i] < key_range;
+      if (!valid) res[i] = 0xFF;
+      isc = valid && op == 0;
+      isu = valid && op != 0;
+      e = make_uint2(i | (op == 2 ? DELETE_FLAG : 0u), keys[i] + 1u);
+    }
+    const uint32_t bc = __ballot_sync(0xFFFFFFFFu, isc), bu = __ballot_sync(0xFFFFFFFFu, isu);
+    if (lane == 0) {
+      wc[warp] = __popc(bc);
+      wu[warp] = __popc(bu);
+    }
+    __syncthreads();
+    uint32_t oc = base_c, ou = base_u;
+    for (int w = 0; w < warp; ++w) {
+      oc += wc[w];
+      ou += wu[w];
+    }
+    const uint32_t below = (1u << lane) - 1u;
+    if (isc) list_c[oc + __popc(bc & below)] = e;
+    if (isu) list_u[ou + __popc(bu & below)] = e;
+    __syncthreads();
+    if (threadIdx.x == 0) {
+      for (int w = 0; w < (int)(blockDim.x >> 5); ++w) {
+        base_c += wc[w];
+        base_u += wu[w];
+      }
+    }
+    __syncthreads();
+  }
+  if (threadIdx.x == 0) {
+    ctl->n_contains = base_c;
+    ctl->n_updates = base_u;
   }
 }
 
 // ------------------------------------------------------------------------------------
 // template dispatch
 
+static SearchOut search_out(gfsl *h) { return SearchOut{h->plan_path, h->plan_top, h->mut_list}; }
+
 template <int N, int TEAM>
-static void launch_contains(gfsl *h, const uint32_t *keys, uint8_t *res, cudaStream_t s) {
+static void launch_contains(gfsl *h, const uint8_t *ops, const uint32_t *keys, uint8_t *res,
+                            cudaStream_t s) {
   if (h->cfg.count_reads)
-    contains_kernel<N, TEAM, true><<<h->contains_grid, 256, 0, s>>>(h->d, keys, res, h->list_c, h->ctl);
+    search_kernel<N, TEAM, true><<<h->contains_grid, 256, 0, s>>>(h->d, res, h->list_c, h->list_u,
+                                                                  h->ctl, search_out(h));
   else
-    contains_kernel<N, TEAM, false><<<h->contains_grid, 256, 0, s>>>(h->d, keys, res, h->list_c, h->ctl);
+    search_kernel<N, TEAM, false><<<h->contains_grid, 256, 0, s>>>(h->d, res, h->list_c, h->list_u,
+                                                                   h->ctl, search_out(h));
 }
 
-#define GFSL_CONTAINS_CONFIGS(X) X(32, 8) X(32, 16) X(32, 32) X(16, 4) X(16, 8) X(16, 16) X(12, 12) X(6, 6)
+#define GFSL_CONTAINS_CONFIGS(X) \
+  X(32, 4) X(32, 8) X(32, 16) X(32, 32) X(16, 2) X(16, 4) X(16, 8) X(16, 16) X(12, 12) X(6, 6)
 
-static bool dispatch_contains(gfsl *h, const uint32_t *keys, uint8_t *res, cudaStream_t s) {
+static bool dispatch_contains(gfsl *h, const uint8_t *ops, const uint32_t *keys, uint8_t *res,
+                              cudaStream_t s) {
   switch (h->N * 100 + h->team) {
-#define X(n, t) case n * 100 + t: launch_contains<n, t>(h, keys, res, s); return true;
+#define X(n, t) case n * 100 + t: launch_contains<n, t>(h, ops, keys, res, s); return true;
     GFSL_CONTAINS_CONFIGS(X)
 #undef X
   }
@@ -149,17 +211,18 @@ static bool dispatch_contains(gfsl *h, const uint32_t *keys, uint8_t *res, cudaS
 template <int N>
 static void launch_update(gfsl *h, const uint8_t *ops, const uint32_t *keys, const uint32_t *vals,
                           uint8_t *res, uint32_t n, cudaStream_t s) {
+  (void)n;
   if (h->cfg.serial_updates) {
-    update_kernel<N><<<1, 32, 0, s>>>(h->d, ops, keys, vals, res, h->list_u, h->ctl, 1, n);
+    update_kernel<N><<<1, 32, 0, s>>>(h->d, vals, res, h->list_u, h->ctl, search_out(h), 1);
   } else {
-    update_kernel<N><<<h->update_grid, 256, 0, s>>>(h->d, ops, keys, vals, res, h->list_u, h->ctl, 0, n);
+    update_kernel<N><<<h->update_grid, 256, 0, s>>>(h->d, vals, res, h->list_u, h->ctl, search_out(h), 0);
   }
 }
 
 template <int N, int TEAM>
 static int occ_contains() {
   int b = 0;
-  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, contains_kernel<N, TEAM, false>, 256, 0);
+  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, search_kernel<N, TEAM, false>, 256, 0);
   return b;
 }
 template <int N>
@@ -218,6 +281,9 @@ static void free_all(gfsl *h) {
   cudaFree(h->ctl);
   cudaFree(h->list_c);
   cudaFree(h->list_u);
+  cudaFree(h->plan_path);
+  cudaFree(h->plan_top);
+  cudaFree(h->mut_list);
   cudaFree(h->st_op);
   cudaFree(h->st_res);
   cudaFree(h->st_key);
@@ -243,7 +309,7 @@ extern "C" gfsl_t gfsl_create_ex(uint64_t key_range, uint64_t capacity, const gf
     return nullptr;
   }
   if (capacity == 0) capacity = key_range;
-  if (cfg.contains_team == 0) cfg.contains_team = (N == 32 || N == 16) ? 8 : N;
+  if (cfg.contains_team == 0) cfg.contains_team = (N == 32) ? 4 : (N == 16) ? 2 : N;
   if (!valid_team(N, cfg.contains_team)) {
     set_last_error("unsupported contains_team for this chunk size");
     return nullptr;
@@ -268,9 +334,9 @@ extern "C" gfsl_t gfsl_create_ex(uint64_t key_range, uint64_t capacity, const gf
   const uint64_t m = std::max<uint64_t>(1, DS / 3);
   uint64_t cap_b = 2 * ((capacity + 1) / m + 1) + 64;
   uint64_t cap_u = cap_b / 8 + 2 * N + 64;
-  if (cap_b + cap_u >= 0xFFFFFFF0ull) {
+  if (cap_b + cap_u >= (1ull << 30)) {  // 30-bit indices: two flag bits ride on shuffles
     free_all(h);
-    set_last_error("capacity too large for 32-bit chunk indices");
+    set_last_error("capacity too large for 30-bit chunk indices");
     return nullptr;
   }
   h->d.cap_bottom = (uint32_t)cap_b;
@@ -309,7 +375,7 @@ extern "C" gfsl_status gfsl_configure(gfsl_t h, const gfsl_config *cfg) {
     set_last_error("gfsl_configure: chunk_entries cannot change");
     return GFSL_EINVAL;
   }
-  const uint32_t team = cfg->contains_team ? cfg->contains_team : ((h->N == 32 || h->N == 16) ? 8 : h->N);
+  const uint32_t team = cfg->contains_team ? cfg->contains_team : (h->N == 32 ? 4 : h->N == 16 ? 2 : h->N);
   if (!valid_team(h->N, team)) {
     set_last_error("gfsl_configure: unsupported contains_team");
     return GFSL_EINVAL;
@@ -351,11 +417,19 @@ static gfsl_status ensure_lists(gfsl *h, uint64_t n) {
   cudaDeviceSynchronize();
   cudaFree(h->list_c);
   cudaFree(h->list_u);
+  cudaFree(h->plan_path);
+  cudaFree(h->plan_top);
+  cudaFree(h->mut_list);
   h->list_c = h->list_u = nullptr;
+  h->plan_path = h->mut_list = nullptr;
+  h->plan_top = nullptr;
   h->list_cap = 0;
   const uint64_t cap = std::max<uint64_t>(n, 1024);
-  CK(cudaMalloc(&h->list_c, cap * 4));
-  CK(cudaMalloc(&h->list_u, cap * 4));
+  CK(cudaMalloc(&h->list_c, cap * 8));
+  CK(cudaMalloc(&h->list_u, cap * 8));
+  CK(cudaMalloc(&h->plan_path, cap * 4 * PLAN_LEVELS));
+  CK(cudaMalloc(&h->plan_top, cap));
+  CK(cudaMalloc(&h->mut_list, cap * 4));
   h->list_cap = cap;
   return GFSL_OK;
 }
@@ -370,11 +444,16 @@ static gfsl_status enqueue_batch(gfsl *h, const uint8_t *ops, const uint32_t *ke
     CK(cudaEventRecord(ev[0], s));
   }
   CK(cudaMemsetAsync(h->ctl, 0, sizeof(BatchCtl), s));
-  const int cgrid = (int)std::min<uint64_t>((n + 255) / 256, (uint64_t)h->sms * 16);
-  classify_kernel<<<std::max(cgrid, 1), 256, 0, s>>>(ops, keys, res, (uint32_t)n, h->key_range,
-                                                    h->list_c, h->list_u, h->ctl);
+  if (h->cfg.serial_updates) {
+    classify_ordered_kernel<<<1, 256, 0, s>>>(ops, keys, res, (uint32_t)n, h->key_range, h->list_c,
+                                              h->list_u, h->ctl);
+  } else {
+    const int cgrid = (int)std::min<uint64_t>((n + 255) / 256, (uint64_t)h->sms * 16);
+    classify_kernel<<<std::max(cgrid, 1), 256, 0, s>>>(ops, keys, res, (uint32_t)n, h->key_range,
+                                                      h->list_c, h->list_u, h->ctl);
+  }
   if (prof) CK(cudaEventRecord(ev[1], s));
-  bool ok = dispatch_contains(h, keys, res, s);
+  bool ok = dispatch_contains(h, ops, keys, res, s);
   if (prof) CK(cudaEventRecord(ev[2], s));
   if (!ok) {
     set_last_error("no contains kernel for this (N, team)");

@@ -55,10 +55,12 @@ struct DevState {
 
 // Per-batch control block (device memory, zeroed before every batch).
 struct BatchCtl {
-  uint32_t n_contains;
-  uint32_t n_updates;
+  uint32_t n_contains;   // Contains ops of the batch (classify)
+  uint32_t n_updates;    // Insert/Delete ops of the batch (classify)
+  uint32_t n_mut;        // update ops that mutate (search kernel)
   uint32_t next_update;  // dynamic work counter of the update kernel
-  uint32_t pad;
+  uint32_t snap_height;  // height seen by the search kernel
+  uint32_t pad[3];
 };
 
 __device__ __forceinline__ uint32_t lo32(uint64_t x) { return (uint32_t)x; }
@@ -89,6 +91,17 @@ __device__ __forceinline__ int32_t ld_relaxed_s32(const int32_t *p) {
   int32_t v;
   asm volatile("ld.relaxed.gpu.global.s32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
   return v;
+}
+__device__ __forceinline__ void st_release(uint64_t *p, uint64_t v) {
+  asm volatile("st.release.gpu.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
+__device__ __forceinline__ uint64_t cas_acquire(uint64_t *p, uint64_t cmp, uint64_t val) {
+  uint64_t old;
+  asm volatile("atom.acquire.gpu.global.cas.b64 %0, [%1], %2, %3;"
+               : "=l"(old)
+               : "l"(p), "l"(cmp), "l"(val)
+               : "memory");
+  return old;
 }
 __device__ __forceinline__ void st_relaxed(uint64_t *p, uint64_t v) {
   asm volatile("st.relaxed.gpu.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");

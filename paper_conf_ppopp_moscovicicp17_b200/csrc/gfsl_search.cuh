@@ -1,0 +1,206 @@
+// gfsl_search.cuh -- B1: the read-only search phase of a batch (Alg 4.1-4.4, 4.6).
+//
+// Under the S1 snapshot semantics (R1) every op of a batch is answered against
+// the structure as it was before the batch.  So ALL traversals of a batch -- the
+// Contains of Alg 4.1 and the searchSlow of every Insert/Delete (Alg 4.5 l.2, Alg 4.11
+// l.3) -- run first, in this kernel, on a quiescent structure: no locks, no fences, no
+// restarts, and chunk reads through the read-only L1 path.
+//
+// Traversal (searchDown, Alg 4.2, then searchLateral, Alg 4.4): each step is one
+// coalesced chunk read followed by the team vote of getTidForNextStep (Alg 4.3):
+//   DATA entry i votes  key_i <= k,   NEXT votes  max < k,   LOCK votes  zombie;
+// the highest voting entry decides: LOCK -> lateral past a zombie (Alg 4.2
+// l.9-11), NEXT -> lateral step keeping the previous chunk for a backtrack (l.15-18),
+// DATA i -> down step through value_i (l.19-23), none -> backtrack through the previous
+// chunk's highest key <= k (l.24-28, 33-38), or restart (l.25; impossible here).  On the
+// bottom level the DATA vote is key_i == k (Alg 4.4).
+//
+// For an Insert/Delete the kernel also records what searchSlow returns (Alg 4.6): the
+// path (chunk of the down step at every level, the enclosing bottom chunk at level 0)
+// and the highest level at which k was seen.  Its result is exact already (under the
+// <=1-mutation-per-key contract the snapshot decides "present?"), and only the ops that
+// will mutate (Insert of an absent key, Delete of a present key) go on to the update
+// kernel (B2), which starts from the recorded path ("the enclosing chunk must
+// either be in the path or reachable from it").
+//
+// B200 design: a team is TEAM lanes (TEAM | 32, TEAM <= N); each lane
+// holds EPL = N/TEAM consecutive entries loaded with one vector load (8/16/32 B), so a
+// warp runs 32/TEAM independent traversals in lockstep (P:205 allows teams smaller than
+// a warp; the paper's one-team-per-warp is TEAM == N).  A team's vote is "highest lane
+// holding a voting entry" (one __ballot_sync) plus that lane's own highest voting entry,
+// and the down pointer comes with one __shfl_sync.  prevKv is reduced to the two
+// values a backtrack needs: the previous chunk and its highest key <= k's down pointer.
+#pragma once
+#include "gfsl_device.cuh"
+
+namespace gfsl_dev {
+
+constexpr int PLAN_LEVELS = 16;  // path levels recorded per update op (height < 16)
+
+// Op lists built by the classify kernel: {op index | DELETE_FLAG if Delete, internal key}.
+constexpr uint32_t DELETE_FLAG = 0x80000000u;
+constexpr uint32_t OPI_MASK = 0x7FFFFFFFu;
+// Chunk indices are < 2^30, so a shuffled pointer carries two flag bits.
+constexpr uint32_t PTR_MASK = 0x3FFFFFFFu;
+constexpr uint32_t F_ZOMBIE = 0x80000000u;   // on the NEXT pointer: the chunk is a zombie
+constexpr uint32_t F_LATERAL = 0x40000000u;  // on the NEXT pointer: max < k
+constexpr uint32_t F_EQUAL = 0x80000000u;    // on the down pointer: the winning key == k
+
+struct SearchOut {
+  uint32_t *plan_path;  // [n_updates * PLAN_LEVELS]
+  uint8_t *plan_top;    // [n_updates]: highest level holding k (0 = bottom only), 0xFF = no-op
+  uint32_t *mut_list;   // [n_updates]: update slots that mutate
+};
+
+template <int N, int TEAM, bool COUNT = false>
+__global__ void __launch_bounds__(256)
+search_kernel(DevState d, uint8_t *__restrict__ res, const uint2 *__restrict__ list_c,
+              const uint2 *__restrict__ list_u, BatchCtl *__restrict__ ctl, SearchOut so) {
+  constexpr int DSIZE = N - 2;
+  constexpr int EPL = N / TEAM;
+  static_assert(EPL * TEAM == N, "TEAM must divide N");
+  constexpr int TPW = 32 / TEAM;                    // teams per warp
+  constexpr uint32_t TEAM_BITS = (TEAM == 32) ? 0xFFFFFFFFu : ((1u << TEAM) - 1u);
+  constexpr int NEXT_E = N - 2, LOCK_E = N - 1;
+  constexpr int NEXT_LANE = NEXT_E / EPL, NEXT_J = NEXT_E % EPL;
+  constexpr int LOCK_LANE = LOCK_E / EPL, LOCK_J = LOCK_E % EPL;
+  constexpr uint32_t FULL = 0xFFFFFFFFu;
+
+  __shared__ uint32_t s_start, s_height;
+  const int lane = threadIdx.x & 31;
+  if (threadIdx.x < 32) {
+    // getHeight / firstChunkAtLevel: lane l reads level l's counter.
+    const int32_t c = (lane < N) ? d.counter[lane] : 0;
+    const uint32_t b = __ballot_sync(FULL, lane >= 1 && lane < N && c > 0);
+    const uint32_t h = b ? 31u - __clz(b) : 0u;
+    if (lane == 0) {
+      s_height = h;
+      s_start = d.head[h];
+      if (blockIdx.x == 0) ctl->snap_height = h;
+    }
+  }
+  __syncthreads();
+  const uint32_t start = s_start;
+  const int height = (int)s_height;
+  const uint32_t nc = ctl->n_contains;
+  const uint32_t n = nc + ctl->n_updates;
+
+  const int team_in_warp = lane / TEAM;
+  const int t = lane - team_in_warp * TEAM;          // tId
+  const bool lane_live = team_in_warp < TPW;         // lanes past TPW*TEAM idle
+  const int team_base = lane_live ? team_in_warp * TEAM : lane;
+  const uint32_t warp_global = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  const uint32_t total_teams = (gridDim.x * blockDim.x >> 5) * TPW;
+  const int next_src = lane_live ? team_base + NEXT_LANE : lane;
+
+  // op slot s: s < nc -> list_c[s]; else update op list_u[s - nc].  One op prefetched.
+  auto load_op = [&](uint32_t sl) -> uint2 {
+    if (!lane_live || sl >= n) return make_uint2(0xFFFFFFFFu, 0u);
+    return sl < nc ? list_c[sl] : list_u[sl - nc];
+  };
+  uint32_t slot = warp_global * TPW + team_in_warp;  // this team's current op slot
+  uint2 cur_op = load_op(slot);
+  uint2 nxt_op = load_op(slot + total_teams);
+  bool active = lane_live && slot < n;
+  uint32_t k = cur_op.y;
+  uint32_t cur = start;
+  int level = height;
+  uint32_t bt = NULL_CHUNK, bt_c = NULL_CHUNK;       // prevKv, reduced
+  int seen_top = 0;                                  // highest level where k was seen
+  unsigned long long restarts = 0;
+  unsigned long long reads = 0, reads_l0 = 0, nops = 0;  // COUNT build only
+
+  while (__any_sync(FULL, active)) {
+    ChunkSlice<EPL> s;
+    ld_slice_nc<EPL>(d.pool + (size_t)cur * N + t * EPL, s);  // idle teams re-read `cur`
+    if (COUNT && active) {
+      ++reads;
+      reads_l0 += (level == 0);
+    }
+    // Per-lane part of the vote.  Upper levels: DATA key <= k (Alg 4.3 l.3); bottom
+    // level: DATA key == k (Alg 4.4 l.4).  EMPTY (+inf) never votes.
+    int bj = -1;
+    uint32_t dv = 0;
+#pragma unroll
+    for (int j = 0; j < EPL; ++j) {
+      const bool data = (t * EPL + j) < DSIZE;
+      const bool v = data && (level == 0 ? s.k[j] == k : s.k[j] <= k);
+      if (v) {
+        bj = j;
+        dv = s.v[j] | (s.k[j] == k ? F_EQUAL : 0u);
+      }
+    }
+    // NEXT / LOCK entries: lateral flags packed on the next pointer
+    uint32_t nx = s.v[NEXT_J] & PTR_MASK;  // NULL (last chunk) is never followed
+    if (t == NEXT_LANE && s.k[NEXT_J] < k) nx |= F_LATERAL;
+    if (t == LOCK_LANE && s.k[LOCK_J] == LOCK_ZOMBIE) nx |= F_ZOMBIE;
+    if (LOCK_LANE != NEXT_LANE) nx |= __shfl_down_sync(FULL, nx & F_ZOMBIE, 1);
+
+    const uint32_t bd = __ballot_sync(FULL, active && bj >= 0);
+    const uint32_t tb = (bd >> (team_base & 31)) & TEAM_BITS;
+    const int src = tb ? team_base + 31 - __clz(tb) : lane;
+    const uint32_t dptr = __shfl_sync(FULL, dv, src);
+    const uint32_t np = __shfl_sync(FULL, nx, next_src);
+
+    if (active) {
+      if (np & (F_ZOMBIE | F_LATERAL)) {
+        // zombie: lateral, prevKv unchanged (Alg 4.2 l.9-11); else lateral step (l.15-18)
+        if (!(np & F_ZOMBIE) && level > 0) {
+          bt = tb ? (dptr & PTR_MASK) : NULL_CHUNK;
+          bt_c = cur;
+        }
+        cur = np & PTR_MASK;
+      } else if (level == 0) {         // bottom enclosing chunk reached (Alg 4.4 l.12)
+        const bool te = tb != 0;
+        const uint32_t opi = cur_op.x & OPI_MASK;
+        if (t == 0) {
+          if (slot < nc) {
+            res[opi] = te ? 1 : 0;
+          } else {
+            // Alg 4.5 l.3-4 / Alg 4.11 l.4-5 on the snapshot: exact under the contract
+            const uint32_t u = slot - nc;
+            const bool mut = (cur_op.x & DELETE_FLAG) ? te : !te;
+            res[opi] = mut ? 1 : 0;
+            so.plan_path[(size_t)u * PLAN_LEVELS] = cur;   // path[0] = enclosing chunk
+            so.plan_top[u] = mut ? (uint8_t)seen_top : (uint8_t)0xFF;
+            if (mut) so.mut_list[atomicAdd(&ctl->n_mut, 1u)] = u;
+          }
+        }
+        if (COUNT) ++nops;
+        // next op of this team (prefetched)
+        slot += total_teams;
+        active = slot < n;
+        cur_op = nxt_op;
+        k = cur_op.y;
+        nxt_op = load_op(slot + total_teams);
+        cur = start;
+        level = height;
+        bt = bt_c = NULL_CHUNK;
+        seen_top = 0;
+      } else {
+        const bool upd = slot >= nc;
+        if (tb || bt != NULL_CHUNK) {  // down step (l.19-23) or backtrack (l.26-27)
+          if (upd && t == 0 && level < PLAN_LEVELS)  // searchSlow's path (Alg 4.6 l.28-29, 36-37)
+            so.plan_path[(size_t)(slot - nc) * PLAN_LEVELS + level] = tb ? cur : bt_c;
+          if (tb && (dptr & F_EQUAL) && seen_top == 0) seen_top = level;
+          cur = tb ? (dptr & PTR_MASK) : bt;
+          --level;
+          bt = bt_c = NULL_CHUNK;
+        } else {                       // restart (l.25); impossible on a quiescent structure
+          ++restarts;
+          cur = start;
+          level = height;
+          seen_top = 0;
+        }
+      }
+    }
+  }
+  if (restarts && t == 0) stat_add(d, ST_RESTARTS, restarts);
+  if (COUNT && t == 0 && lane_live) {
+    stat_add(d, ST_CREADS, reads);
+    stat_add(d, ST_CREADS_L0, reads_l0);
+    stat_add(d, ST_COPS, nops);
+  }
+}
+
+}  // namespace gfsl_dev
