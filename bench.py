@@ -209,12 +209,17 @@ def make_inputs(w: Workload, b: int, dev):
 
 
 def prefill_gpu(g, R, count, dev, chunk=1 << 24, key_lo=0, seed=SEED_BASE):
-    for s in range(0, count, chunk):
-        c = min(chunk, count - s)
+    """Random-order inserts in insert-only batches that grow with the structure
+    (a batch never exceeds ~1/4 of the keys already present, so concurrent inserts spread
+    over many chunks instead of queueing on the few chunks of a small structure)."""
+    s = 0
+    while s < count:
+        c = min(chunk, count - s, max(4096, s // 4))
         k = prefill_keys(seed, R, c, start=s, device=dev) + key_lo
         v = prefill_values(seed, k)
         g.batch(torch.ones(c, dtype=torch.uint8, device=dev), k.to(torch.int32),
                 v.to(torch.int32))
+        s += c
     torch.cuda.synchronize()
 
 
@@ -251,6 +256,7 @@ def run_gpu(args, world, rank, local):
     barrier(world)
     local_g = g.local if world > 1 else g
     local_g.phase_times()  # reset the per-phase sums
+    mut0 = local_g.stats()["mutations"]
 
     starts = [torch.cuda.Event(enable_timing=True) for _ in range(steps)]
     ends = [torch.cuda.Event(enable_timing=True) for _ in range(steps)]
@@ -274,6 +280,7 @@ def run_gpu(args, world, rank, local):
     ops_total = B1 * steps * world
     mops = ops_total / (total_ms / 1e3) / 1e6
     phases, nbat = local_g.phase_times()
+    n_mut = (local_g.stats()["mutations"] - mut0) / max(steps, 1)
 
     # algorithmic bytes: chunk reads per Contains op, counted on a Contains-only replay
     # of the last timed batch's keys (untimed, non-mutating)
@@ -291,29 +298,29 @@ def run_gpu(args, world, rank, local):
     reads_per_op = (st1["contains_reads"] - st0["contains_reads"]) / cops
     reads_l0_per_op = (st1["contains_reads_l0"] - st0["contains_reads_l0"]) / cops
 
-    n_contains = int(round(B1 * mix[2] / 100.0))
-    n_update = B1 - n_contains
+    n_search = B1  # the search kernel traverses every valid op of the batch
     c_ms = phases["contains"] / max(nbat, 1)
     u_ms = phases["update"] / max(nbat, 1)
     i_ms = phases["intake"] / max(nbat, 1)
-    def roof(bytes_per_launch, ms):
+
+    def roof(bytes_per_launch, ms, kernel):
         if ms <= 0 or bytes_per_launch <= 0:
             return None
         ach = bytes_per_launch / (ms / 1e3) / 1e9
         return {"bound": "hbm", "achieved": round(ach, 1), "peak": hbm_peak, "unit": "GB/s",
-                "frac": round(ach / hbm_peak, 4), "traffic": None,
-                "peak_kind": peak_kind}
-    # Contains: every chunk gather of the traversal is C_b random bytes
-    c_bytes = n_contains * reads_per_op * Cb
-    # update: the traversal (same chunk reads) + the entries written (~DSIZE/2 + NEXT/LOCK)
-    u_bytes = n_update * (reads_per_op * Cb + (N // 2) * 8 * 2)
-    roof_c = roof(c_bytes, c_ms)
-    roof_u = roof(u_bytes, u_ms)
-    dominant = "contains" if c_ms >= u_ms else "update"
-    roofline = roof_c if dominant == "contains" else roof_u
-    if roofline is not None:
-        roofline["kernel"] = dominant
-        roofline["algorithmic_bytes_per_launch"] = int(c_bytes if dominant == "contains" else u_bytes)
+                "frac": round(ach / hbm_peak, 4), "traffic": None, "peak_kind": peak_kind,
+                "kernel": kernel, "algorithmic_bytes_per_launch": int(bytes_per_launch)}
+    # search kernel: SURVEY 8(d) -- the compulsory DRAM bytes of a traversal are its
+    # bottom-level chunk gathers (upper levels are cache-resident): L0 reads x C_b
+    s_bytes = n_search * reads_l0_per_op * Cb
+    # update kernel: per mutation one chunk read under the lock + the entries written
+    u_bytes = n_mut * (Cb + 8 * (N // 2 + 2))
+    roof_c = roof(s_bytes, c_ms, "search")
+    roof_u = roof(u_bytes, u_ms, "update")
+    roofline = roof_c if c_ms >= u_ms else roof_u
+    gather = {"chunk_gathers_per_op": round(reads_per_op, 3),
+              "gather_GBps": round(n_search * reads_per_op * Cb / (c_ms / 1e3) / 1e9, 1) if c_ms > 0 else None,
+              "note": "all chunk gathers of the search kernel incl. L1/L2-resident upper levels"}
 
     # end to end through the C ABI with host buffers (fresh handle, same sequence)
     e2e = None
@@ -359,8 +366,10 @@ def run_gpu(args, world, rank, local):
                        "l2": "flushed (256 MiB write) between timed steps",
                        "parallelism": f"range-shard x{world}" if world > 1 else "1 GPU"},
             "roofline": roofline,
-            "roofline_kernels": {"contains": roof_c, "update": roof_u},
-            "phase_ms_per_step": {"intake": round(i_ms, 4), "contains": round(c_ms, 4),
+            "roofline_kernels": {"search": roof_c, "update": roof_u},
+            "search_gathers": gather,
+            "mutations_per_step": round(n_mut, 1),
+            "phase_ms_per_step": {"intake": round(i_ms, 4), "search": round(c_ms, 4),
                                   "update": round(u_ms, 4)},
             "chunk_reads_per_contains": round(reads_per_op, 3),
             "chunk_reads_l0_per_contains": round(reads_l0_per_op, 3),

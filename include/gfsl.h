@@ -157,7 +157,8 @@ typedef struct gfsl_stats {
   uint64_t contains_reads;  /* chunk reads by Contains traversals (count_reads=1) */
   uint64_t contains_reads_l0; /* ... of which on the bottom level */
   uint64_t contains_ops;    /* Contains ops counted (count_reads=1) */
-  uint64_t reserved[5];
+  uint64_t mutations;       /* Insert/Delete ops that changed the map */
+  uint64_t reserved[4];
 } gfsl_stats;
 gfsl_status gfsl_get_stats(gfsl_t h, gfsl_stats *out);
 

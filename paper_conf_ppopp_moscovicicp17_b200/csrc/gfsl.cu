@@ -556,6 +556,7 @@ extern "C" gfsl_status gfsl_get_stats(gfsl_t h, gfsl_stats *out) {
   out->contains_reads = s[ST_CREADS];
   out->contains_reads_l0 = s[ST_CREADS_L0];
   out->contains_ops = s[ST_COPS];
+  out->mutations = s[ST_MUTATIONS];
   return GFSL_OK;
 }
 

@@ -37,6 +37,7 @@ enum StatSlot {
   ST_CREADS,      // chunk reads of Contains traversals (counting build only)
   ST_CREADS_L0,   // ... of which on the bottom level
   ST_COPS,        // Contains ops counted
+  ST_MUTATIONS,   // ops the update kernel applied (all batches)
   ST_NSTATS
 };
 

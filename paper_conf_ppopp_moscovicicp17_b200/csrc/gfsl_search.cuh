@@ -117,57 +117,78 @@ search_kernel(DevState d, uint8_t *__restrict__ res, const uint2 *__restrict__ l
       ++reads;
       reads_l0 += (level == 0);
     }
-    // Per-lane part of the vote.  Upper levels: DATA key <= k (Alg 4.3 l.3); bottom
-    // level: DATA key == k (Alg 4.4 l.4).  EMPTY (+inf) never votes.
-    int bj = -1;
-    uint32_t dv = 0;
+    // NEXT / LOCK entries: the lateral and zombie flags ride on the next pointer; their
+    // keys are replaced by EMPTY so that they never take part in the DATA vote.
+    uint32_t nx = s.v[NEXT_J] & PTR_MASK;  // NULL (last chunk) is never followed
+    if (t == NEXT_LANE) {
+      if (s.k[NEXT_J] < k) nx |= F_LATERAL;  // NEXT votes max < k (Alg 4.3 l.4)
+      s.k[NEXT_J] = KEY_EMPTY;
+    }
+    if (t == LOCK_LANE) {
+      if (s.k[LOCK_J] == LOCK_ZOMBIE) nx |= F_ZOMBIE;
+      s.k[LOCK_J] = KEY_EMPTY;
+    }
+    if (LOCK_LANE != NEXT_LANE) nx |= __shfl_down_sync(FULL, nx & F_ZOMBIE, 1);
+    // DATA vote as one unsigned range test klo <= key <= k: klo = 0 above the bottom
+    // level (key <= k, Alg 4.3 l.3), klo = k on it (key == k, Alg 4.4 l.4).  EMPTY
+    // (+inf) never votes.  Keys ascend within a lane: the last voter is the highest.
+    const uint32_t klo = level == 0 ? k : 0u;
+    const uint32_t span = k - klo;
+    bool any = false;
+    uint32_t dv = 0, dk = 0;
 #pragma unroll
     for (int j = 0; j < EPL; ++j) {
-      const bool data = (t * EPL + j) < DSIZE;
-      const bool v = data && (level == 0 ? s.k[j] == k : s.k[j] <= k);
-      if (v) {
-        bj = j;
-        dv = s.v[j] | (s.k[j] == k ? F_EQUAL : 0u);
-      }
+      const bool v = (s.k[j] - klo) <= span;
+      any |= v;
+      dv = v ? s.v[j] : dv;
+      dk = v ? s.k[j] : dk;
     }
-    // NEXT / LOCK entries: lateral flags packed on the next pointer
-    uint32_t nx = s.v[NEXT_J] & PTR_MASK;  // NULL (last chunk) is never followed
-    if (t == NEXT_LANE && s.k[NEXT_J] < k) nx |= F_LATERAL;
-    if (t == LOCK_LANE && s.k[LOCK_J] == LOCK_ZOMBIE) nx |= F_ZOMBIE;
-    if (LOCK_LANE != NEXT_LANE) nx |= __shfl_down_sync(FULL, nx & F_ZOMBIE, 1);
+    dv |= (dk == k) ? F_EQUAL : 0u;
 
-    const uint32_t bd = __ballot_sync(FULL, active && bj >= 0);
+    const uint32_t bd = __ballot_sync(FULL, active && any);
     const uint32_t tb = (bd >> (team_base & 31)) & TEAM_BITS;
     const int src = tb ? team_base + 31 - __clz(tb) : lane;
     const uint32_t dptr = __shfl_sync(FULL, dv, src);
     const uint32_t np = __shfl_sync(FULL, nx, next_src);
 
     if (active) {
-      if (np & (F_ZOMBIE | F_LATERAL)) {
-        // zombie: lateral, prevKv unchanged (Alg 4.2 l.9-11); else lateral step (l.15-18)
-        if (!(np & F_ZOMBIE) && level > 0) {
-          bt = tb ? (dptr & PTR_MASK) : NULL_CHUNK;
-          bt_c = cur;
-        }
-        cur = np & PTR_MASK;
-      } else if (level == 0) {         // bottom enclosing chunk reached (Alg 4.4 l.12)
+      const bool lat = (np & (F_ZOMBIE | F_LATERAL)) != 0;  // zombie (l.9-11) / lateral (l.15-18)
+      const bool done = !lat && level == 0;                 // bottom enclosing chunk (Alg 4.4)
+      const bool down = !lat && level > 0;                  // down step (l.19-23) / backtrack
+      const bool restart = down && !tb && bt == NULL_CHUNK; // (l.25) impossible when quiescent
+      const bool upd = slot >= nc;
+      const uint32_t here = cur;
+      if (down && upd && t == 0 && level < PLAN_LEVELS)     // searchSlow's path (Alg 4.6 l.28-37)
+        so.plan_path[(size_t)(slot - nc) * PLAN_LEVELS + level] = tb ? cur : bt_c;
+      if (down && tb && (dptr & F_EQUAL) && seen_top == 0) seen_top = level;
+      const bool set_bt = lat && !(np & F_ZOMBIE) && level > 0;  // prevKv = currKv (l.16)
+      const uint32_t next_cur = lat ? (np & PTR_MASK) : (tb ? (dptr & PTR_MASK) : bt);
+      bt = set_bt ? (tb ? (dptr & PTR_MASK) : NULL_CHUNK) : (down ? NULL_CHUNK : bt);
+      bt_c = set_bt ? cur : (down ? NULL_CHUNK : bt_c);
+      cur = restart ? start : next_cur;
+      level = restart ? height : level - (down ? 1 : 0);
+      if (restart) {
+        ++restarts;
+        seen_top = 0;
+      }
+      if (done) {
         const bool te = tb != 0;
         const uint32_t opi = cur_op.x & OPI_MASK;
         if (t == 0) {
-          if (slot < nc) {
+          if (!upd) {
             res[opi] = te ? 1 : 0;
           } else {
             // Alg 4.5 l.3-4 / Alg 4.11 l.4-5 on the snapshot: exact under the contract
             const uint32_t u = slot - nc;
             const bool mut = (cur_op.x & DELETE_FLAG) ? te : !te;
             res[opi] = mut ? 1 : 0;
-            so.plan_path[(size_t)u * PLAN_LEVELS] = cur;   // path[0] = enclosing chunk
+            so.plan_path[(size_t)u * PLAN_LEVELS] = here;  // path[0] = enclosing chunk
             so.plan_top[u] = mut ? (uint8_t)seen_top : (uint8_t)0xFF;
             if (mut) so.mut_list[atomicAdd(&ctl->n_mut, 1u)] = u;
           }
         }
         if (COUNT) ++nops;
-        // next op of this team (prefetched)
+        // next op of this team (prefetched one ahead)
         slot += total_teams;
         active = slot < n;
         cur_op = nxt_op;
@@ -177,21 +198,6 @@ search_kernel(DevState d, uint8_t *__restrict__ res, const uint2 *__restrict__ l
         level = height;
         bt = bt_c = NULL_CHUNK;
         seen_top = 0;
-      } else {
-        const bool upd = slot >= nc;
-        if (tb || bt != NULL_CHUNK) {  // down step (l.19-23) or backtrack (l.26-27)
-          if (upd && t == 0 && level < PLAN_LEVELS)  // searchSlow's path (Alg 4.6 l.28-29, 36-37)
-            so.plan_path[(size_t)(slot - nc) * PLAN_LEVELS + level] = tb ? cur : bt_c;
-          if (tb && (dptr & F_EQUAL) && seen_top == 0) seen_top = level;
-          cur = tb ? (dptr & PTR_MASK) : bt;
-          --level;
-          bt = bt_c = NULL_CHUNK;
-        } else {                       // restart (l.25); impossible on a quiescent structure
-          ++restarts;
-          cur = start;
-          level = height;
-          seen_top = 0;
-        }
       }
     }
   }

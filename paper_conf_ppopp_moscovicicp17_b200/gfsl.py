@@ -49,7 +49,7 @@ class gfsl_stats(ctypes.Structure):
                 ("merges", ctypes.c_uint64), ("zombie_unlinks", ctypes.c_uint64),
                 ("lock_retries", ctypes.c_uint64), ("contains_reads", ctypes.c_uint64),
                 ("contains_reads_l0", ctypes.c_uint64), ("contains_ops", ctypes.c_uint64),
-                ("reserved", ctypes.c_uint64 * 5)]
+                ("mutations", ctypes.c_uint64), ("reserved", ctypes.c_uint64 * 4)]
 
 
 class gfsl_meta(ctypes.Structure):
