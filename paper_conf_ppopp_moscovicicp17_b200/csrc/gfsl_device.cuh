@@ -104,6 +104,15 @@ __device__ __forceinline__ uint64_t cas_acquire(uint64_t *p, uint64_t cmp, uint6
                : "memory");
   return old;
 }
+// 32-bit CAS with acquire on the lock-state half (lo32) of a LOCK entry.
+__device__ __forceinline__ uint32_t cas32_acquire(uint64_t *p, uint32_t cmp, uint32_t val) {
+  uint32_t old;
+  asm volatile("atom.acquire.gpu.global.cas.b32 %0, [%1], %2, %3;"
+               : "=r"(old)
+               : "l"(p), "r"(cmp), "r"(val)
+               : "memory");
+  return old;
+}
 __device__ __forceinline__ void st_relaxed(uint64_t *p, uint64_t v) {
   asm volatile("st.relaxed.gpu.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
 }
