@@ -1,0 +1,511 @@
+"""Oracle-B: the GFSL algorithm of PAPER.md §4, step by step, one team, no concurrency.
+
+TEST INFRASTRUCTURE ONLY (see oracle/__init__.py).  Plain Python, written from the paper
+and the readings R1-R22 of DESIGN.md §3; it shares no code with the CUDA path.  It exists
+because the exact *structure* (not only the results) is defined for a single team: the
+GPU's serial mode (one team applies the batch's updates in op order) must produce the
+same pool, entry for entry, except the lock versions (test_gpu_structure.py).
+
+Pinned by (tests/test_oracle_b.py): the worked examples of Fig 4.1-4.6 (P:287-289,
+P:429) on the fixtures of SURVEY
+Appendix B; Oracle-A's results and final sets on random sequences; its own invariant
+checker; the special case "one chunk holds everything" (a sorted array).
+
+Layout (Fig 3.1): chunk = N entries of 64 bits; DATA i = key | value << 32,
+NEXT = max | next << 32, LOCK = state | version << 32.  Internal key = user key + 1;
+-inf = 0; +inf = EMPTY = null = 0xFFFFFFFF (R3).  Level-0 chunks come from the bottom
+pool, chunks of levels >= 1 from the upper pool (R18); every pool chunk starts in the
+allocated state of P:237 (all +inf, locked).
+"""
+from __future__ import annotations
+
+NEG_INF = 0
+INF = 0xFFFFFFFF
+EMPTY = 0xFFFFFFFFFFFFFFFF
+NULL = 0xFFFFFFFF
+FREE, HELD, ZOMBIE = 0, 1, 2
+PLAN_LEVELS = 16
+
+
+def K(e):  # key (or max / lock state) half of an entry
+    return e & 0xFFFFFFFF
+
+
+def V(e):  # value (or next / version) half of an entry
+    return e >> 32
+
+
+def E(k, v):
+    return (k & 0xFFFFFFFF) | ((v & 0xFFFFFFFF) << 32)
+
+
+class PoolExhausted(Exception):
+    pass
+
+
+class GFSLModel:
+    def __init__(self, N: int, key_range: int, cap_bottom: int, cap_upper: int):
+        assert N >= 6
+        self.N, self.DSIZE, self.NEXT, self.LOCK, self.MAXL = N, N - 2, N - 2, N - 1, N
+        self.key_range = key_range
+        self.cap_bottom, self.cap_upper = cap_bottom, cap_upper
+        # every chunk is allocated locked with +inf everywhere
+        self.pool = [[EMPTY] * (N - 1) + [HELD] for _ in range(cap_upper + cap_bottom)]
+        self.head = [NULL] * 32
+        self.counter = [0] * 32
+        # one unlocked chunk per level holding -inf with a pointer to the level below
+        for l in range(N):
+            c = cap_upper if l == 0 else l - 1
+            below = 0 if l == 0 else (cap_upper if l == 1 else l - 2)
+            ch = self.pool[c]
+            ch[0] = E(NEG_INF, below)
+            ch[self.NEXT] = E(INF, NULL)
+            ch[self.LOCK] = E(FREE, 0)
+            self.head[l] = c
+        self.bump = [1, N - 1]  # [bottom pool, upper pool]
+        self.trace = None       # chunks read by the last search (for the worked examples)
+
+    # ---- chunk accessors ----------------------------------------------------------------
+    def keys(self, c):
+        return [K(e) for e in self.pool[c][: self.DSIZE]]
+
+    def mx(self, c):
+        return K(self.pool[c][self.NEXT])
+
+    def nxt(self, c):
+        return V(self.pool[c][self.NEXT])
+
+    def state(self, c):
+        return K(self.pool[c][self.LOCK])
+
+    def zombie(self, c):
+        return self.state(c) == ZOMBIE
+
+    def count(self, c):  # numNonEmpty (Alg 4.12 l.3): -inf counts (R8)
+        return sum(1 for k in self.keys(c) if k != INF)
+
+    def eq_idx(self, c, k):  # isTidWithEqualKey (Alg 4.4)
+        ks = self.keys(c)
+        for i in range(self.DSIZE - 1, -1, -1):
+            if ks[i] == k:
+                return i
+        return None
+
+    def le_idx(self, c, k):  # highest DATA index with key <= k (Alg 4.3, DATA votes)
+        ks = self.keys(c)
+        for i in range(self.DSIZE - 1, -1, -1):
+            if ks[i] <= k:
+                return i
+        return None
+
+    def height(self):  # getHeight
+        h = 0
+        for l in range(1, self.N):
+            if self.counter[l] > 0:
+                h = l
+        return h
+
+    # ---- locks (serial: a lock is never found held by someone else) ---------------------
+    def lock(self, c):
+        assert self.state(c) == FREE
+        ch = self.pool[c]
+        ch[self.LOCK] = E(HELD, V(ch[self.LOCK]))
+
+    def unlock(self, c, state=FREE):
+        ch = self.pool[c]
+        ch[self.LOCK] = E(state, V(ch[self.LOCK]) + 1)
+
+    def alloc(self, level):  # bump a counter, the chunk is already +inf and locked
+        p = 1 if level > 0 else 0
+        cap = self.cap_upper if p else self.cap_bottom
+        i = self.bump[p]
+        if i >= cap:
+            raise PoolExhausted
+        self.bump[p] += 1
+        return i if p else self.cap_upper + i
+
+    # ---- search phase (Alg 4.1-4.4 and searchSlow's path, on the snapshot; R1, R21) ------
+    def search(self, k):
+        """Returns (found, path{level: chunk}, top level that held k)."""
+        height = self.height()
+        cur, level = self.head[height], height
+        bt = bt_c = None
+        top = 0
+        path = {}
+        self.trace = []
+        while True:
+            self.trace.append(cur)
+            if self.zombie(cur):                      # Alg 4.2 l.9-11
+                cur = self.nxt(cur)
+                continue
+            w = self.le_idx(cur, k) if level > 0 else None
+            if self.mx(cur) < k:                      # lateral step (l.15-18)
+                if level > 0:
+                    bt = None if w is None else V(self.pool[cur][w])
+                    bt_c = cur
+                cur = self.nxt(cur)
+                continue
+            if level == 0:                            # searchLateral result (Alg 4.4)
+                path[0] = cur
+                return self.eq_idx(cur, k) is not None, path, top
+            if w is not None:                         # down step (l.19-23)
+                path[level] = cur
+                if self.keys(cur)[w] == k and top == 0:
+                    top = level
+                cur = V(self.pool[cur][w])
+            elif bt is not None:                      # backtrack (l.24-28, 33-38)
+                path[level] = bt_c
+                cur = bt
+            else:                                     # restart (l.25): not on a snapshot
+                raise AssertionError("restart on a quiescent structure")
+            level -= 1
+            bt = bt_c = None
+
+    def search_down_to_level(self, L, k):  # Alg 4.10 l.4
+        height = self.height()
+        if height <= L:
+            return self.head[L]
+        cur, level, prev = self.head[height], height, None
+        while level > L:
+            if self.zombie(cur):
+                cur = self.nxt(cur)
+                continue
+            if self.mx(cur) < k:
+                prev = cur
+                cur = self.nxt(cur)
+                continue
+            w = self.le_idx(cur, k)
+            if w is not None:
+                cur = V(self.pool[cur][w])
+            else:
+                assert prev is not None
+                cur = V(self.pool[prev][self.le_idx(prev, k)])
+            level -= 1
+            prev = None
+        return cur
+
+    # ---- findAndLockEnclosing (Alg 4.8) with the lazy zombie redirect (Alg 4.6, R15, R21) -
+    def first_non_zombie(self, z):
+        c = self.nxt(z)
+        while self.zombie(c):
+            c = self.nxt(c)
+        return c
+
+    def redirect_zombie(self, prev, z, fnz):  # Alg 4.6 l.13-14 (try-lock succeeds serially)
+        if self.zombie(prev) or self.nxt(prev) != z or self.state(prev) != FREE:
+            return
+        self.lock(prev)
+        if self.nxt(prev) == z:
+            self.pool[prev][self.NEXT] = E(self.mx(prev), fnz)
+        self.unlock(prev)
+
+    def find_and_lock_enclosing(self, c, k, level):
+        prev = None
+        while True:
+            if self.state(c) == FREE:                 # optimistic lock, validated under it
+                self.lock(c)
+                if self.mx(c) < k:                    # l.17-21
+                    nx = self.nxt(c)
+                    self.unlock(c)
+                    prev, c = c, nx
+                    continue
+                return c
+            if self.zombie(c):
+                fnz = self.first_non_zombie(c)
+                if prev is not None:
+                    self.redirect_zombie(prev, c, fnz)
+                elif level >= 0 and c == self.head[level]:
+                    self.head[level] = fnz            # updateHeadArray (Alg 4.6 l.15)
+                c = fnz
+            if self.mx(c) < k:                        # chunkNotEnclosing (l.5-8)
+                prev, c = c, self.nxt(c)
+                continue
+            assert self.state(c) == FREE, "serial model: lock held"
+
+    def lock_next_chunk(self, c):  # Alg 4.9 l.17 / Alg 4.12 l.9
+        n = self.nxt(c)
+        skipped = False
+        while n != NULL:
+            if self.zombie(n):
+                n = self.nxt(n)
+                skipped = True
+                continue
+            if skipped:  # unlink the zombies from c's NEXT (we hold c)
+                self.pool[c][self.NEXT] = E(self.mx(c), n)
+            self.lock(n)
+            return n
+        return None
+
+    # ---- the chunk operations ---------------------------------------------------------
+    def execute_insert(self, c, k, v):  # Alg 4.7, Fig 4.3: shift right from insertIdx
+        ch = self.pool[c]
+        ks = self.keys(c)
+        idx = sum(1 for x in ks if x < k)
+        cnt = self.count(c)
+        old = ch[:]
+        for t in range(idx, min(cnt, self.DSIZE - 1) + 1):
+            ch[t] = E(k, v) if t == idx else old[t - 1]
+
+    def execute_remove_no_merge(self, c, k):  # P:900-902, Fig 4.6, R13
+        ch = self.pool[c]
+        idx = self.eq_idx(c, k)
+        cnt = self.count(c)
+        last = self.nxt(c) == NULL
+        old = ch[:]
+        for t in range(idx, cnt - 1):
+            ch[t] = old[t + 1]
+        ch[cnt - 1] = EMPTY
+        if idx == cnt - 1 and not last:  # the max follows the largest key
+            ch[self.NEXT] = E(K(old[idx - 1]), V(old[self.NEXT]))
+
+    def split(self, level, c):  # Alg 4.9 preSplit + splitCopy (also splitRemove)
+        HALF = self.DSIZE // 2
+        pnext = self.lock_next_chunk(c)
+        pnew = self.alloc(level)
+        ch, nw = self.pool[c], self.pool[pnew]
+        cnt = self.count(c)
+        thresh = K(ch[HALF - 1])
+        oldmax = self.mx(c)
+        for t in range(cnt - HALF):
+            nw[t] = ch[t + HALF]
+        nw[self.NEXT] = E(oldmax, NULL if pnext is None else pnext)
+        ch[self.NEXT] = E(thresh, pnew)               # one 64-bit write links the new chunk
+        for t in range(HALF, cnt):
+            ch[t] = EMPTY                             # setMovedValsEmpty
+        if pnext is not None:
+            self.unlock(pnext)
+        self.counter[level] += 1                      # Alg 4.5 l.42 / 4.12 l.18 (R9)
+        return pnew
+
+    def update_down_ptrs(self, level, moved, lower):  # Alg 4.10, R14
+        if level + 1 >= self.MAXL or not moved:
+            return
+        moved = list(moved)
+        upper = self.search_down_to_level(level + 1, moved[0])
+        lc = lower
+        while moved:
+            km0 = moved[0]
+            while self.zombie(upper) or self.mx(upper) < km0:
+                upper = self.nxt(upper)
+            umax = self.mx(upper)
+            here = [km for km in moved if km <= umax]
+            moved = [km for km in moved if km > umax]
+            if not any(self.eq_idx(upper, km) is not None for km in here):
+                continue
+            upper = self.find_and_lock_enclosing(upper, km0, level + 1)
+            for j, km in enumerate(here):
+                if km > self.mx(upper):
+                    moved = here[j:] + moved
+                    break
+                ui = self.eq_idx(upper, km)
+                if ui is None:
+                    continue
+                while self.zombie(lc) or self.mx(lc) < km:
+                    lc = self.nxt(lc)
+                if self.eq_idx(lc, km) is not None and V(self.pool[upper][ui]) != lc:
+                    self.pool[upper][ui] = E(km, lc)
+            self.unlock(upper)
+
+    # ---- Insert (Alg 4.5) ---------------------------------------------------------------
+    def insert_to_level(self, level, pe, k, v):
+        """Returns (ok, pins, pextra, raise, rkey, rptr); pins (and pextra) stay locked."""
+        pe = self.find_and_lock_enclosing(pe, k, level)   # l.30
+        if self.eq_idx(pe, k) is not None:                # l.32
+            return False, pe, None, False, 0, 0
+        if self.count(pe) < self.DSIZE:                   # l.35
+            first = self.keys(pe)[0] == NEG_INF
+            self.execute_insert(pe, k, v)                 # l.36
+            if first and self.counter[level] == 0:        # l.37-38 (R9: every level)
+                self.counter[level] = 1
+            return True, pe, None, False, 0, 0
+        HALF = self.DSIZE // 2
+        moved = self.keys(pe)[HALF:self.count(pe)]
+        thresh = self.keys(pe)[HALF - 1]
+        pnew = self.split(level, pe)
+        minK = self.keys(pnew)[0]
+        if k < thresh:                                    # insertNewData (Alg 4.9 l.4)
+            self.execute_insert(pe, k, v)
+            pins, other = pe, pnew
+        else:
+            self.execute_insert(pnew, k, v)
+            pins, other = pnew, pe
+        if level == 0:                                    # keyForNextLevel
+            rkey, rptr = max(k, minK), pnew               # R10
+            hold = pins != pnew                           # R11
+        else:
+            rkey, rptr, hold = k, pins, False
+        pextra = other if hold else None
+        if not hold:
+            self.unlock(other)                            # Alg 4.9 l.6-9
+        self.update_down_ptrs(level, moved, pnew)         # Alg 4.9 l.12
+        return True, pins, pextra, True, rkey, rptr       # p_chunk = 1 (R16)
+
+    def insert(self, k, v, path):
+        ok, pins, pextra, raise_, rkey, rptr = self.insert_to_level(0, path[0], k, v)
+        if not ok:
+            self.unlock(pins)
+            return False
+        level = 1
+        while raise_ and level < self.MAXL:               # Alg 4.5 l.15-22
+            ok2, p2, _, r2, rk2, rp2 = self.insert_to_level(level, path[level], rkey, rptr)
+            self.unlock(p2)
+            raise_ = ok2 and r2                           # R19
+            rkey, rptr = rk2, rp2
+            level += 1
+        if pextra is not None:
+            self.unlock(pextra)
+        self.unlock(pins)
+        return True
+
+    # ---- Delete (Alg 4.11-4.12) -----------------------------------------------------------
+    def execute_remove_merge(self, e, f, k):
+        idx = self.eq_idx(e, k)
+        eent = [x for i, x in enumerate(self.pool[e][: self.count(e)]) if i != idx]
+        fent = self.pool[f][: self.count(f)]
+        for t, x in enumerate(eent + fent):
+            self.pool[f][t] = x
+
+    def remove_from_chunk(self, level, pe, k):
+        cnt = self.count(pe)
+        only_neg_inf_after = cnt == 2 and self.keys(pe)[0] == NEG_INF
+        if cnt > self.DSIZE // 3:                         # l.4-7 (R8)
+            last = self.nxt(pe) == NULL
+            self.execute_remove_no_merge(pe, k)
+            if only_neg_inf_after and last:               # R17
+                self.counter[level] -= 1
+            self.unlock(pe)
+            return
+        pnext = self.lock_next_chunk(pe)                  # l.9
+        if pnext is None:                                 # l.10-13
+            self.execute_remove_no_merge(pe, k)
+            if only_neg_inf_after:
+                self.counter[level] -= 1
+            self.unlock(pe)
+            return
+        pg = None
+        g_moved = []
+        nf = self.count(pnext)
+        if nf + cnt - 1 > self.DSIZE:                     # l.16-19 splitRemove
+            HALF = self.DSIZE // 2
+            g_moved = self.keys(pnext)[HALF:nf]
+            pg = self.split(level, pnext)
+            self.unlock(pg)
+            nf = HALF
+        e_moved = [x for x in self.keys(pe)[:cnt] if x != k]
+        self.execute_remove_merge(pe, pnext, k)           # l.21
+        self.unlock(pe, ZOMBIE)                           # l.22 markAsZombie (R6)
+        self.counter[level] -= 1                          # l.24
+        if nf + cnt - 1 == 1 and self.nxt(pnext) == NULL and self.keys(pe)[0] == NEG_INF:
+            self.counter[level] -= 1                      # R17
+        self.unlock(pnext)                                # l.25
+        self.update_down_ptrs(level, e_moved, pnext)      # l.27
+        if pg is not None:
+            self.update_down_ptrs(level, g_moved, pg)
+
+    def search_lateral(self, k, c):  # Alg 4.4 (exact: no concurrency here)
+        while self.zombie(c) or self.mx(c) < k:
+            c = self.nxt(c)
+        return self.eq_idx(c, k) is not None
+
+    def delete(self, k, path, top):
+        pb = self.find_and_lock_enclosing(path[0], k, 0)  # l.8
+        if self.eq_idx(pb, k) is None:                    # l.9-10 (R15)
+            self.unlock(pb)
+            return False
+        m = top                                           # l.12-16 (R12)
+        while m + 1 < self.MAXL and self.search_lateral(k, path[m + 1]):
+            m += 1
+        for i in range(m, 0, -1):                         # l.13-20
+            pe = self.find_and_lock_enclosing(path[i], k, i)
+            if self.eq_idx(pe, k) is None:
+                self.unlock(pe)
+                continue
+            self.remove_from_chunk(i, pe, k)
+        self.remove_from_chunk(0, pb, k)                  # l.22
+        return True
+
+    # ---- a batch (R1: search phase on the snapshot, then the mutations in op order) -----
+    def batch(self, ops, keys, vals=None):
+        n = len(ops)
+        res = [0xFF] * n
+        snap_h = self.height()
+        plans = []
+        for i in range(n):
+            op, key = int(ops[i]), int(keys[i])
+            if op > 2 or key >= self.key_range:
+                continue
+            k = key + 1
+            found, path, top = self.search(k)
+            if op == 0:
+                res[i] = int(found)
+            else:
+                mut = (not found) if op == 1 else found
+                res[i] = int(mut)
+                if mut:
+                    plans.append((i, op, k, path, top))
+        head_at_start = list(self.head)  # levels above the snapshot height start at head[l]
+        for i, op, k, path, top in plans:
+            full = [path[l] if (l <= snap_h and l < PLAN_LEVELS) else head_at_start[l]
+                    for l in range(self.N)]
+            if op == 1:
+                r = self.insert(k, 0 if vals is None else int(vals[i]), full)
+            else:
+                r = self.delete(k, full, top)
+            if not r:
+                res[i] = 0
+        return res
+
+    # ---- views ------------------------------------------------------------------------
+    def level_chain(self, l):
+        out, c = [], self.head[l]
+        while c != NULL:
+            out.append(c)
+            c = self.nxt(c)
+        return out
+
+    def level_keys(self, l, with_values=False):
+        out = []
+        for c in self.level_chain(l):
+            if self.zombie(c):
+                continue
+            for e in self.pool[c][: self.DSIZE]:
+                if K(e) not in (INF, NEG_INF):
+                    out.append((K(e) - (1 if l == 0 else 0), V(e)) if with_values else K(e))
+        return out
+
+    def export(self):
+        kv = self.level_keys(0, with_values=True)
+        return [k for k, _ in kv], [v for _, v in kv]
+
+    def check_invariants(self):
+        """The structural invariants (§4.3); returns a list of violations."""
+        bad = []
+        for l in range(self.N):
+            chain = self.level_chain(l)
+            nz = [c for c in chain if not self.zombie(c)]
+            if chain and self.zombie(chain[-1]):
+                bad.append(f"V8 L{l}")
+            if not nz or self.keys(nz[0])[0] != NEG_INF:
+                bad.append(f"V9 L{l}")
+            prev_max = None
+            for c in nz:
+                ks = [k for k in self.keys(c) if k != INF]
+                if self.keys(c)[: len(ks)] != ks or sorted(set(ks)) != ks:
+                    bad.append(f"V1 L{l} c{c}")
+                if self.state(c) != FREE:
+                    bad.append(f"V7 L{l} c{c}")
+                if self.nxt(c) == NULL:
+                    if self.mx(c) != INF:
+                        bad.append(f"V2 L{l} c{c}")
+                elif not ks or self.mx(c) != ks[-1]:
+                    bad.append(f"V2 L{l} c{c}")
+                if ks and prev_max is not None and not prev_max < ks[0]:
+                    bad.append(f"V3 L{l} c{c}")
+                if ks:
+                    prev_max = ks[-1]
+            if l + 1 < self.N:
+                lower = set(self.level_keys(l))
+                for k in self.level_keys(l + 1):
+                    if k not in lower:
+                        bad.append(f"V4 L{l + 1} k{k}")
+        return bad
