@@ -51,6 +51,20 @@ CONFIGS = {
 L2_FLUSH_BYTES = 256 << 20
 
 
+def load_traffic(cfg):
+    """ncu DRAM bytes per launch of each kernel for this config (profiles/traffic_*.json)."""
+    import glob
+    for p in sorted(glob.glob(os.path.join(ROOT, "profiles", "traffic_r*.json")), reverse=True):
+        try:
+            with open(p) as f:
+                t = json.load(f)["traffic_bytes_per_launch"].get(cfg)
+            if t:
+                return t, os.path.basename(p)
+        except Exception:
+            pass
+    return {}, None
+
+
 def load_peaks():
     p = os.path.join(ROOT, "MEASURED_PEAKS.json")
     try:
@@ -317,6 +331,11 @@ def run_gpu(args, world, rank, local):
     u_bytes = n_mut * (Cb + 8 * (N // 2 + 2))
     roof_c = roof(s_bytes, c_ms, "search")
     roof_u = roof(u_bytes, u_ms, "update")
+    traffic, tsrc = load_traffic(args.config) if world == 1 else ({}, None)
+    for r, kname in ((roof_c, "search"), (roof_u, "update")):
+        if r is not None and traffic.get(kname) is not None:
+            r["traffic"] = int(traffic[kname])
+            r["traffic_source"] = f"profiles/{tsrc} (ncu, one launch of this config)"
     roofline = roof_c if c_ms >= u_ms else roof_u
     gather = {"chunk_gathers_per_op": round(reads_per_op, 3),
               "gather_GBps": round(n_search * reads_per_op * Cb / (c_ms / 1e3) / 1e9, 1) if c_ms > 0 else None,
