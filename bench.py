@@ -258,6 +258,8 @@ def run_gpu(args, world, rank, local):
     else:
         g = GFSL(R, capacity=R, chunk_entries=N, contains_team=args.team, profile_phases=True)
         prefill_gpu(g, R, pre1, dev)
+    if args.l2_window:
+        (g.local if world > 1 else g).configure(l2_window=1)
     w = Workload(R, B1, mix=mix, dist=dist, seed=SEED_BASE + 1 + 7919 * rank)
     inputs = [make_inputs(w, b, dev) for b in range(W + steps)]
     redraws = sum(x[3] for x in inputs)
@@ -337,6 +339,22 @@ def run_gpu(args, world, rank, local):
             r["traffic"] = int(traffic[kname])
             r["traffic_source"] = f"profiles/{tsrc} (ncu, one launch of this config)"
     roofline = roof_c if c_ms >= u_ms else roof_u
+    # B6: achievable random-access throughput for this chunk size, measured
+    # now on this GPU -- the denominator of the north star's ">= 40%" target
+    rand = None
+    if not args.no_ubench and rank == 0:
+        from paper_conf_ppopp_moscovicicp17_b200.gfsl import ubench
+        r_hbm, t_hbm = ubench(Cb, 16 << 30)
+        r_l2, t_l2 = ubench(Cb, 32 << 20)
+        rand = {"block_bytes": Cb, "R_rand_hbm_GBps": round(r_hbm, 1), "R_rand_l2_GBps": round(r_l2, 1),
+                "chase_latency_hbm_ns": round(t_hbm, 1), "chase_latency_l2_ns": round(t_l2, 1)}
+        for r in (roof_c, roof_u):
+            if r is not None:
+                r["frac_of_random_access_peak"] = round(r["achieved"] / r_hbm, 4)
+                if r.get("traffic"):
+                    ms_k = c_ms if r["kernel"] == "search" else u_ms
+                    r["dram_GBps_measured_traffic"] = round(r["traffic"] / (ms_k / 1e3) / 1e9, 1)
+                    r["frac_traffic_of_random_access_peak"] = round(r["dram_GBps_measured_traffic"] / r_hbm, 4)
     gather = {"chunk_gathers_per_op": round(reads_per_op, 3),
               "gather_GBps": round(n_search * reads_per_op * Cb / (c_ms / 1e3) / 1e9, 1) if c_ms > 0 else None,
               "note": "all chunk gathers of the search kernel incl. L1/L2-resident upper levels"}
@@ -387,6 +405,7 @@ def run_gpu(args, world, rank, local):
             "roofline": roofline,
             "roofline_kernels": {"search": roof_c, "update": roof_u},
             "search_gathers": gather,
+            "random_access_roofline": rand,
             "mutations_per_step": round(n_mut, 1),
             "phase_ms_per_step": {"intake": round(i_ms, 4), "search": round(c_ms, 4),
                                   "update": round(u_ms, 4)},
@@ -415,6 +434,9 @@ def main():
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--validate", action="store_true")
+    ap.add_argument("--no-ubench", action="store_true", help="skip the B6 roofline microbenchmark")
+    ap.add_argument("--l2-window", action="store_true",
+                    help="pin the upper-level pool in L2 (access-policy window; ablation)")
     args = ap.parse_args()
     if args.warmup < 3:
         args.warmup = 3

@@ -66,7 +66,9 @@ typedef struct gfsl_config {
                                measurement builds only, slower */
   uint32_t profile_phases;  /* 1 = record CUDA events between the phases of every batch
                                (read with gfsl_phase_times) */
-  uint32_t reserved[1];
+  uint32_t l2_window;       /* 1 = launch the search kernel with an L2 access-policy window
+                               marking the upper-level pool persisting (opt-in; see
+                               DESIGN.md §9 for why it is off by default) */
 } gfsl_config;
 
 /*
@@ -208,6 +210,15 @@ gfsl_status gfsl_route_pack(const uint32_t *perm, const uint8_t *op_types,
                             void *stream);
 gfsl_status gfsl_route_unpack(const uint32_t *perm, const uint8_t *recv_res, uint64_t n,
                               uint8_t *results, void *stream);
+
+/* ---- measurement: the roofline denominators of SURVEY 8(d) (B6) ----
+ * gfsl_ubench: random aligned `block_bytes` (256 or 128) gathers over a fresh device buffer
+ * of `buffer_bytes` (choose >> L2), issued like the search kernel's chunk reads (teams of
+ * 4 / 2 lanes, 32-B vector loads), many independent gathers per warp: *gather_gbps =
+ * R_rand(block).  *chase_ns = the latency of one dependent block gather.  Synchronous;
+ * allocates and frees the buffer itself. */
+gfsl_status gfsl_ubench(uint32_t block_bytes, uint64_t buffer_bytes, double *gather_gbps,
+                        double *chase_ns);
 
 #ifdef __cplusplus
 }

@@ -8,6 +8,7 @@
 #include <cuda_runtime.h>
 
 #include <algorithm>
+#include <cstdlib>
 #include <array>
 #include <cstdio>
 #include <cstring>
@@ -18,6 +19,7 @@
 #include "gfsl_search.cuh"
 #include "gfsl_device.cuh"
 #include "gfsl_update.cuh"
+#include "gfsl_ubench.cuh"
 
 using namespace gfsl_dev;
 
@@ -59,6 +61,9 @@ struct gfsl {
   uint64_t st_cap = 0;
   uint64_t batches = 0, ops = 0;
   std::vector<std::array<cudaEvent_t, 4>> phase_ev;  // profile_phases
+  // L2 persistence for the upper pool (the search kernel's access-policy window)
+  size_t persist_max = 0, window_max = 0;
+  uint32_t *h_bump = nullptr;  // pinned copy of the bump counters, refreshed every batch
 };
 
 // ------------------------------------------------------------------------------------
@@ -184,15 +189,42 @@ __global__ void classify_ordered_kernel(const uint8_t *__restrict__ ops, const u
 
 static SearchOut search_out(gfsl *h) { return SearchOut{h->plan_path, h->plan_top, h->mut_list}; }
 
+// The upper levels live in one contiguous range (the upper pool, chunks [0, cap_upper)),
+// so the search kernel is launched with an L2 access-policy window that marks the used
+// part of it persisting (north_star: "upper levels pinned in L2").  The used size lags by
+// one batch (read back asynchronously); it only steers a cache hint.
+static void fill_window(gfsl *h, cudaLaunchAttribute &a) {
+  a.id = cudaLaunchAttributeAccessPolicyWindow;
+  const size_t used = (size_t)std::min(h->h_bump[1] + 64u, h->d.cap_upper) * h->N * 8;
+  const size_t bytes = std::min(used, h->window_max);
+  a.val.accessPolicyWindow.base_ptr = h->d.pool;
+  a.val.accessPolicyWindow.num_bytes = bytes;
+  a.val.accessPolicyWindow.hitRatio = bytes ? std::min(1.0f, (float)h->persist_max / (float)bytes) : 0.f;
+  a.val.accessPolicyWindow.hitProp = cudaAccessPropertyPersisting;
+  a.val.accessPolicyWindow.missProp = cudaAccessPropertyStreaming;
+}
+
 template <int N, int TEAM>
 static void launch_contains(gfsl *h, const uint8_t *ops, const uint32_t *keys, uint8_t *res,
                             cudaStream_t s) {
+  (void)ops;
+  (void)keys;
+  cudaLaunchConfig_t lc{};
+  lc.gridDim = dim3(h->contains_grid);
+  lc.blockDim = dim3(256);
+  lc.stream = s;
+  cudaLaunchAttribute attr[1];
+  if (h->persist_max && h->window_max) {
+    fill_window(h, attr[0]);
+    lc.attrs = attr;
+    lc.numAttrs = 1;
+  }
   if (h->cfg.count_reads)
-    search_kernel<N, TEAM, true><<<h->contains_grid, 256, 0, s>>>(h->d, res, h->list_c, h->list_u,
-                                                                  h->ctl, search_out(h));
+    cudaLaunchKernelEx(&lc, search_kernel<N, TEAM, true>, h->d, res, (const uint2 *)h->list_c,
+                       (const uint2 *)h->list_u, h->ctl, search_out(h));
   else
-    search_kernel<N, TEAM, false><<<h->contains_grid, 256, 0, s>>>(h->d, res, h->list_c, h->list_u,
-                                                                   h->ctl, search_out(h));
+    cudaLaunchKernelEx(&lc, search_kernel<N, TEAM, false>, h->d, res, (const uint2 *)h->list_c,
+                       (const uint2 *)h->list_u, h->ctl, search_out(h));
 }
 
 #define GFSL_CONTAINS_CONFIGS(X) \
@@ -262,6 +294,27 @@ static int update_occupancy(uint32_t N) {
 // ------------------------------------------------------------------------------------
 // create / destroy
 
+// Opt-in (cfg.l2_window): reserve the device's persisting-L2 carve-out for the upper
+// pool.  Measured on B200: no gain for the search kernel, which is bound
+// by the L1 data pipe, and a slower update kernel (the carve-out shrinks its L2), so the
+// default is off.
+static void setup_l2_window(gfsl *h) {
+  h->persist_max = h->window_max = 0;
+  if (!h->cfg.l2_window) return;
+  int pmax = 0, wmax = 0;
+  cudaDeviceGetAttribute(&pmax, cudaDevAttrMaxPersistingL2CacheSize, h->device);
+  cudaDeviceGetAttribute(&wmax, cudaDevAttrMaxAccessPolicyWindowSize, h->device);
+  if (pmax > 0 && wmax > 0) {
+    size_t cur = 0;
+    cudaDeviceGetLimit(&cur, cudaLimitPersistingL2CacheSize);
+    if (cur < (size_t)pmax) cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, (size_t)pmax);
+    cudaDeviceGetLimit(&cur, cudaLimitPersistingL2CacheSize);
+    h->persist_max = cur;
+    h->window_max = (size_t)wmax;
+  }
+  cudaGetLastError();
+}
+
 static void apply_launch_shape(gfsl *h) {
   int bc = contains_occupancy(h->N, h->team);
   if (h->cfg.contains_blocks_per_sm) bc = std::min<int>(bc, h->cfg.contains_blocks_per_sm);
@@ -289,6 +342,7 @@ static void free_all(gfsl *h) {
   cudaFree(h->st_key);
   cudaFree(h->st_val);
   if (h->h_error) cudaFreeHost(h->h_error);
+  if (h->h_bump) cudaFreeHost(h->h_bump);
   if (h->last) cudaEventDestroy(h->last);
   for (auto &ev : h->phase_ev)
     for (auto &e : ev) cudaEventDestroy(e);
@@ -353,6 +407,10 @@ extern "C" gfsl_t gfsl_create_ex(uint64_t key_range, uint64_t capacity, const gf
   *h->h_error = 0;
   if ((e = cudaHostGetDevicePointer(&h->d.error, h->h_error, 0)) != cudaSuccess) return fail("cudaHostGetDevicePointer", e);
   if ((e = cudaEventCreateWithFlags(&h->last, cudaEventDisableTiming)) != cudaSuccess) return fail("cudaEventCreate", e);
+  if ((e = cudaHostAlloc(&h->h_bump, 8, cudaHostAllocDefault)) != cudaSuccess) return fail("cudaHostAlloc", e);
+  h->h_bump[0] = 1;
+  h->h_bump[1] = N - 1;
+  setup_l2_window(h);
   cudaMemset(h->d.head, 0xFF, 32 * 4);
   cudaMemset(h->d.counter, 0, 32 * 4);
   cudaMemset(h->d.stats, 0, ST_NSTATS * 8);
@@ -385,6 +443,7 @@ extern "C" gfsl_status gfsl_configure(gfsl_t h, const gfsl_config *cfg) {
   h->cfg.contains_team = team;
   h->team = team;
   apply_launch_shape(h);
+  setup_l2_window(h);
   return GFSL_OK;
 }
 
@@ -475,6 +534,7 @@ static gfsl_status enqueue_batch(gfsl *h, const uint8_t *ops, const uint32_t *ke
     CK(cudaEventRecord(ev[3], s));
     h->phase_ev.push_back(ev);
   }
+  CK(cudaMemcpyAsync(h->h_bump, h->d.bump, 8, cudaMemcpyDeviceToHost, s));
   CK(cudaEventRecord(h->last, s));
   h->batches++;
   h->ops += n;
@@ -975,6 +1035,66 @@ extern "C" gfsl_status gfsl_route_unpack(const uint32_t *perm, const uint8_t *re
   if (n == 0) return GFSL_OK;
   const int grid = (int)std::min<uint64_t>((n + 255) / 256, 148 * 16);
   route_unpack_kernel<<<grid, 256, 0, (cudaStream_t)stream>>>(perm, recv_res, (uint32_t)n, results);
+  CK(cudaGetLastError());
+  return GFSL_OK;
+}
+
+// ------------------------------------------------------------------------------------
+// B6 roofline microbenchmarks; measurement only, not part of a batch.
+
+extern "C" gfsl_status gfsl_ubench(uint32_t block_bytes, uint64_t buffer_bytes, double *gather_gbps,
+                                   double *chase_ns) {
+  if ((block_bytes != 256 && block_bytes != 128) || buffer_bytes < (1ull << 24)) return GFSL_EINVAL;
+  int dev = 0, sms = 148;
+  CK(cudaGetDevice(&dev));
+  cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+  void *buf = nullptr;
+  uint32_t *sink = nullptr;
+  CK(cudaMalloc(&buf, buffer_bytes));
+  CK(cudaMalloc(&sink, 4096 * 4));
+  uint64_t nblocks = 1;
+  while (nblocks * 2 * block_bytes <= buffer_bytes) nblocks *= 2;  // power of two
+  ubench_fill_chase<<<sms * 8, 256>>>((uint32_t *)buf, nblocks, block_bytes / 4, 12345u);
+  cudaEvent_t a, b;
+  cudaEventCreate(&a);
+  cudaEventCreate(&b);
+  const uint32_t iters = 256;
+  int occ = 0;
+  if (block_bytes == 256)
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, ubench_gather<256, 4>, 256, 0);
+  else
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, ubench_gather<128, 2>, 256, 0);
+  const int grid = sms * std::max(occ, 1);
+  const uint32_t teams_per_block = 256 / (block_bytes == 256 ? 4 : 2);
+  float best = 1e30f;
+  for (int rep = 0; rep < 5; ++rep) {
+    cudaEventRecord(a);
+    if (block_bytes == 256)
+      ubench_gather<256, 4><<<grid, 256>>>((const uint4 *)buf, nblocks, iters, 77u + rep, sink);
+    else
+      ubench_gather<128, 2><<<grid, 256>>>((const uint4 *)buf, nblocks, iters, 77u + rep, sink);
+    cudaEventRecord(b);
+    CK(cudaEventSynchronize(b));
+    float ms = 0;
+    cudaEventElapsedTime(&ms, a, b);
+    if (rep > 0) best = std::min(best, ms);
+  }
+  const double bytes = (double)grid * teams_per_block * iters * block_bytes;
+  if (gather_gbps) *gather_gbps = bytes / (best * 1e-3) / 1e9;
+  // dependent chase: one warp, 2000 steps
+  const uint32_t steps = 2000;
+  float cms = 0;
+  cudaEventRecord(a);
+  if (block_bytes == 256) ubench_chase<256><<<1, 32>>>((const uint32_t *)buf, 1u, steps, sink);
+  else ubench_chase<128><<<1, 32>>>((const uint32_t *)buf, 1u, steps, sink);
+  cudaEventRecord(b);
+  CK(cudaEventSynchronize(b));
+  cudaEventElapsedTime(&cms, a, b);
+  if (chase_ns) *chase_ns = cms * 1e6 / steps;
+  cudaEventDestroy(a);
+  cudaEventDestroy(b);
+  cudaFree(buf);
+  cudaFree(sink);
   CK(cudaGetLastError());
   return GFSL_OK;
 }

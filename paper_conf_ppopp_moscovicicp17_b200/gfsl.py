@@ -30,7 +30,7 @@ class gfsl_config(ctypes.Structure):
                 ("contains_blocks_per_sm", ctypes.c_uint32),
                 ("update_blocks_per_sm", ctypes.c_uint32),
                 ("serial_updates", ctypes.c_uint32), ("count_reads", ctypes.c_uint32),
-                ("profile_phases", ctypes.c_uint32), ("reserved", ctypes.c_uint32 * 1)]
+                ("profile_phases", ctypes.c_uint32), ("l2_window", ctypes.c_uint32)]
 
 
 class gfsl_report(ctypes.Structure):
@@ -64,7 +64,7 @@ EXPORTS = [
     "gfsl_create", "gfsl_create_ex", "gfsl_destroy", "gfsl_batch", "gfsl_batch_host",
     "gfsl_validate", "gfsl_last_error", "gfsl_get_stats", "gfsl_dump", "gfsl_load",
     "gfsl_route_plan", "gfsl_route_pack", "gfsl_route_unpack", "gfsl_phase_times",
-    "gfsl_configure",
+    "gfsl_configure", "gfsl_ubench",
 ]
 
 _lib = None
@@ -102,6 +102,8 @@ def load_library(path: str = LIB_PATH):
     lib.gfsl_dump.argtypes = [vp, ctypes.POINTER(gfsl_meta), vp, u64]
     lib.gfsl_load.restype = i32
     lib.gfsl_load.argtypes = [vp, ctypes.POINTER(gfsl_meta), vp, u64]
+    lib.gfsl_ubench.restype = i32
+    lib.gfsl_ubench.argtypes = [u32, u64, ctypes.POINTER(ctypes.c_double), ctypes.POINTER(ctypes.c_double)]
     lib.gfsl_configure.restype = i32
     lib.gfsl_configure.argtypes = [vp, ctypes.POINTER(gfsl_config)]
     lib.gfsl_phase_times.restype = i32
@@ -308,3 +310,11 @@ def route_unpack(perm, recv_res, out, stream=None):
     _check(lib.gfsl_route_unpack(_ptr(perm), _ptr(recv_res), recv_res.numel(), _ptr(out),
                                  _stream(stream)), "gfsl_route_unpack")
     return out
+
+
+def ubench(block_bytes: int = 256, buffer_bytes: int = 16 << 30):
+    """B6 roofline denominators: (R_rand GB/s, dependent-gather latency ns)."""
+    lib = load_library()
+    g, c = ctypes.c_double(), ctypes.c_double()
+    _check(lib.gfsl_ubench(block_bytes, buffer_bytes, ctypes.byref(g), ctypes.byref(c)), "gfsl_ubench")
+    return g.value, c.value
