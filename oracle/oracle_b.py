@@ -64,6 +64,7 @@ class GFSLModel:
             self.head[l] = c
         self.bump = [1, N - 1]  # [bottom pool, upper pool]
         self.trace = None       # chunks read by the last search (for the worked examples)
+        self.merges = 0         # merges of the current batch (-> upkeep)
 
     # ---- chunk accessors ----------------------------------------------------------------
     def keys(self, c):
@@ -395,6 +396,7 @@ class GFSLModel:
         self.execute_remove_merge(pe, pnext, k)           # l.21
         self.unlock(pe, ZOMBIE)                           # l.22 markAsZombie (R6)
         self.counter[level] -= 1                          # l.24
+        self.merges += 1
         if nf + cnt - 1 == 1 and self.nxt(pnext) == NULL and self.keys(pe)[0] == NEG_INF:
             self.counter[level] -= 1                      # R17
         self.unlock(pnext)                                # l.25
@@ -444,6 +446,7 @@ class GFSLModel:
                 if mut:
                     plans.append((i, op, k, path, top))
         head_at_start = list(self.head)  # levels above the snapshot height start at head[l]
+        self.merges = 0
         for i, op, k, path, top in plans:
             full = [path[l] if (l <= snap_h and l < PLAN_LEVELS) else head_at_start[l]
                     for l in range(self.N)]
@@ -453,7 +456,29 @@ class GFSLModel:
                 r = self.delete(k, full, top)
             if not r:
                 res[i] = 0
+        if self.merges:
+            self.upkeep()
         return res
+
+    def upkeep(self):
+        """R23: between batches, point every live chunk past the zombie chains that follow
+        it and move zombie first chunks out of the head array ("compact the structure
+        between kernel launches"; the values are those of Alg 4.6's lazy redirect)."""
+        used = list(range(self.bump[1])) + [self.cap_upper + i for i in range(self.bump[0])]
+        for c in used:
+            if self.zombie(c):
+                continue
+            n = self.nxt(c)
+            if n == NULL or not self.zombie(n):
+                continue
+            while self.zombie(n):
+                n = self.nxt(n)
+            self.pool[c][self.NEXT] = E(self.mx(c), n)
+        for l in range(self.N):
+            h = self.head[l]
+            while self.zombie(h):
+                h = self.nxt(h)
+            self.head[l] = h
 
     # ---- views ------------------------------------------------------------------------
     def level_chain(self, l):

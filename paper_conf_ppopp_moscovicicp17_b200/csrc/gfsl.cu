@@ -98,12 +98,14 @@ __global__ void init_heads_kernel(DevState d, uint32_t N) {
 }
 
 // Batch intake: range/op-code check (invalid -> 0xFF, no effect) and the split into the
-// Contains list and the Insert/Delete list (warp-aggregated appends).
-__global__ void classify_kernel(const uint8_t *__restrict__ ops, const uint32_t *__restrict__ keys,
-                                uint8_t *__restrict__ res, uint32_t n, uint64_t key_range,
-                                uint2 *__restrict__ list_c, uint2 *__restrict__ list_u,
-                                BatchCtl *ctl) {
-  const int lane = threadIdx.x & 31;
+// Contains list and the Insert/Delete list.  Appends are aggregated per block (one global
+// atomic per list per 256-op tile) so the two list counters do not serialize at L2.
+__global__ void __launch_bounds__(256)
+classify_kernel(const uint8_t *__restrict__ ops, const uint32_t *__restrict__ keys,
+                uint8_t *__restrict__ res, uint32_t n, uint64_t key_range,
+                uint2 *__restrict__ list_c, uint2 *__restrict__ list_u, BatchCtl *ctl) {
+  __shared__ uint32_t wc[8], wu[8], base_c, base_u;
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
   const uint32_t stride = gridDim.x * blockDim.x;
   for (uint32_t base = blockIdx.x * blockDim.x; base < n; base += stride) {
     const uint32_t i = base + threadIdx.x;
@@ -120,16 +122,28 @@ __global__ void classify_kernel(const uint8_t *__restrict__ ops, const uint32_t 
     }
     const uint32_t bc = __ballot_sync(0xFFFFFFFFu, isc);
     const uint32_t bu = __ballot_sync(0xFFFFFFFFu, isu);
-    uint32_t oc = 0, ou = 0;
     if (lane == 0) {
-      if (bc) oc = atomicAdd(&ctl->n_contains, __popc(bc));
-      if (bu) ou = atomicAdd(&ctl->n_updates, __popc(bu));
+      wc[warp] = __popc(bc);
+      wu[warp] = __popc(bu);
     }
-    oc = __shfl_sync(0xFFFFFFFFu, oc, 0);
-    ou = __shfl_sync(0xFFFFFFFFu, ou, 0);
+    __syncthreads();
+    if (threadIdx.x == 0) {
+      uint32_t tc = 0, tu = 0;
+      for (int w = 0; w < 8; ++w) {
+        const uint32_t c = wc[w], u = wu[w];
+        wc[w] = tc;
+        wu[w] = tu;
+        tc += c;
+        tu += u;
+      }
+      base_c = tc ? atomicAdd(&ctl->n_contains, tc) : 0;
+      base_u = tu ? atomicAdd(&ctl->n_updates, tu) : 0;
+    }
+    __syncthreads();
     const uint32_t below = (1u << lane) - 1u;
-    if (isc) list_c[oc + __popc(bc & below)] = e;
-    if (isu) list_u[ou + __popc(bu & below)] = e;
+    if (isc) list_c[base_c + wc[warp] + __popc(bc & below)] = e;
+    if (isu) list_u[base_u + wu[warp] + __popc(bu & below)] = e;
+    __syncthreads();
   }
 }
 
@@ -249,6 +263,7 @@ static void launch_update(gfsl *h, const uint8_t *ops, const uint32_t *keys, con
   } else {
     update_kernel<N><<<h->update_grid, 256, 0, s>>>(h->d, vals, res, h->list_u, h->ctl, search_out(h), 0);
   }
+  upkeep_kernel<N><<<h->sms * 4, 256, 0, s>>>(h->d);
 }
 
 template <int N, int TEAM>
@@ -403,6 +418,7 @@ extern "C" gfsl_t gfsl_create_ex(uint64_t key_range, uint64_t capacity, const gf
   if ((e = cudaMalloc(&h->d.bump, 2 * 4)) != cudaSuccess) return fail("cudaMalloc", e);
   if ((e = cudaMalloc(&h->d.stats, ST_NSTATS * 8)) != cudaSuccess) return fail("cudaMalloc", e);
   if ((e = cudaMalloc(&h->ctl, sizeof(BatchCtl))) != cudaSuccess) return fail("cudaMalloc", e);
+  h->d.ctl = h->ctl;
   if ((e = cudaHostAlloc(&h->h_error, 4, cudaHostAllocMapped)) != cudaSuccess) return fail("cudaHostAlloc", e);
   *h->h_error = 0;
   if ((e = cudaHostGetDevicePointer(&h->d.error, h->h_error, 0)) != cudaSuccess) return fail("cudaHostGetDevicePointer", e);

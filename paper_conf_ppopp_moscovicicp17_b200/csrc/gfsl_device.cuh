@@ -41,6 +41,8 @@ enum StatSlot {
   ST_NSTATS
 };
 
+struct BatchCtl;
+
 // Device view of one handle.
 struct DevState {
   uint64_t *pool;        // (cap_upper + cap_bottom) * N entries
@@ -52,6 +54,7 @@ struct DevState {
   uint32_t cap_bottom;   // bottom-pool chunks, indices [cap_upper, cap_upper + cap_bottom)
   uint32_t cap_upper;    // upper-pool chunks, indices [0, cap_upper)
   uint32_t key_max;      // largest valid internal key (= key_range)
+  BatchCtl *ctl;         // the handle's per-batch control block
 };
 
 // Per-batch control block (device memory, zeroed before every batch).
@@ -61,7 +64,8 @@ struct BatchCtl {
   uint32_t n_mut;        // update ops that mutate (search kernel)
   uint32_t next_update;  // dynamic work counter of the update kernel
   uint32_t snap_height;  // height seen by the search kernel
-  uint32_t pad[3];
+  uint32_t n_merges;     // merges of this batch (update kernel) -> upkeep sweep
+  uint32_t pad[2];
 };
 
 __device__ __forceinline__ uint32_t lo32(uint64_t x) { return (uint32_t)x; }
