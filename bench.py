@@ -36,17 +36,21 @@ from paper_conf_ppopp_moscovicicp17_b200.workload import (  # noqa: E402
 METRIC = "Mops/s (mixed insert/delete/contains)"
 
 # name: (R, prefill, batch, n_batches, mix, dist, N)
+# N = chunk entries.  The paper's runs use N = 32; on B200 a chunk read costs L1
+# data-pipe wavefronts in proportion to its bytes, and N = 16 (128-B chunks, 2-lane teams)
+# is faster on every config measured, so it is the default here; the
+# C4 pair compares the two, and --chunk 32 runs any config at the paper's size.
 CONFIGS = {
-    "C1": (10_000, 5_000, 6_250, 16, (10, 10, 80), "uniform", 32),
-    "C2": (1_000_000, 500_000, 625_000, 16, (10, 10, 80), "uniform", 32),
-    "C2-100": (1_000_000, 1_000_000, 10_000_000, 1, (0, 0, 100), "uniform", 32),
-    "C2-2020": (1_000_000, 500_000, 312_500, 32, (20, 20, 60), "uniform", 32),
-    "C2-5050": (1_000_000, 500_000, 125_000, 80, (50, 50, 0), "uniform", 32),
-    "C3": (10_000_000, 5_000_000, 6_250_000, 16, (10, 10, 80), "uniform", 32),
-    "C3-zipf": (10_000_000, 5_000_000, 6_250_000, 16, (10, 10, 80), "zipf", 32),
+    "C1": (10_000, 5_000, 6_250, 16, (10, 10, 80), "uniform", 16),
+    "C2": (1_000_000, 500_000, 625_000, 16, (10, 10, 80), "uniform", 16),
+    "C2-100": (1_000_000, 1_000_000, 10_000_000, 1, (0, 0, 100), "uniform", 16),
+    "C2-2020": (1_000_000, 500_000, 312_500, 32, (20, 20, 60), "uniform", 16),
+    "C2-5050": (1_000_000, 500_000, 125_000, 80, (50, 50, 0), "uniform", 16),
+    "C3": (10_000_000, 5_000_000, 6_250_000, 16, (10, 10, 80), "uniform", 16),
+    "C3-zipf": (10_000_000, 5_000_000, 6_250_000, 16, (10, 10, 80), "zipf", 16),
     "C4-32": (100_000_000, 100_000_000, 50_000_000, 10, (0, 0, 100), "uniform", 32),
     "C4-16": (100_000_000, 100_000_000, 50_000_000, 10, (0, 0, 100), "uniform", 16),
-    "C5": (1_000_000_000, 500_000_000, 125_000_000, 8, (10, 10, 80), "uniform", 32),
+    "C5": (1_000_000_000, 500_000_000, 125_000_000, 8, (10, 10, 80), "uniform", 16),
 }
 L2_FLUSH_BYTES = 256 << 20
 

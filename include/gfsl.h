@@ -54,7 +54,7 @@ enum { GFSL_RESULT_FALSE = 0, GFSL_RESULT_TRUE = 1, GFSL_RESULT_INVALID = 0xFF }
 
 typedef struct gfsl_config {
   uint32_t chunk_entries;   /* N: 16 (128-B chunks) or 32 (256-B chunks).
-                               0 = 32.  MAX_LEVEL = N (path held one level per lane,
+                               0 = 16 (fastest on B200).  MAX_LEVEL = N (path held one level per lane,
                                P:493-495). */
   uint32_t contains_team;   /* lanes per Contains team (a power of two dividing N, >= 4);
                                0 = the tuned default.  P:205 allows teams <= a warp. */

@@ -242,7 +242,8 @@ static void launch_contains(gfsl *h, const uint8_t *ops, const uint32_t *keys, u
 }
 
 #define GFSL_CONTAINS_CONFIGS(X) \
-  X(32, 4) X(32, 8) X(32, 16) X(32, 32) X(16, 2) X(16, 4) X(16, 8) X(16, 16) X(12, 12) X(6, 6)
+  X(32, 2) X(32, 4) X(32, 8) X(32, 16) X(32, 32) X(16, 1) X(16, 2) X(16, 4) X(16, 8) X(16, 16) \
+  X(12, 12) X(6, 6)
 
 static bool dispatch_contains(gfsl *h, const uint8_t *ops, const uint32_t *keys, uint8_t *res,
                               cudaStream_t s) {
@@ -367,7 +368,7 @@ static void free_all(gfsl *h) {
 extern "C" gfsl_t gfsl_create_ex(uint64_t key_range, uint64_t capacity, const gfsl_config *cfg_in) {
   gfsl_config cfg{};
   if (cfg_in) cfg = *cfg_in;
-  if (cfg.chunk_entries == 0) cfg.chunk_entries = 32;
+  if (cfg.chunk_entries == 0) cfg.chunk_entries = 16;  // B200 default
   const uint32_t N = cfg.chunk_entries;
   if (N != 32 && N != 16 && N != 12 && N != 6) {
     set_last_error("chunk_entries must be 6, 12, 16 or 32");

@@ -162,6 +162,16 @@ __device__ __forceinline__ void ld_slice_nc<8>(const uint64_t *p, ChunkSlice<8> 
                : "l"(p + 4));
 }
 
+template <>
+__device__ __forceinline__ void ld_slice_nc<16>(const uint64_t *p, ChunkSlice<16> &s) {
+#pragma unroll
+  for (int q = 0; q < 4; ++q)
+    asm volatile("ld.global.nc.v8.u32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];"
+                 : "=r"(s.k[4 * q]), "=r"(s.v[4 * q]), "=r"(s.k[4 * q + 1]), "=r"(s.v[4 * q + 1]),
+                   "=r"(s.k[4 * q + 2]), "=r"(s.v[4 * q + 2]), "=r"(s.k[4 * q + 3]), "=r"(s.v[4 * q + 3])
+                 : "l"(p + 4 * q));
+}
+
 __device__ __forceinline__ void set_error(const DevState &d, uint32_t bit) {
   atomicOr(d.error, bit);
 }

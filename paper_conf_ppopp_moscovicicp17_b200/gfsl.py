@@ -160,7 +160,7 @@ class Report:
 class GFSL:
     """One GFSL map on the current CUDA device (C handle ``gfsl_t``)."""
 
-    def __init__(self, key_range: int, capacity: int = 0, chunk_entries: int = 32,
+    def __init__(self, key_range: int, capacity: int = 0, chunk_entries: int = 16,
                  contains_team: int = 0, serial_updates: bool = False,
                  contains_blocks_per_sm: int = 0, update_blocks_per_sm: int = 0,
                  count_reads: bool = False, profile_phases: bool = False):
