@@ -415,8 +415,9 @@ class GFSLModel:
             self.unlock(pb)
             return False
         m = top                                           # l.12-16 (R12)
-        while m + 1 < self.MAXL and self.search_lateral(k, path[m + 1]):
-            m += 1
+        if pb != path[0]:  # k moved since the snapshot: it may have been raised as a minK
+            while m + 1 < self.MAXL and self.search_lateral(k, path[m + 1]):
+                m += 1
         for i in range(m, 0, -1):                         # l.13-20
             pe = self.find_and_lock_enclosing(path[i], k, i)
             if self.eq_idx(pe, k) is None:
