@@ -128,14 +128,19 @@ class ClockSampler:
                 "samples": len(self.samples)}
 
 
-def dist_setup():
+def dist_setup(backend="nccl"):
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
+    if backend == "gloo":  # test path: several ranks may share one GPU
+        local = local % max(1, torch.cuda.device_count())
     if world > 1:
         import torch.distributed as dist
         torch.cuda.set_device(local)
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        if backend == "nccl":
+            dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        else:
+            dist.init_process_group(backend)
     else:
         torch.cuda.set_device(local)
     return world, rank, local
@@ -151,7 +156,8 @@ def max_over_ranks(x: float, world: int) -> float:
     if world == 1:
         return x
     import torch.distributed as dist
-    t = torch.tensor([x], dtype=torch.float64, device="cuda")
+    dev = "cuda" if dist.get_backend() == "nccl" else "cpu"
+    t = torch.tensor([x], dtype=torch.float64, device=dev)
     dist.all_reduce(t, op=dist.ReduceOp.MAX)
     return float(t.item())
 
@@ -417,7 +423,7 @@ def run_gpu(args, world, rank, local):
             "chunk_reads_l0_per_contains": round(reads_l0_per_op, 3),
             "cpu_baseline": cpu,
             "e2e": e2e,
-            "gpu_launches": 3 * steps * (1 if world == 1 else 1) + (4 * steps if world > 1 else 0),
+            "gpu_launches": 4 * steps + (5 * steps if world > 1 else 0),  # classify, search, update, upkeep (+ route plan x3, pack, unpack)
             "clocks": clk,
             "wall_s_timed_region": round(wall, 4),
             "generator_redraws": int(redraws),
@@ -439,6 +445,8 @@ def main():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--validate", action="store_true")
     ap.add_argument("--no-ubench", action="store_true", help="skip the B6 roofline microbenchmark")
+    ap.add_argument("--dist-backend", default="nccl", choices=["nccl", "gloo"],
+                    help="gloo: exercise the multi-rank path with ranks sharing a GPU (no timing value)")
     ap.add_argument("--l2-window", action="store_true",
                     help="pin the upper-level pool in L2 (access-policy window; ablation)")
     args = ap.parse_args()
@@ -451,7 +459,7 @@ def main():
             args.steps = CONFIGS[args.config][3]
         run_reference(args, world, rank)
         return
-    world, rank, local = dist_setup()
+    world, rank, local = dist_setup(args.dist_backend)
     run_gpu(args, world, rank, local)
     if world > 1:
         import torch.distributed as dist

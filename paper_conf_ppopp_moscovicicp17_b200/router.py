@@ -67,6 +67,12 @@ class ShardedGFSL:
         self.last_counts = None
 
     def _a2a(self, out, inp, out_splits, in_splits):
+        if out.is_cuda and dist.get_backend(self.group) == "gloo":
+            # gloo has no CUDA all-to-all: stage through host memory (test path only)
+            tmp = torch.empty(out.shape, dtype=out.dtype)
+            dist.all_to_all_single(tmp, inp.cpu(), out_splits, in_splits, group=self.group)
+            out.copy_(tmp)
+            return out
         dist.all_to_all_single(out, inp, out_splits, in_splits, group=self.group)
         return out
 

@@ -1,0 +1,34 @@
+"""bench.py end to end on the GPU: the 1-GPU JSON line carries the contract's keys, and
+the N>1 path (router + all-to-all exchange) runs as 2 ranks sharing one GPU over gloo."""
+import json
+import os
+import subprocess
+import sys
+
+import pytest
+
+pytestmark = pytest.mark.gpu
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+def run(cmd, timeout=600):
+    r = subprocess.run(cmd, cwd=ROOT, capture_output=True, text=True, timeout=timeout)
+    assert r.returncode == 0, r.stdout[-2000:] + r.stderr[-2000:]
+    lines = [l for l in r.stdout.splitlines() if l.startswith("{")]
+    return json.loads(lines[-1])
+
+
+def test_bench_single_gpu_line():
+    d = run([sys.executable, "bench.py", "--config", "C1", "--steps", "4", "--no-e2e"])
+    for k in ["metric", "value", "unit", "n_gpus", "steps", "warmup", "ms_per_step",
+              "higher_is_better", "scaling", "dtype", "config", "roofline", "cpu_baseline",
+              "clocks", "gpu_launches"]:
+        assert k in d, k
+    assert d["value"] > 0 and d["roofline"]["peak"] > 0 and d["cpu_baseline"]["kind"] == "oracle"
+
+
+def test_bench_two_ranks_gloo():
+    d = run([sys.executable, "-m", "torch.distributed.run", "--nnodes=1", "--nproc-per-node", "2",
+             "--master-addr", "127.0.0.1", "--master-port", "29533", "bench.py", "--gpus", "2",
+             "--config", "C1", "--steps", "3", "--dist-backend", "gloo", "--validate", "--no-ubench"])
+    assert d["n_gpus"] == 2 and d["value"] > 0 and d["validate"]["violations"] == 0
