@@ -262,16 +262,19 @@ def run_gpu(args, world, rank, local):
     if world > 1:
         from paper_conf_ppopp_moscovicicp17_b200.router import ShardedGFSL
         g = ShardedGFSL(R, rank, world, capacity=R1, chunk_entries=N,
-                        contains_team=args.team, profile_phases=True)
+                        contains_team=args.team)
         lo = g.key_lo
         prefill_gpu(g.local, R1, pre1, dev, key_lo=lo, seed=SEED_BASE + 1000 * rank)
     else:
-        g = GFSL(R, capacity=R, chunk_entries=N, contains_team=args.team, profile_phases=True)
+        g = GFSL(R, capacity=R, chunk_entries=N, contains_team=args.team)
         prefill_gpu(g, R, pre1, dev)
     if args.l2_window:
         (g.local if world > 1 else g).configure(l2_window=1)
+    if args.no_pdl:
+        (g.local if world > 1 else g).configure(no_pdl=1)
+    PROF = 3  # extra batches after the timed region, for the per-kernel breakdown
     w = Workload(R, B1, mix=mix, dist=dist, seed=SEED_BASE + 1 + 7919 * rank)
-    inputs = [make_inputs(w, b, dev) for b in range(W + steps)]
+    inputs = [make_inputs(w, b, dev) for b in range(W + steps + PROF)]
     redraws = sum(x[3] for x in inputs)
     flush = torch.empty(L2_FLUSH_BYTES, dtype=torch.uint8, device=dev)
     stream = torch.cuda.current_stream()
@@ -281,7 +284,6 @@ def run_gpu(args, world, rank, local):
     torch.cuda.synchronize()
     barrier(world)
     local_g = g.local if world > 1 else g
-    local_g.phase_times()  # reset the per-phase sums
     mut0 = local_g.stats()["mutations"]
 
     starts = [torch.cuda.Event(enable_timing=True) for _ in range(steps)]
@@ -305,21 +307,30 @@ def run_gpu(args, world, rank, local):
     total_ms = max_over_ranks(local_ms, world)
     ops_total = B1 * steps * world
     mops = ops_total / (total_ms / 1e3) / 1e6
-    phases, nbat = local_g.phase_times()
     n_mut = (local_g.stats()["mutations"] - mut0) / max(steps, 1)
+    # per-kernel breakdown: CUDA events between the kernels of PROF extra batches (events
+    # between kernels would defeat the programmatic dependent launch of the timed steps)
+    local_g.configure(profile_phases=1)
+    local_g.phase_times()
+    for j in range(PROF):
+        flush.zero_()
+        g.batch(*inputs[W + steps + j][:3])
+    torch.cuda.synchronize()
+    phases, nbat = local_g.phase_times()
+    local_g.configure(profile_phases=0)
 
     # algorithmic bytes: chunk reads per Contains op, counted on a Contains-only replay
     # of the last timed batch's keys (untimed, non-mutating)
     Cb = N * 8
-    local_g.configure(count_reads=1, profile_phases=0)
+    local_g.configure(count_reads=1)
     st0 = local_g.stats()
-    key_last = inputs[W + steps - 1][1]
+    key_last = inputs[W + steps + PROF - 1][1]
     if world > 1:
         key_last = key_last[(key_last >= g.key_lo) & (key_last < g.key_hi)].contiguous()
     local_g.batch(torch.zeros(key_last.numel(), dtype=torch.uint8, device=dev), key_last)
     torch.cuda.synchronize()
     st1 = local_g.stats()
-    local_g.configure(count_reads=0, profile_phases=1)
+    local_g.configure(count_reads=0)
     cops = max(1, st1["contains_ops"] - st0["contains_ops"])
     reads_per_op = (st1["contains_reads"] - st0["contains_reads"]) / cops
     reads_l0_per_op = (st1["contains_reads_l0"] - st0["contains_reads_l0"]) / cops
@@ -445,6 +456,7 @@ def main():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--validate", action="store_true")
     ap.add_argument("--no-ubench", action="store_true", help="skip the B6 roofline microbenchmark")
+    ap.add_argument("--no-pdl", action="store_true", help="no programmatic dependent launch (ablation)")
     ap.add_argument("--dist-backend", default="nccl", choices=["nccl", "gloo"],
                     help="gloo: exercise the multi-rank path with ranks sharing a GPU (no timing value)")
     ap.add_argument("--l2-window", action="store_true",

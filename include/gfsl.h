@@ -69,6 +69,8 @@ typedef struct gfsl_config {
   uint32_t l2_window;       /* 1 = launch the search kernel with an L2 access-policy window
                                marking the upper-level pool persisting (opt-in; see
                                DESIGN.md §9 for why it is off by default) */
+  uint32_t no_pdl;          /* 1 = launch the kernels of a batch without programmatic
+                               dependent launch (ablation) */
 } gfsl_config;
 
 /*

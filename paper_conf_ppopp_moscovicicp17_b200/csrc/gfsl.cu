@@ -201,6 +201,14 @@ __global__ void classify_ordered_kernel(const uint8_t *__restrict__ ops, const u
 // ------------------------------------------------------------------------------------
 // template dispatch
 
+// Programmatic dependent launch between the kernels of a batch (search -> update ->
+// upkeep): each is launched while its predecessor drains and waits in-kernel
+// (griddepcontrol.wait) before reading its outputs.
+static void set_pdl(gfsl *h, cudaLaunchAttribute &a) {
+  a.id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  a.val.programmaticStreamSerializationAllowed = h->cfg.no_pdl ? 0 : 1;
+}
+
 static SearchOut search_out(gfsl *h) { return SearchOut{h->plan_path, h->plan_top, h->mut_list}; }
 
 // The upper levels live in one contiguous range (the upper pool, chunks [0, cap_upper)),
@@ -227,12 +235,10 @@ static void launch_contains(gfsl *h, const uint8_t *ops, const uint32_t *keys, u
   lc.gridDim = dim3(h->contains_grid);
   lc.blockDim = dim3(256);
   lc.stream = s;
-  cudaLaunchAttribute attr[1];
-  if (h->persist_max && h->window_max) {
-    fill_window(h, attr[0]);
-    lc.attrs = attr;
-    lc.numAttrs = 1;
-  }
+  cudaLaunchAttribute attr[2];
+  lc.attrs = attr;
+  if (h->persist_max && h->window_max) fill_window(h, attr[lc.numAttrs++]);
+  set_pdl(h, attr[lc.numAttrs++]);
   if (h->cfg.count_reads)
     cudaLaunchKernelEx(&lc, search_kernel<N, TEAM, true>, h->d, res, (const uint2 *)h->list_c,
                        (const uint2 *)h->list_u, h->ctl, search_out(h));
@@ -259,12 +265,20 @@ template <int N>
 static void launch_update(gfsl *h, const uint8_t *ops, const uint32_t *keys, const uint32_t *vals,
                           uint8_t *res, uint32_t n, cudaStream_t s) {
   (void)n;
-  if (h->cfg.serial_updates) {
-    update_kernel<N><<<1, 32, 0, s>>>(h->d, vals, res, h->list_u, h->ctl, search_out(h), 1);
-  } else {
-    update_kernel<N><<<h->update_grid, 256, 0, s>>>(h->d, vals, res, h->list_u, h->ctl, search_out(h), 0);
-  }
-  upkeep_kernel<N><<<h->sms * 4, 256, 0, s>>>(h->d);
+  cudaLaunchConfig_t lc{};
+  cudaLaunchAttribute attr[1];
+  set_pdl(h, attr[0]);
+  lc.attrs = attr;
+  lc.numAttrs = 1;
+  lc.stream = s;
+  lc.blockDim = dim3(h->cfg.serial_updates ? 32 : 256);
+  lc.gridDim = dim3(h->cfg.serial_updates ? 1 : h->update_grid);
+  const int serial = h->cfg.serial_updates ? 1 : 0;
+  cudaLaunchKernelEx(&lc, update_kernel<N>, h->d, vals, res, (const uint2 *)h->list_u, h->ctl,
+                     search_out(h), serial);
+  lc.blockDim = dim3(256);
+  lc.gridDim = dim3(h->sms * 4);
+  cudaLaunchKernelEx(&lc, upkeep_kernel<N>, h->d);
 }
 
 template <int N, int TEAM>

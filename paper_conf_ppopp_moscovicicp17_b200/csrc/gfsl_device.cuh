@@ -172,6 +172,12 @@ __device__ __forceinline__ void ld_slice_nc<16>(const uint64_t *p, ChunkSlice<16
                  : "l"(p + 4 * q));
 }
 
+// Programmatic dependent launch: a kernel launched with programmatic stream serialization
+// may start while its predecessor drains; it waits here before touching the predecessor's
+// outputs, and lets its own dependents launch early.
+__device__ __forceinline__ void pdl_wait() { asm volatile("griddepcontrol.wait;" ::: "memory"); }
+__device__ __forceinline__ void pdl_trigger() { asm volatile("griddepcontrol.launch_dependents;" ::: "memory"); }
+
 __device__ __forceinline__ void set_error(const DevState &d, uint32_t bit) {
   atomicOr(d.error, bit);
 }

@@ -68,6 +68,8 @@ search_kernel(DevState d, uint8_t *__restrict__ res, const uint2 *__restrict__ l
 
   __shared__ uint32_t s_start, s_height;
   const int lane = threadIdx.x & 31;
+  pdl_wait();
+  pdl_trigger();
   if (threadIdx.x < 32) {
     // getHeight / firstChunkAtLevel: lane l reads level l's counter.
     const int32_t c = (lane < N) ? d.counter[lane] : 0;

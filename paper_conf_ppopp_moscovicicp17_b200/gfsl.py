@@ -30,7 +30,8 @@ class gfsl_config(ctypes.Structure):
                 ("contains_blocks_per_sm", ctypes.c_uint32),
                 ("update_blocks_per_sm", ctypes.c_uint32),
                 ("serial_updates", ctypes.c_uint32), ("count_reads", ctypes.c_uint32),
-                ("profile_phases", ctypes.c_uint32), ("l2_window", ctypes.c_uint32)]
+                ("profile_phases", ctypes.c_uint32), ("l2_window", ctypes.c_uint32),
+                ("no_pdl", ctypes.c_uint32)]
 
 
 class gfsl_report(ctypes.Structure):
