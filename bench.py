@@ -272,6 +272,8 @@ def run_gpu(args, world, rank, local):
         (g.local if world > 1 else g).configure(l2_window=1)
     if args.no_pdl:
         (g.local if world > 1 else g).configure(no_pdl=1)
+    (g.local if world > 1 else g).configure(
+        rebuild_every=0xFFFFFFFF if args.rebuild_every < 0 else args.rebuild_every)
     PROF = 3  # extra batches after the timed region, for the per-kernel breakdown
     w = Workload(R, B1, mix=mix, dist=dist, seed=SEED_BASE + 1 + 7919 * rank)
     inputs = [make_inputs(w, b, dev) for b in range(W + steps + PROF)]
@@ -418,7 +420,7 @@ def run_gpu(args, world, rank, local):
             "steps": steps, "warmup": W, "ms_per_step": round(total_ms / steps, 4),
             "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
             "dtype": "u32", "data": "synthetic",
-            "config": {"workload": args.config, "key_range": R, "prefill": pre1 * world,
+            "config": {"workload": args.config, "key_range": R, "rebuild_every": args.rebuild_every, "prefill": pre1 * world,
                        "batch_ops": B1 * world, "mix_ins_del_con": list(mix), "keys": dist,
                        "chunk_entries": N, "contains_team": local_g.cfg.contains_team or (4 if N == 32 else 2),
                        "l2": "flushed (256 MiB write) between timed steps",
@@ -457,6 +459,9 @@ def main():
     ap.add_argument("--validate", action="store_true")
     ap.add_argument("--no-ubench", action="store_true", help="skip the B6 roofline microbenchmark")
     ap.add_argument("--no-pdl", action="store_true", help="no programmatic dependent launch (ablation)")
+    ap.add_argument("--rebuild-every", type=int, default=0,
+                    help="rebuild the upper levels after every k-th batch (R24); "
+                         "0 = library default (2), -1 = never (the paper's dynamics only)")
     ap.add_argument("--dist-backend", default="nccl", choices=["nccl", "gloo"],
                     help="gloo: exercise the multi-rank path with ranks sharing a GPU (no timing value)")
     ap.add_argument("--l2-window", action="store_true",

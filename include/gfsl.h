@@ -47,6 +47,9 @@ typedef enum gfsl_status {
   GFSL_ECORRUPT = 5  /* gfsl_validate found an invariant violation */
 } gfsl_status;
 
+#define GFSL_REBUILD_DEFAULT_PERIOD 2u
+#define GFSL_REBUILD_NEVER 0xFFFFFFFFu
+
 /* Op codes (the "operation type" of the op array). */
 enum { GFSL_CONTAINS = 0, GFSL_INSERT = 1, GFSL_DELETE = 2 };
 /* Per-op result codes. */
@@ -71,6 +74,10 @@ typedef struct gfsl_config {
                                DESIGN.md §9 for why it is off by default) */
   uint32_t no_pdl;          /* 1 = launch the kernels of a batch without programmatic
                                dependent launch (ablation) */
+  uint32_t rebuild_every;   /* after every k-th batch, rebuild the levels >= 1 from level 0
+                               (R24: "compact the structure between kernel
+                               launches").  0 = GFSL_REBUILD_DEFAULT_PERIOD;
+                               GFSL_REBUILD_NEVER = the paper's structure dynamics only */
 } gfsl_config;
 
 /*

@@ -44,8 +44,11 @@ class PoolExhausted(Exception):
 
 
 class GFSLModel:
-    def __init__(self, N: int, key_range: int, cap_bottom: int, cap_upper: int):
+    def __init__(self, N: int, key_range: int, cap_bottom: int, cap_upper: int,
+                 rebuild_every: int = 0):
         assert N >= 6
+        self.rebuild_every = rebuild_every
+        self.batches = 0
         self.N, self.DSIZE, self.NEXT, self.LOCK, self.MAXL = N, N - 2, N - 2, N - 1, N
         self.key_range = key_range
         self.cap_bottom, self.cap_upper = cap_bottom, cap_upper
@@ -459,7 +462,71 @@ class GFSLModel:
                 res[i] = 0
         if self.merges:
             self.upkeep()
+        if n and self.rebuild_every and (self.batches + 1) % self.rebuild_every == 0:
+            self.rebuild()
+        if n:
+            self.batches += 1
         return res
+
+    def rebuild(self):
+        """R24: re-derive levels >= 1 from level 0 between batches ("compact the
+        structure between kernel launches").  Level 1 = [-inf -> head[0]] + (min key of C
+        -> C) for every live non-first level-0 chunk C holding a key, in key order, F per
+        chunk; level l+1 = [-inf -> first chunk of level l] + (first key of chunk j -> chunk
+        j); chunks of level l: the head chunk l-1, then the next free upper indices."""
+        N, F = self.N, self.N - 4
+        live = []
+        for i in range(self.bump[0]):
+            c = self.cap_upper + i
+            k0 = K(self.pool[c][0])
+            if not self.zombie(c) and k0 not in (NEG_INF, INF):
+                live.append((k0, c))
+        live.sort()
+        n1 = len(live)
+        m, base, pw = {}, {}, {}
+        length, b, p, top = n1 + 1, N - 1, 1, N - 1
+        for l in range(1, N):
+            m[l], base[l], pw[l] = -(-length // F), b, p
+            b += m[l] - 1
+            if m[l] == 1:
+                top = l
+                for q in range(l + 1, N):
+                    m[q], base[q], pw[q] = 1, b, p * F
+                break
+            length, p = m[l], p * F
+
+        def chunk(l, j):
+            return l - 1 if j == 0 else base[l] + j - 1
+
+        head0, old_used = self.head[0], self.bump[1]
+        for l in range(1, N):
+            length = 1 if l > top else (n1 + 1 if l == 1 else m[l - 1])
+            for j in range(m[l]):
+                ch = self.pool[chunk(l, j)]
+                last_key = 0
+                for e in range(self.DSIZE):
+                    i = j * F + e
+                    if e < F and i < length:
+                        if i == 0:
+                            key, val = NEG_INF, (head0 if l == 1 else l - 2)
+                        else:
+                            key = live[i * pw[l] - 1][0]
+                            val = live[i - 1][1] if l == 1 else chunk(l - 1, i)
+                        ch[e] = E(key, val)
+                        last_key = key
+                    else:
+                        ch[e] = EMPTY
+                last = j + 1 == m[l]
+                ch[self.NEXT] = E(INF, NULL) if last else E(last_key, chunk(l, j + 1))
+                ch[self.LOCK] = E(FREE, 0)
+        for l in range(1, N):
+            self.head[l] = l - 1
+            real = (n1 > 0) if l == 1 else (m[l - 1] > 1)
+            self.counter[l] = m[l] if (l <= top and real) else 0
+        new_used = base[N - 1] + (m[N - 1] - 1 if top == N - 1 else 0)
+        self.bump[1] = new_used
+        for c in range(new_used, old_used):  # back to the allocated state of P:237
+            self.pool[c] = [EMPTY] * (N - 1) + [HELD]
 
     def upkeep(self):
         """R23: between batches, point every live chunk past the zombie chains that follow

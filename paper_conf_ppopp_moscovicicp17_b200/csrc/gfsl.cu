@@ -20,6 +20,7 @@
 #include "gfsl_device.cuh"
 #include "gfsl_update.cuh"
 #include "gfsl_ubench.cuh"
+#include "gfsl_rebuild.cuh"
 
 using namespace gfsl_dev;
 
@@ -64,6 +65,7 @@ struct gfsl {
   // L2 persistence for the upper pool (the search kernel's access-policy window)
   size_t persist_max = 0, window_max = 0;
   uint32_t *h_bump = nullptr;  // pinned copy of the bump counters, refreshed every batch
+  RebuildBufs rb{};            // upper-level rebuild (R24)
 };
 
 // ------------------------------------------------------------------------------------
@@ -279,6 +281,28 @@ static void launch_update(gfsl *h, const uint8_t *ops, const uint32_t *keys, con
   lc.blockDim = dim3(256);
   lc.gridDim = dim3(h->sms * 4);
   cudaLaunchKernelEx(&lc, upkeep_kernel<N>, h->d);
+  // R24: rebuild the upper levels from level 0 after every `rebuild_every`-th batch
+  const uint32_t every = h->cfg.rebuild_every == 0 ? GFSL_REBUILD_DEFAULT_PERIOD : h->cfg.rebuild_every;
+  if (every != GFSL_REBUILD_NEVER && (h->batches + 1) % every == 0) {
+    const RebuildBufs &b = h->rb;
+    lc.gridDim = dim3(h->sms * 4);
+    cudaLaunchKernelEx(&lc, rebuild_mark_kernel<N>, h->d, b);
+    lc.gridDim = dim3(b.blocks);
+    lc.blockDim = dim3(1024);
+    cudaLaunchKernelEx(&lc, rebuild_scan_kernel, b);
+    lc.gridDim = dim3(1);
+    cudaLaunchKernelEx(&lc, rebuild_scan_top_kernel, b);
+    lc.blockDim = dim3(256);
+    lc.gridDim = dim3(h->sms * 4);
+    cudaLaunchKernelEx(&lc, rebuild_rank_kernel<N>, h->d, b);
+    lc.gridDim = dim3(h->sms * 2);
+    cudaLaunchKernelEx(&lc, rebuild_pack_kernel<N>, h->d, b);
+    lc.gridDim = dim3(h->sms * 4);
+    cudaLaunchKernelEx(&lc, rebuild_clear_kernel<N>, h->d, b);
+    lc.gridDim = dim3(1);
+    lc.blockDim = dim3(32);
+    cudaLaunchKernelEx(&lc, rebuild_reset_kernel, b);
+  }
 }
 
 template <int N, int TEAM>
@@ -371,6 +395,12 @@ static void free_all(gfsl *h) {
   cudaFree(h->st_res);
   cudaFree(h->st_key);
   cudaFree(h->st_val);
+  cudaFree(h->rb.bitmap);
+  cudaFree(h->rb.word_prefix);
+  cudaFree(h->rb.block_sum);
+  cudaFree(h->rb.order_key);
+  cudaFree(h->rb.order_chunk);
+  cudaFree(h->rb.n1);
   if (h->h_error) cudaFreeHost(h->h_error);
   if (h->h_bump) cudaFreeHost(h->h_bump);
   if (h->last) cudaEventDestroy(h->last);
@@ -442,6 +472,20 @@ extern "C" gfsl_t gfsl_create_ex(uint64_t key_range, uint64_t capacity, const gf
   h->h_bump[0] = 1;
   h->h_bump[1] = N - 1;
   setup_l2_window(h);
+  {
+    RebuildBufs &b = h->rb;
+    b.words = (uint32_t)((key_range + 2 + 31) / 32);
+    b.blocks = (b.words + RB_BLOCK_WORDS - 1) / RB_BLOCK_WORDS;
+    b.fill = N - 4;  // leaves 2 free DATA slots per rebuilt chunk for later raises
+    if ((e = cudaMalloc(&b.bitmap, (size_t)b.words * 4)) != cudaSuccess) return fail("cudaMalloc(rebuild)", e);
+    if ((e = cudaMalloc(&b.word_prefix, (size_t)b.words * 4)) != cudaSuccess) return fail("cudaMalloc(rebuild)", e);
+    if ((e = cudaMalloc(&b.block_sum, (size_t)b.blocks * 4)) != cudaSuccess) return fail("cudaMalloc(rebuild)", e);
+    if ((e = cudaMalloc(&b.order_key, (size_t)cap_b * 4)) != cudaSuccess) return fail("cudaMalloc(rebuild)", e);
+    if ((e = cudaMalloc(&b.order_chunk, (size_t)cap_b * 4)) != cudaSuccess) return fail("cudaMalloc(rebuild)", e);
+    if ((e = cudaMalloc(&b.n1, 8)) != cudaSuccess) return fail("cudaMalloc(rebuild)", e);
+    cudaMemset(b.bitmap, 0, (size_t)b.words * 4);
+    cudaMemset(b.n1, 0, 8);
+  }
   cudaMemset(h->d.head, 0xFF, 32 * 4);
   cudaMemset(h->d.counter, 0, 32 * 4);
   cudaMemset(h->d.stats, 0, ST_NSTATS * 8);

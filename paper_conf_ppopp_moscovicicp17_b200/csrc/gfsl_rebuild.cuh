@@ -1,0 +1,257 @@
+// gfsl_rebuild.cuh -- upkeep: rebuild of the upper levels between batches (R24).
+//
+// "A possible reclamation scheme would be to compact the structure between
+// kernel launches"; "a between-batch rebuild of levels >= 1 from level 0".
+// Keys rise only through splits while deletes strip every level, so under
+// churn the upper levels thin out and traversals take ever more lateral steps.  Between
+// batches the structure is quiescent, so the upper levels are re-derived from level 0:
+//   level 1 = [-inf -> head[0]] ++ [(min key of C) -> C for every live non-first level-0
+//             chunk C holding a key, in key order], packed F entries per chunk;
+//   level l+1 = [-inf -> first chunk of level l] ++ [(first key of chunk j) -> chunk j
+//             of level l, j >= 1], packed F per chunk, until a level fits one chunk.
+// So entry i of level l (i >= 1) carries the key of entry i*F^(l-1) of level 1, and every
+// level-0 chunk is the direct target of a level-1 entry.  Level 0 is not touched.
+// The chunks of levels >= 1 are rewritten in place in the upper pool: level l's first
+// chunk is the head chunk l-1 of P:235, the others are allocated in level order after
+// the heads; upper chunks no longer used are returned to the allocated state.
+//
+// Ordering level-0 chunks by key without a host round trip: every chunk marks its min key
+// in a key_range-bit bitmap; a two-level popcount scan ranks the marks; each chunk writes
+// itself at its rank.
+#pragma once
+#include "gfsl_device.cuh"
+
+namespace gfsl_dev {
+
+struct RebuildBufs {
+  uint32_t *bitmap;       // [words]      key marks (all zero between rebuilds)
+  uint32_t *word_prefix;  // [words]      exclusive popcount prefix within a 1024-word block
+  uint32_t *block_sum;    // [blocks]     popcount of each block, then its exclusive prefix
+  uint32_t *order_key;    // [cap_bottom] min keys in key order
+  uint32_t *order_chunk;  // [cap_bottom] their chunks
+  uint32_t *n1;           // [2]          marked chunks; old upper bump
+  uint32_t words, blocks;
+  uint32_t fill;          // F: entries per rebuilt upper chunk
+};
+
+constexpr int RB_BLOCK_WORDS = 1024;
+
+__device__ __forceinline__ bool rb_candidate(const DevState &d, uint32_t c, int N, uint32_t &minkey) {
+  const uint64_t *ch = d.pool + (size_t)c * N;
+  if (lo32(ch[N - 1]) == LOCK_ZOMBIE) return false;
+  const uint32_t k0 = lo32(ch[0]);
+  if (k0 == KEY_NEG_INF || k0 == KEY_EMPTY) return false;  // first chunk / empty last chunk
+  minkey = k0;
+  return true;
+}
+
+// (1) mark min keys of the live non-first level-0 chunks
+template <int N>
+__global__ void __launch_bounds__(256) rebuild_mark_kernel(const __grid_constant__ DevState d, RebuildBufs b) {
+  pdl_wait();
+  const uint32_t used = min(d.bump[0], d.cap_bottom);
+  uint32_t cnt = 0;
+  for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < used; i += gridDim.x * blockDim.x) {
+    uint32_t k;
+    if (rb_candidate(d, d.cap_upper + i, N, k)) {
+      atomicOr(b.bitmap + (k >> 5), 1u << (k & 31));
+      ++cnt;
+    }
+  }
+  for (int o = 16; o; o >>= 1) cnt += __shfl_xor_sync(0xFFFFFFFFu, cnt, o);
+  if ((threadIdx.x & 31) == 0 && cnt) atomicAdd(b.n1, cnt);
+  if (blockIdx.x == 0 && threadIdx.x == 0) b.n1[1] = d.bump[1];
+}
+
+// (2) per-block popcount scan of the bitmap: one block of 1024 threads per 1024 words
+__global__ void __launch_bounds__(1024) rebuild_scan_kernel(RebuildBufs b) {
+  pdl_wait();
+  __shared__ uint32_t warp_tot[32];
+  const uint32_t w = blockIdx.x * RB_BLOCK_WORDS + threadIdx.x;
+  const uint32_t v = w < b.words ? __popc(b.bitmap[w]) : 0u;
+  uint32_t incl = v;
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  for (int o = 1; o < 32; o <<= 1) {
+    const uint32_t y = __shfl_up_sync(0xFFFFFFFFu, incl, o);
+    if (lane >= o) incl += y;
+  }
+  if (lane == 31) warp_tot[warp] = incl;
+  __syncthreads();
+  if (warp == 0) {
+    uint32_t t = warp_tot[lane], ti = t;
+    for (int o = 1; o < 32; o <<= 1) {
+      const uint32_t y = __shfl_up_sync(0xFFFFFFFFu, ti, o);
+      if (lane >= o) ti += y;
+    }
+    warp_tot[lane] = ti - t;  // exclusive
+    if (lane == 31) b.block_sum[blockIdx.x] = ti;
+  }
+  __syncthreads();
+  if (w < b.words) b.word_prefix[w] = warp_tot[warp] + incl - v;
+}
+
+// (3) exclusive scan of the block sums (one block)
+__global__ void __launch_bounds__(1024) rebuild_scan_top_kernel(RebuildBufs b) {
+  pdl_wait();
+  __shared__ uint32_t carry;
+  if (threadIdx.x == 0) carry = 0;
+  __syncthreads();
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  __shared__ uint32_t warp_tot[32];
+  for (uint32_t base = 0; base < b.blocks; base += 1024) {
+    const uint32_t i = base + threadIdx.x;
+    const uint32_t v = i < b.blocks ? b.block_sum[i] : 0u;
+    uint32_t incl = v;
+    for (int o = 1; o < 32; o <<= 1) {
+      const uint32_t y = __shfl_up_sync(0xFFFFFFFFu, incl, o);
+      if (lane >= o) incl += y;
+    }
+    if (lane == 31) warp_tot[warp] = incl;
+    __syncthreads();
+    if (warp == 0) {
+      uint32_t t = warp_tot[lane], ti = t;
+      for (int o = 1; o < 32; o <<= 1) {
+        const uint32_t y = __shfl_up_sync(0xFFFFFFFFu, ti, o);
+        if (lane >= o) ti += y;
+      }
+      warp_tot[lane] = ti - t;
+    }
+    __syncthreads();
+    if (i < b.blocks) b.block_sum[i] = carry + warp_tot[warp] + incl - v;
+    __syncthreads();
+    if (threadIdx.x == 1023) carry += warp_tot[warp] + incl;
+    __syncthreads();
+  }
+}
+
+// (4) each marked chunk writes itself at its rank
+template <int N>
+__global__ void __launch_bounds__(256) rebuild_rank_kernel(const __grid_constant__ DevState d, RebuildBufs b) {
+  pdl_wait();
+  const uint32_t used = min(d.bump[0], d.cap_bottom);
+  for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < used; i += gridDim.x * blockDim.x) {
+    const uint32_t c = d.cap_upper + i;
+    uint32_t k;
+    if (!rb_candidate(d, c, N, k)) continue;
+    const uint32_t w = k >> 5;
+    const uint32_t r = b.block_sum[w / RB_BLOCK_WORDS] + b.word_prefix[w] +
+                       __popc(b.bitmap[w] & ((1u << (k & 31)) - 1u));
+    b.order_key[r] = k;
+    b.order_chunk[r] = c;
+  }
+}
+
+// level geometry from n1 (identical in every thread)
+struct RbLevels {
+  uint32_t m[MAX_N];     // chunks of level l (l >= 1)
+  uint32_t base[MAX_N];  // index of chunk 1 of level l (chunk 0 is the head chunk l-1)
+  uint64_t pw[MAX_N];    // F^(l-1)
+  int top;               // highest rebuilt level (its m == 1)
+};
+
+template <int N>
+__device__ __forceinline__ void rb_levels(uint32_t n1, uint32_t F, RbLevels &L) {
+  uint32_t len = n1 + 1;  // |A_1| including -inf
+  uint32_t base = N - 1;
+  uint64_t pw = 1;
+  L.top = N - 1;
+  for (int l = 1; l < N; ++l) {
+    L.m[l] = (len + F - 1) / F;
+    L.base[l] = base;
+    L.pw[l] = pw;
+    base += L.m[l] - 1;
+    if (L.m[l] == 1) {
+      L.top = l;
+      for (int q = l + 1; q < N; ++q) {
+        L.m[q] = 1;
+        L.base[q] = base;
+        L.pw[q] = pw * F;
+      }
+      break;
+    }
+    len = L.m[l];
+    pw *= F;
+  }
+}
+
+template <int N>
+__device__ __forceinline__ uint32_t rb_chunk(const RbLevels &L, int l, uint32_t j) {
+  return j == 0 ? (uint32_t)(l - 1) : L.base[l] + j - 1;
+}
+
+// (5) write every chunk of levels >= 1; one thread per chunk
+template <int N>
+__global__ void __launch_bounds__(256) rebuild_pack_kernel(const __grid_constant__ DevState d, RebuildBufs b) {
+  pdl_wait();
+  const uint32_t n1 = b.n1[0];
+  const uint32_t F = b.fill;
+  RbLevels L;
+  rb_levels<N>(n1, F, L);
+  uint32_t total = 0;
+  for (int l = 1; l < N; ++l) total += L.m[l];
+  const uint32_t head0 = d.head[0];
+  for (uint32_t g = blockIdx.x * blockDim.x + threadIdx.x; g < total; g += gridDim.x * blockDim.x) {
+    int l = 1;
+    uint32_t j = g;
+    while (j >= L.m[l]) {
+      j -= L.m[l];
+      ++l;
+    }
+    // entries i in [j*F, (j+1)*F) of A_l, |A_l| = (l == 1 ? n1 + 1 : m[l-1]), or just the
+    // -inf entry for levels above the top
+    const uint32_t len = l > L.top ? 1u : (l == 1 ? n1 + 1 : L.m[l - 1]);
+    uint64_t *ch = d.pool + (size_t)rb_chunk<N>(L, l, j) * N;
+    uint32_t lastkey = 0;
+    for (int e = 0; e < N - 2; ++e) {
+      const uint32_t i = j * F + e;
+      uint64_t ent = EMPTY_ENTRY;
+      if (e < (int)F && i < len) {
+        uint32_t key, val;
+        if (i == 0) {
+          key = KEY_NEG_INF;
+          val = (l == 1) ? head0 : (uint32_t)(l - 2);
+        } else {
+          key = b.order_key[(uint64_t)i * L.pw[l] - 1];
+          val = (l == 1) ? b.order_chunk[i - 1] : rb_chunk<N>(L, l - 1, i);
+        }
+        ent = mk64(key, val);
+        lastkey = key;
+      }
+      ch[e] = ent;
+    }
+    const bool last = (j + 1 == L.m[l]);
+    ch[N - 2] = last ? mk64(KEY_POS_INF, NULL_CHUNK) : mk64(lastkey, rb_chunk<N>(L, l, j + 1));
+    ch[N - 1] = mk64(LOCK_FREE, 0u);
+  }
+  if (blockIdx.x == 0 && threadIdx.x < N && threadIdx.x >= 1) {
+    const int l = threadIdx.x;
+    d.head[l] = l - 1;
+    d.counter[l] = (l <= L.top && (l == 1 ? n1 > 0 : L.m[l - 1] > 1)) ? (int32_t)L.m[l] : 0;
+  }
+  if (blockIdx.x == 0 && threadIdx.x == 0) d.bump[1] = L.base[N - 1] + (L.top == N - 1 ? L.m[N - 1] - 1 : 0);
+}
+
+// (6) clear the bitmap marks; return the upper chunks past the new bump to the allocated
+// state; reset the counters for the next rebuild
+template <int N>
+__global__ void __launch_bounds__(256) rebuild_clear_kernel(const __grid_constant__ DevState d, RebuildBufs b) {
+  pdl_wait();
+  const uint32_t n1 = b.n1[0];
+  const uint32_t old_used = b.n1[1];
+  const uint32_t new_used = d.bump[1];
+  const uint32_t stride = gridDim.x * blockDim.x;
+  const uint32_t tid = blockIdx.x * blockDim.x + threadIdx.x;
+  for (uint32_t i = tid; i < n1; i += stride) b.bitmap[b.order_key[i] >> 5] = 0u;
+  if (old_used > new_used) {
+    const uint64_t first = (uint64_t)new_used * N, lastx = (uint64_t)old_used * N;
+    for (uint64_t e = first + tid; e < lastx; e += stride)
+      d.pool[e] = ((e % N) == (uint64_t)(N - 1)) ? (uint64_t)LOCK_HELD : EMPTY_ENTRY;
+  }
+}
+
+__global__ void rebuild_reset_kernel(RebuildBufs b) {
+  pdl_wait();
+  b.n1[0] = 0;
+}
+
+}  // namespace gfsl_dev

@@ -56,7 +56,6 @@ template <int N, int TEAM, bool COUNT = false>
 __global__ void __launch_bounds__(256)
 search_kernel(DevState d, uint8_t *__restrict__ res, const uint2 *__restrict__ list_c,
               const uint2 *__restrict__ list_u, BatchCtl *__restrict__ ctl, SearchOut so) {
-  constexpr int DSIZE = N - 2;
   constexpr int EPL = N / TEAM;
   static_assert(EPL * TEAM == N, "TEAM must divide N");
   constexpr int TPW = 32 / TEAM;                    // teams per warp

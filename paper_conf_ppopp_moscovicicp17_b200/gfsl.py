@@ -22,6 +22,7 @@ LIB_PATH = os.path.join(_HERE, "libgfsl.so")
 GFSL_OK, GFSL_EINVAL, GFSL_ENOMEM, GFSL_EPOOL, GFSL_ECUDA, GFSL_ECORRUPT = range(6)
 CONTAINS, INSERT, DELETE = 0, 1, 2
 RES_FALSE, RES_TRUE, RES_INVALID = 0, 1, 0xFF
+REBUILD_DEFAULT, REBUILD_NEVER = 0, 0xFFFFFFFF  # rebuild_every: library default period / never
 STATUS_NAMES = ["OK", "EINVAL", "ENOMEM", "EPOOL", "ECUDA", "ECORRUPT"]
 
 
@@ -31,7 +32,8 @@ class gfsl_config(ctypes.Structure):
                 ("update_blocks_per_sm", ctypes.c_uint32),
                 ("serial_updates", ctypes.c_uint32), ("count_reads", ctypes.c_uint32),
                 ("profile_phases", ctypes.c_uint32), ("l2_window", ctypes.c_uint32),
-                ("no_pdl", ctypes.c_uint32)]
+                ("no_pdl", ctypes.c_uint32),
+                ("rebuild_every", ctypes.c_uint32)]
 
 
 class gfsl_report(ctypes.Structure):
@@ -164,14 +166,16 @@ class GFSL:
     def __init__(self, key_range: int, capacity: int = 0, chunk_entries: int = 16,
                  contains_team: int = 0, serial_updates: bool = False,
                  contains_blocks_per_sm: int = 0, update_blocks_per_sm: int = 0,
-                 count_reads: bool = False, profile_phases: bool = False):
+                 count_reads: bool = False, profile_phases: bool = False,
+                 rebuild_every: int = 0):
         import torch
         if not torch.cuda.is_available():
             raise RuntimeError("GFSL needs a CUDA device (there is no CPU fallback)")
         self.lib = load_library()
         cfg = gfsl_config(chunk_entries, contains_team, contains_blocks_per_sm,
                           update_blocks_per_sm, 1 if serial_updates else 0,
-                          1 if count_reads else 0, 1 if profile_phases else 0)
+                          1 if count_reads else 0, 1 if profile_phases else 0, 0, 0,
+                          rebuild_every)
         self.key_range = int(key_range)
         self.chunk_entries = int(chunk_entries)
         self.cfg = cfg

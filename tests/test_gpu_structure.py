@@ -9,16 +9,17 @@ import pytest
 import torch
 
 from oracle.oracle_b import GFSLModel
-from paper_conf_ppopp_moscovicicp17_b200.gfsl import GFSL
+from paper_conf_ppopp_moscovicicp17_b200.gfsl import GFSL, REBUILD_NEVER
 from paper_conf_ppopp_moscovicicp17_b200.workload import SEED_BASE, Workload
 from tests import gfsl_fixtures as fx
 
 pytestmark = pytest.mark.gpu
 
 
-def model_like(g: GFSL, key_range):
+def model_like(g: GFSL, key_range, rebuild_every=0):
     meta, _ = g.dump()
-    return GFSLModel(meta["chunk_entries"], key_range, meta["cap_bottom"], meta["cap_upper"])
+    return GFSLModel(meta["chunk_entries"], key_range, meta["cap_bottom"], meta["cap_upper"],
+                     rebuild_every=rebuild_every)
 
 
 def assert_same_structure(g: GFSL, m: GFSLModel, where=""):
@@ -52,7 +53,7 @@ def dev(op, key, val):
     (16, 300, 150, 30, (45, 55, 0)),
 ])
 def test_serial_mode_is_byte_identical_to_oracle_b(N, R, B, nb, mix):
-    g = GFSL(R, chunk_entries=N, serial_updates=True)
+    g = GFSL(R, chunk_entries=N, serial_updates=True, rebuild_every=REBUILD_NEVER)
     m = model_like(g, R)
     assert_same_structure(g, m, "init")
     w = Workload(R, B, mix=mix, seed=SEED_BASE + 17 * N)
@@ -74,7 +75,7 @@ def test_serial_fill_then_drain_byte_identical(N):
     """Grow to a multi-level structure, then delete most keys: merges, splitRemove,
     zombies, level counters going back down."""
     R = 6000
-    g = GFSL(R, chunk_entries=N, serial_updates=True)
+    g = GFSL(R, chunk_entries=N, serial_updates=True, rebuild_every=REBUILD_NEVER)
     m = model_like(g, R)
     rng = np.random.default_rng(N)
     perm = rng.permutation(R).astype(np.uint32)
@@ -92,10 +93,28 @@ def test_serial_fill_then_drain_byte_identical(N):
     assert g.stats()["merges"] > 0
 
 
+@pytest.mark.parametrize("N,every", [(16, 1), (32, 2), (6, 1), (12, 3), (16, 0)])
+def test_serial_with_rebuild_byte_identical(N, every):
+    """R24 on the GPU (rebuild kernels) equals Oracle-B's rebuild, entry for entry."""
+    R = 3000 if N >= 16 else 500
+    g = GFSL(R, chunk_entries=N, serial_updates=True, rebuild_every=every)
+    m = model_like(g, R, rebuild_every=every or 2)  # 0 = the library default period (2)
+    w = Workload(R, R // 4, mix=(30, 30, 40), seed=SEED_BASE + 5 * N)
+    for b in range(14):
+        op, key, val, _ = w.make_batch(b)
+        opn, kn, vn = op.numpy(), key.numpy().astype(np.uint32), val.numpy().astype(np.uint32)
+        r_gpu = g.batch(*dev(opn, kn, vn)).cpu().numpy()
+        r_ora = np.array(m.batch(opn.tolist(), kn.tolist(), vn.tolist()), np.uint8)
+        assert np.array_equal(r_gpu, r_ora), f"batch {b}"
+        assert_same_structure(g, m, f"after batch {b}")
+    rep, _, _ = g.validate()
+    assert rep.violations == 0
+
+
 def run_fixture_on_gpu(spec, N, ops, keys, vals=None):
     """Loads the fixture into a GPU handle with the same pool geometry as Oracle-B,
     runs one serial batch on both, and checks they end identical."""
-    g = GFSL(100, capacity=64, chunk_entries=N, serial_updates=True)
+    g = GFSL(100, capacity=64, chunk_entries=N, serial_updates=True, rebuild_every=REBUILD_NEVER)
     meta0, _ = g.dump()
     m, names = fx.build(spec, N, key_range=100, cap_bottom=meta0["cap_bottom"],
                         cap_upper=meta0["cap_upper"])

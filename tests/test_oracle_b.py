@@ -119,3 +119,25 @@ def test_model_matches_oracle_a(N):
         ok, ov = o.export()
         assert ks == ok.tolist() and vs == ov.tolist()
         assert m.check_invariants() == []
+
+
+@pytest.mark.parametrize("N,every", [(6, 1), (12, 2), (16, 1), (32, 3)])
+def test_model_with_rebuild_matches_oracle_a(N, every):
+    """R24: rebuilding the upper levels between batches changes no result and keeps
+    every invariant; after a rebuild every level-0 chunk is the target of a level-1 key."""
+    R = 400 if N <= 12 else 2000
+    m = GFSLModel(N, R, cap_bottom=4000, cap_upper=1000, rebuild_every=every)
+    o = OracleMap(R)
+    w = Workload(R, 150, mix=(35, 35, 30), seed=SEED_BASE + 3 * N)
+    for b in range(24):
+        op, key, val, _ = w.make_batch(b)
+        opn, kn, vn = op.numpy(), key.numpy().astype(np.uint32), val.numpy().astype(np.uint32)
+        assert m.batch(opn.tolist(), kn.tolist(), vn.tolist()) == o.batch(opn, kn, vn).tolist()
+        ks, vs = m.export()
+        ok, ov = o.export()
+        assert ks == ok.tolist() and vs == ov.tolist()
+        assert m.check_invariants() == []
+        if (b + 1) % every == 0:
+            l0 = [c for c in m.level_chain(0) if not m.zombie(c)][1:]
+            targets = {V(e) for c in m.level_chain(1) for e in m.pool[c][: m.DSIZE] if K(e) != INF}
+            assert all(c in targets for c in l0 if m.keys(c)[0] != INF)
