@@ -49,6 +49,7 @@ class GFSLModel:
         assert N >= 6
         self.rebuild_every = rebuild_every
         self.batches = 0
+        self.dirty = False
         self.N, self.DSIZE, self.NEXT, self.LOCK, self.MAXL = N, N - 2, N - 2, N - 1, N
         self.key_range = key_range
         self.cap_bottom, self.cap_upper = cap_bottom, cap_upper
@@ -462,8 +463,11 @@ class GFSLModel:
                 res[i] = 0
         if self.merges:
             self.upkeep()
-        if n and self.rebuild_every and (self.batches + 1) % self.rebuild_every == 0:
+        if plans:
+            self.dirty = True  # a mutating batch since the last rebuild
+        if n and self.rebuild_every and (self.batches + 1) % self.rebuild_every == 0 and self.dirty:
             self.rebuild()
+            self.dirty = False
         if n:
             self.batches += 1
         return res

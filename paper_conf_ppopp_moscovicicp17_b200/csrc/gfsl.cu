@@ -285,6 +285,10 @@ static void launch_update(gfsl *h, const uint8_t *ops, const uint32_t *keys, con
   const uint32_t every = h->cfg.rebuild_every == 0 ? GFSL_REBUILD_DEFAULT_PERIOD : h->cfg.rebuild_every;
   if (every != GFSL_REBUILD_NEVER && (h->batches + 1) % every == 0) {
     const RebuildBufs &b = h->rb;
+    lc.gridDim = dim3(1);
+    lc.blockDim = dim3(32);
+    cudaLaunchKernelEx(&lc, rebuild_begin_kernel, b);
+    lc.blockDim = dim3(256);
     lc.gridDim = dim3(h->sms * 4);
     cudaLaunchKernelEx(&lc, rebuild_mark_kernel<N>, h->d, b);
     lc.gridDim = dim3(b.blocks);
@@ -295,13 +299,10 @@ static void launch_update(gfsl *h, const uint8_t *ops, const uint32_t *keys, con
     lc.blockDim = dim3(256);
     lc.gridDim = dim3(h->sms * 4);
     cudaLaunchKernelEx(&lc, rebuild_rank_kernel<N>, h->d, b);
-    lc.gridDim = dim3(h->sms * 2);
+    lc.gridDim = dim3(h->sms * 8);
     cudaLaunchKernelEx(&lc, rebuild_pack_kernel<N>, h->d, b);
     lc.gridDim = dim3(h->sms * 4);
     cudaLaunchKernelEx(&lc, rebuild_clear_kernel<N>, h->d, b);
-    lc.gridDim = dim3(1);
-    lc.blockDim = dim3(32);
-    cudaLaunchKernelEx(&lc, rebuild_reset_kernel, b);
   }
 }
 
@@ -482,9 +483,10 @@ extern "C" gfsl_t gfsl_create_ex(uint64_t key_range, uint64_t capacity, const gf
     if ((e = cudaMalloc(&b.block_sum, (size_t)b.blocks * 4)) != cudaSuccess) return fail("cudaMalloc(rebuild)", e);
     if ((e = cudaMalloc(&b.order_key, (size_t)cap_b * 4)) != cudaSuccess) return fail("cudaMalloc(rebuild)", e);
     if ((e = cudaMalloc(&b.order_chunk, (size_t)cap_b * 4)) != cudaSuccess) return fail("cudaMalloc(rebuild)", e);
-    if ((e = cudaMalloc(&b.n1, 8)) != cudaSuccess) return fail("cudaMalloc(rebuild)", e);
+    if ((e = cudaMalloc(&b.n1, 16)) != cudaSuccess) return fail("cudaMalloc(rebuild)", e);
     cudaMemset(b.bitmap, 0, (size_t)b.words * 4);
-    cudaMemset(b.n1, 0, 8);
+    cudaMemset(b.n1, 0, 16);
+    h->d.dirty = b.n1 + 2;
   }
   cudaMemset(h->d.head, 0xFF, 32 * 4);
   cudaMemset(h->d.counter, 0, 32 * 4);

@@ -55,6 +55,7 @@ struct DevState {
   uint32_t cap_upper;    // upper-pool chunks, indices [0, cap_upper)
   uint32_t key_max;      // largest valid internal key (= key_range)
   BatchCtl *ctl;         // the handle's per-batch control block
+  uint32_t *dirty;       // set when a batch mutated the structure (-> upper-level rebuild)
 };
 
 // Per-batch control block (device memory, zeroed before every batch).

@@ -29,7 +29,7 @@ struct RebuildBufs {
   uint32_t *block_sum;    // [blocks]     popcount of each block, then its exclusive prefix
   uint32_t *order_key;    // [cap_bottom] min keys in key order
   uint32_t *order_chunk;  // [cap_bottom] their chunks
-  uint32_t *n1;           // [2]          marked chunks; old upper bump
+  uint32_t *n1;           // [4]          marked chunks; old upper bump; dirty; active
   uint32_t words, blocks;
   uint32_t fill;          // F: entries per rebuilt upper chunk
 };
@@ -45,27 +45,34 @@ __device__ __forceinline__ bool rb_candidate(const DevState &d, uint32_t c, int 
   return true;
 }
 
+// A rebuild is skipped when no batch mutated the structure since the last one: n1[2] is
+// the dirty flag (set by the update kernel), n1[3] says whether this rebuild runs.
+__device__ __forceinline__ bool rb_active(const RebuildBufs &b) { return *(volatile uint32_t *)(b.n1 + 3) != 0; }
+
+// (0) decide (one thread)
+__global__ void rebuild_begin_kernel(RebuildBufs b) {
+  pdl_wait();
+  b.n1[3] = b.n1[2];
+  b.n1[2] = 0;
+}
+
 // (1) mark min keys of the live non-first level-0 chunks
 template <int N>
 __global__ void __launch_bounds__(256) rebuild_mark_kernel(const __grid_constant__ DevState d, RebuildBufs b) {
   pdl_wait();
+  if (!rb_active(b)) return;
   const uint32_t used = min(d.bump[0], d.cap_bottom);
-  uint32_t cnt = 0;
   for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < used; i += gridDim.x * blockDim.x) {
     uint32_t k;
-    if (rb_candidate(d, d.cap_upper + i, N, k)) {
-      atomicOr(b.bitmap + (k >> 5), 1u << (k & 31));
-      ++cnt;
-    }
+    if (rb_candidate(d, d.cap_upper + i, N, k)) atomicOr(b.bitmap + (k >> 5), 1u << (k & 31));
   }
-  for (int o = 16; o; o >>= 1) cnt += __shfl_xor_sync(0xFFFFFFFFu, cnt, o);
-  if ((threadIdx.x & 31) == 0 && cnt) atomicAdd(b.n1, cnt);
   if (blockIdx.x == 0 && threadIdx.x == 0) b.n1[1] = d.bump[1];
 }
 
 // (2) per-block popcount scan of the bitmap: one block of 1024 threads per 1024 words
 __global__ void __launch_bounds__(1024) rebuild_scan_kernel(RebuildBufs b) {
   pdl_wait();
+  if (!rb_active(b)) return;
   __shared__ uint32_t warp_tot[32];
   const uint32_t w = blockIdx.x * RB_BLOCK_WORDS + threadIdx.x;
   const uint32_t v = w < b.words ? __popc(b.bitmap[w]) : 0u;
@@ -93,6 +100,7 @@ __global__ void __launch_bounds__(1024) rebuild_scan_kernel(RebuildBufs b) {
 // (3) exclusive scan of the block sums (one block)
 __global__ void __launch_bounds__(1024) rebuild_scan_top_kernel(RebuildBufs b) {
   pdl_wait();
+  if (!rb_active(b)) return;
   __shared__ uint32_t carry;
   if (threadIdx.x == 0) carry = 0;
   __syncthreads();
@@ -122,12 +130,14 @@ __global__ void __launch_bounds__(1024) rebuild_scan_top_kernel(RebuildBufs b) {
     if (threadIdx.x == 1023) carry += warp_tot[warp] + incl;
     __syncthreads();
   }
+  if (threadIdx.x == 0) b.n1[0] = carry;  // marked chunks = total popcount
 }
 
 // (4) each marked chunk writes itself at its rank
 template <int N>
 __global__ void __launch_bounds__(256) rebuild_rank_kernel(const __grid_constant__ DevState d, RebuildBufs b) {
   pdl_wait();
+  if (!rb_active(b)) return;
   const uint32_t used = min(d.bump[0], d.cap_bottom);
   for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < used; i += gridDim.x * blockDim.x) {
     const uint32_t c = d.cap_upper + i;
@@ -179,10 +189,11 @@ __device__ __forceinline__ uint32_t rb_chunk(const RbLevels &L, int l, uint32_t 
   return j == 0 ? (uint32_t)(l - 1) : L.base[l] + j - 1;
 }
 
-// (5) write every chunk of levels >= 1; one thread per chunk
+// (5) write every chunk of levels >= 1; one warp per chunk, lane e writes entry e
 template <int N>
 __global__ void __launch_bounds__(256) rebuild_pack_kernel(const __grid_constant__ DevState d, RebuildBufs b) {
   pdl_wait();
+  if (!rb_active(b)) return;
   const uint32_t n1 = b.n1[0];
   const uint32_t F = b.fill;
   RbLevels L;
@@ -190,7 +201,10 @@ __global__ void __launch_bounds__(256) rebuild_pack_kernel(const __grid_constant
   uint32_t total = 0;
   for (int l = 1; l < N; ++l) total += L.m[l];
   const uint32_t head0 = d.head[0];
-  for (uint32_t g = blockIdx.x * blockDim.x + threadIdx.x; g < total; g += gridDim.x * blockDim.x) {
+  const int lane = threadIdx.x & 31;
+  const uint32_t warp = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  const uint32_t nwarps = (gridDim.x * blockDim.x) >> 5;
+  for (uint32_t g = warp; g < total; g += nwarps) {
     int l = 1;
     uint32_t j = g;
     while (j >= L.m[l]) {
@@ -201,27 +215,28 @@ __global__ void __launch_bounds__(256) rebuild_pack_kernel(const __grid_constant
     // -inf entry for levels above the top
     const uint32_t len = l > L.top ? 1u : (l == 1 ? n1 + 1 : L.m[l - 1]);
     uint64_t *ch = d.pool + (size_t)rb_chunk<N>(L, l, j) * N;
-    uint32_t lastkey = 0;
-    for (int e = 0; e < N - 2; ++e) {
-      const uint32_t i = j * F + e;
-      uint64_t ent = EMPTY_ENTRY;
-      if (e < (int)F && i < len) {
-        uint32_t key, val;
-        if (i == 0) {
-          key = KEY_NEG_INF;
-          val = (l == 1) ? head0 : (uint32_t)(l - 2);
-        } else {
-          key = b.order_key[(uint64_t)i * L.pw[l] - 1];
-          val = (l == 1) ? b.order_chunk[i - 1] : rb_chunk<N>(L, l - 1, i);
-        }
-        ent = mk64(key, val);
-        lastkey = key;
+    const uint32_t i = j * F + lane;
+    uint64_t ent = EMPTY_ENTRY;
+    uint32_t key = 0;
+    const bool has = lane < N - 2 && lane < (int)F && i < len;
+    if (has) {
+      uint32_t val;
+      if (i == 0) {
+        key = KEY_NEG_INF;
+        val = (l == 1) ? head0 : (uint32_t)(l - 2);
+      } else {
+        key = b.order_key[(uint64_t)i * L.pw[l] - 1];
+        val = (l == 1) ? b.order_chunk[i - 1] : rb_chunk<N>(L, l - 1, i);
       }
-      ch[e] = ent;
+      ent = mk64(key, val);
     }
+    const uint32_t hb = __ballot_sync(0xFFFFFFFFu, has);
+    const int lastlane = 31 - __clz(hb);
+    const uint32_t lastkey = __shfl_sync(0xFFFFFFFFu, key, lastlane);
     const bool last = (j + 1 == L.m[l]);
-    ch[N - 2] = last ? mk64(KEY_POS_INF, NULL_CHUNK) : mk64(lastkey, rb_chunk<N>(L, l, j + 1));
-    ch[N - 1] = mk64(LOCK_FREE, 0u);
+    if (lane < N - 2) ch[lane] = ent;
+    else if (lane == N - 2) ch[N - 2] = last ? mk64(KEY_POS_INF, NULL_CHUNK) : mk64(lastkey, rb_chunk<N>(L, l, j + 1));
+    else if (lane == N - 1) ch[N - 1] = mk64(LOCK_FREE, 0u);
   }
   if (blockIdx.x == 0 && threadIdx.x < N && threadIdx.x >= 1) {
     const int l = threadIdx.x;
@@ -236,6 +251,7 @@ __global__ void __launch_bounds__(256) rebuild_pack_kernel(const __grid_constant
 template <int N>
 __global__ void __launch_bounds__(256) rebuild_clear_kernel(const __grid_constant__ DevState d, RebuildBufs b) {
   pdl_wait();
+  if (!rb_active(b)) return;
   const uint32_t n1 = b.n1[0];
   const uint32_t old_used = b.n1[1];
   const uint32_t new_used = d.bump[1];
@@ -249,9 +265,5 @@ __global__ void __launch_bounds__(256) rebuild_clear_kernel(const __grid_constan
   }
 }
 
-__global__ void rebuild_reset_kernel(RebuildBufs b) {
-  pdl_wait();
-  b.n1[0] = 0;
-}
 
 }  // namespace gfsl_dev
