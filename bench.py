@@ -341,6 +341,7 @@ def run_gpu(args, world, rank, local):
     c_ms = phases["contains"] / max(nbat, 1)
     u_ms = phases["update"] / max(nbat, 1)
     i_ms = phases["intake"] / max(nbat, 1)
+    k_ms = phases["upkeep"] / max(nbat, 1)
 
     def roof(bytes_per_launch, ms, kernel):
         if ms <= 0 or bytes_per_launch <= 0:
@@ -420,7 +421,8 @@ def run_gpu(args, world, rank, local):
             "steps": steps, "warmup": W, "ms_per_step": round(total_ms / steps, 4),
             "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
             "dtype": "u32", "data": "synthetic",
-            "config": {"workload": args.config, "key_range": R, "rebuild_every": args.rebuild_every, "prefill": pre1 * world,
+            "config": {"workload": args.config, "key_range": R,
+                       "rebuild_every": "never" if args.rebuild_every < 0 else (args.rebuild_every or 2), "prefill": pre1 * world,
                        "batch_ops": B1 * world, "mix_ins_del_con": list(mix), "keys": dist,
                        "chunk_entries": N, "contains_team": local_g.cfg.contains_team or (4 if N == 32 else 2),
                        "l2": "flushed (256 MiB write) between timed steps",
@@ -431,7 +433,7 @@ def run_gpu(args, world, rank, local):
             "random_access_roofline": rand,
             "mutations_per_step": round(n_mut, 1),
             "phase_ms_per_step": {"intake": round(i_ms, 4), "search": round(c_ms, 4),
-                                  "update": round(u_ms, 4)},
+                                  "update": round(u_ms, 4), "upkeep_rebuild": round(k_ms, 4)},
             "chunk_reads_per_contains": round(reads_per_op, 3),
             "chunk_reads_l0_per_contains": round(reads_l0_per_op, 3),
             "cpu_baseline": cpu,

@@ -175,8 +175,9 @@ gfsl_status gfsl_get_stats(gfsl_t h, gfsl_stats *out);
 
 /*
  * Per-phase device time of the batches enqueued since the last call (profile_phases=1):
- * ms[0] intake (memset + classify), ms[1] Contains kernel, ms[2] update kernel,
- * ms[3] whole batches; *batches = how many.  Synchronizes the device; resets the sums.
+ * ms[0] intake (memset + classify), ms[1] search kernel, ms[2] update kernel,
+ * ms[3] upkeep + upper-level rebuild, ms[4] whole batches (ms must hold 5 doubles);
+ * *batches = how many.  Synchronizes the device; resets the sums.
  */
 gfsl_status gfsl_phase_times(gfsl_t h, double *ms, uint64_t *batches);
 

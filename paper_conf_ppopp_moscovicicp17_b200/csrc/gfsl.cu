@@ -61,7 +61,7 @@ struct gfsl {
   uint32_t *st_key = nullptr, *st_val = nullptr;
   uint64_t st_cap = 0;
   uint64_t batches = 0, ops = 0;
-  std::vector<std::array<cudaEvent_t, 4>> phase_ev;  // profile_phases
+  std::vector<std::array<cudaEvent_t, 5>> phase_ev;  // profile_phases
   // L2 persistence for the upper pool (the search kernel's access-policy window)
   size_t persist_max = 0, window_max = 0;
   uint32_t *h_bump = nullptr;  // pinned copy of the bump counters, refreshed every batch
@@ -265,7 +265,7 @@ static bool dispatch_contains(gfsl *h, const uint8_t *ops, const uint32_t *keys,
 
 template <int N>
 static void launch_update(gfsl *h, const uint8_t *ops, const uint32_t *keys, const uint32_t *vals,
-                          uint8_t *res, uint32_t n, cudaStream_t s) {
+                          uint8_t *res, uint32_t n, cudaStream_t s, cudaEvent_t after_update) {
   (void)n;
   cudaLaunchConfig_t lc{};
   cudaLaunchAttribute attr[1];
@@ -278,6 +278,7 @@ static void launch_update(gfsl *h, const uint8_t *ops, const uint32_t *keys, con
   const int serial = h->cfg.serial_updates ? 1 : 0;
   cudaLaunchKernelEx(&lc, update_kernel<N>, h->d, vals, res, (const uint2 *)h->list_u, h->ctl,
                      search_out(h), serial);
+  if (after_update) cudaEventRecord(after_update, s);
   lc.blockDim = dim3(256);
   lc.gridDim = dim3(h->sms * 4);
   cudaLaunchKernelEx(&lc, upkeep_kernel<N>, h->d);
@@ -573,7 +574,7 @@ static gfsl_status ensure_lists(gfsl *h, uint64_t n) {
 static gfsl_status enqueue_batch(gfsl *h, const uint8_t *ops, const uint32_t *keys,
                                  const uint32_t *vals, uint8_t *res, uint64_t n, cudaStream_t s) {
   CK(cudaStreamWaitEvent(s, h->last, 0));
-  std::array<cudaEvent_t, 4> ev{};
+  std::array<cudaEvent_t, 5> ev{};
   const bool prof = h->cfg.profile_phases != 0;
   if (prof) {
     for (auto &e : ev) CK(cudaEventCreate(&e));
@@ -596,10 +597,10 @@ static gfsl_status enqueue_batch(gfsl *h, const uint8_t *ops, const uint32_t *ke
     return GFSL_EINVAL;
   }
   switch (h->N) {
-    case 32: launch_update<32>(h, ops, keys, vals, res, (uint32_t)n, s); break;
-    case 16: launch_update<16>(h, ops, keys, vals, res, (uint32_t)n, s); break;
-    case 12: launch_update<12>(h, ops, keys, vals, res, (uint32_t)n, s); break;
-    case 6: launch_update<6>(h, ops, keys, vals, res, (uint32_t)n, s); break;
+    case 32: launch_update<32>(h, ops, keys, vals, res, (uint32_t)n, s, prof ? ev[3] : nullptr); break;
+    case 16: launch_update<16>(h, ops, keys, vals, res, (uint32_t)n, s, prof ? ev[3] : nullptr); break;
+    case 12: launch_update<12>(h, ops, keys, vals, res, (uint32_t)n, s, prof ? ev[3] : nullptr); break;
+    case 6: launch_update<6>(h, ops, keys, vals, res, (uint32_t)n, s, prof ? ev[3] : nullptr); break;
   }
   cudaError_t e = cudaGetLastError();
   if (e != cudaSuccess) {
@@ -608,7 +609,7 @@ static gfsl_status enqueue_batch(gfsl *h, const uint8_t *ops, const uint32_t *ke
     return GFSL_ECUDA;
   }
   if (prof) {
-    CK(cudaEventRecord(ev[3], s));
+    CK(cudaEventRecord(ev[4], s));
     h->phase_ev.push_back(ev);
   }
   CK(cudaMemcpyAsync(h->h_bump, h->d.bump, 8, cudaMemcpyDeviceToHost, s));
@@ -700,20 +701,22 @@ extern "C" gfsl_status gfsl_get_stats(gfsl_t h, gfsl_stats *out) {
 extern "C" gfsl_status gfsl_phase_times(gfsl_t h, double *ms, uint64_t *batches) {
   if (!h || !ms) return GFSL_EINVAL;
   CK(cudaDeviceSynchronize());
-  double acc[4] = {0, 0, 0, 0};
+  double acc[5] = {0, 0, 0, 0, 0};
   for (auto &ev : h->phase_ev) {
-    float a = 0, b = 0, c = 0, t = 0;
+    float a = 0, b = 0, c = 0, u = 0, t = 0;
     CK(cudaEventElapsedTime(&a, ev[0], ev[1]));
     CK(cudaEventElapsedTime(&b, ev[1], ev[2]));
     CK(cudaEventElapsedTime(&c, ev[2], ev[3]));
-    CK(cudaEventElapsedTime(&t, ev[0], ev[3]));
+    CK(cudaEventElapsedTime(&u, ev[3], ev[4]));
+    CK(cudaEventElapsedTime(&t, ev[0], ev[4]));
     acc[0] += a;
     acc[1] += b;
     acc[2] += c;
-    acc[3] += t;
+    acc[3] += u;
+    acc[4] += t;
     for (auto &e : ev) cudaEventDestroy(e);
   }
-  for (int i = 0; i < 4; ++i) ms[i] = acc[i];
+  for (int i = 0; i < 5; ++i) ms[i] = acc[i];
   if (batches) *batches = h->phase_ev.size();
   h->phase_ev.clear();
   return GFSL_OK;

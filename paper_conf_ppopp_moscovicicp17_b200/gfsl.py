@@ -255,10 +255,10 @@ class GFSL:
 
     def phase_times(self):
         """(ms dict of intake/contains/update/total since the last call, batches)."""
-        ms = (ctypes.c_double * 4)()
+        ms = (ctypes.c_double * 5)()
         nb = ctypes.c_uint64()
         _check(self.lib.gfsl_phase_times(self.h, ms, ctypes.byref(nb)), "gfsl_phase_times")
-        return dict(intake=ms[0], contains=ms[1], update=ms[2], total=ms[3]), nb.value
+        return dict(intake=ms[0], contains=ms[1], update=ms[2], upkeep=ms[3], total=ms[4]), nb.value
 
     def dump(self):
         """(meta dict, entries uint64 array of shape [chunks, N]) -- test-only."""

@@ -1,0 +1,24 @@
+"""Small end-to-end run for compute-sanitizer: concurrent and serial batches with splits,
+merges, zombies, upkeep and rebuilds, checked against the oracle."""
+import os, sys
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+import numpy as np
+import torch
+from oracle.oracle_a import OracleMap
+from paper_conf_ppopp_moscovicicp17_b200.gfsl import GFSL
+from paper_conf_ppopp_moscovicicp17_b200.workload import SEED_BASE, Workload
+
+dev = torch.device("cuda")
+for N, serial in [(16, False), (32, False), (16, True)]:
+    R = 3000
+    g = GFSL(R, chunk_entries=N, serial_updates=serial, rebuild_every=1)
+    o = OracleMap(R)
+    w = Workload(R, 800, mix=(40, 40, 20), seed=SEED_BASE + N)
+    for b in range(10):
+        op, key, val, _ = w.make_batch(b)
+        r = g.batch(op.to(dev), key.to(torch.int32).to(dev), val.to(torch.int32).to(dev)).cpu().numpy()
+        e = o.batch(op.numpy(), key.numpy().astype(np.uint32), val.numpy().astype(np.uint32))
+        assert np.array_equal(r, e)
+    rep, ks, vs = g.validate()
+    assert rep.violations == 0 and np.array_equal(ks, o.export()[0])
+    print("ok", N, serial, g.stats())
