@@ -50,6 +50,7 @@ class GFSLModel:
         self.rebuild_every = rebuild_every
         self.batches = 0
         self.dirty = False
+        self.free, self.free_taken = [], 0  # R25 free list of reclaimed level-0 chunks
         self.N, self.DSIZE, self.NEXT, self.LOCK, self.MAXL = N, N - 2, N - 2, N - 1, N
         self.key_range = key_range
         self.cap_bottom, self.cap_upper = cap_bottom, cap_upper
@@ -121,6 +122,10 @@ class GFSLModel:
         ch[self.LOCK] = E(state, V(ch[self.LOCK]) + 1)
 
     def alloc(self, level):  # bump a counter, the chunk is already +inf and locked
+        if level == 0 and self.free_taken < len(self.free):  # R25: reclaimed chunks first
+            c = self.free[self.free_taken]
+            self.free_taken += 1
+            return c
         p = 1 if level > 0 else 0
         cap = self.cap_upper if p else self.cap_bottom
         i = self.bump[p]
@@ -467,10 +472,20 @@ class GFSLModel:
             self.dirty = True  # a mutating batch since the last rebuild
         if n and self.rebuild_every and (self.batches + 1) % self.rebuild_every == 0 and self.dirty:
             self.rebuild()
+            self.reclaim()
             self.dirty = False
         if n:
             self.batches += 1
         return res
+
+    def reclaim(self):
+        """R25: after a rebuild no pointer reaches a zombie; reset them to the allocated
+        state and append them (ascending) after the unused part of the free list."""
+        zombies = [self.cap_upper + i for i in range(self.bump[0]) if self.zombie(self.cap_upper + i)]
+        for c in zombies:
+            self.pool[c] = [EMPTY] * (self.N - 1) + [HELD]
+        self.free = self.free[self.free_taken:] + zombies
+        self.free_taken = 0
 
     def rebuild(self):
         """R24: re-derive levels >= 1 from level 0 between batches ("compact the

@@ -66,6 +66,7 @@ struct gfsl {
   size_t persist_max = 0, window_max = 0;
   uint32_t *h_bump = nullptr;  // pinned copy of the bump counters, refreshed every batch
   RebuildBufs rb{};            // upper-level rebuild (R24)
+  uint32_t *rc_tiles = nullptr;  // zombie reclamation scratch (R25)
 };
 
 // ------------------------------------------------------------------------------------
@@ -296,14 +297,21 @@ static void launch_update(gfsl *h, const uint8_t *ops, const uint32_t *keys, con
     lc.blockDim = dim3(1024);
     cudaLaunchKernelEx(&lc, rebuild_scan_kernel, b);
     lc.gridDim = dim3(1);
-    cudaLaunchKernelEx(&lc, rebuild_scan_top_kernel, b);
+    cudaLaunchKernelEx(&lc, rebuild_scan_top_kernel<N>, b);
     lc.blockDim = dim3(256);
     lc.gridDim = dim3(h->sms * 4);
     cudaLaunchKernelEx(&lc, rebuild_rank_kernel<N>, h->d, b);
     lc.gridDim = dim3(h->sms * 8);
     cudaLaunchKernelEx(&lc, rebuild_pack_kernel<N>, h->d, b);
+    // R25: reclaim the (now unreachable) zombie level-0 chunks (+ the bitmap clear)
     lc.gridDim = dim3(h->sms * 4);
-    cudaLaunchKernelEx(&lc, rebuild_clear_kernel<N>, h->d, b);
+    cudaLaunchKernelEx(&lc, reclaim_count_kernel<N>, h->d, b, h->rc_tiles);
+    lc.gridDim = dim3(1);
+    lc.blockDim = dim3(1024);
+    cudaLaunchKernelEx(&lc, reclaim_scan_kernel, h->d, b, h->rc_tiles);
+    lc.gridDim = dim3(h->sms * 4);
+    lc.blockDim = dim3(256);
+    cudaLaunchKernelEx(&lc, reclaim_write_kernel<N>, h->d, b, (const uint32_t *)h->rc_tiles);
   }
 }
 
@@ -403,6 +411,10 @@ static void free_all(gfsl *h) {
   cudaFree(h->rb.order_key);
   cudaFree(h->rb.order_chunk);
   cudaFree(h->rb.n1);
+  cudaFree(h->rb.levels);
+  cudaFree(h->rc_tiles);
+  cudaFree(h->d.freelist);
+  cudaFree(h->d.fl);
   if (h->h_error) cudaFreeHost(h->h_error);
   if (h->h_bump) cudaFreeHost(h->h_bump);
   if (h->last) cudaEventDestroy(h->last);
@@ -485,9 +497,14 @@ extern "C" gfsl_t gfsl_create_ex(uint64_t key_range, uint64_t capacity, const gf
     if ((e = cudaMalloc(&b.order_key, (size_t)cap_b * 4)) != cudaSuccess) return fail("cudaMalloc(rebuild)", e);
     if ((e = cudaMalloc(&b.order_chunk, (size_t)cap_b * 4)) != cudaSuccess) return fail("cudaMalloc(rebuild)", e);
     if ((e = cudaMalloc(&b.n1, 16)) != cudaSuccess) return fail("cudaMalloc(rebuild)", e);
+    if ((e = cudaMalloc(&b.levels, sizeof(RbLevels))) != cudaSuccess) return fail("cudaMalloc(rebuild)", e);
     cudaMemset(b.bitmap, 0, (size_t)b.words * 4);
     cudaMemset(b.n1, 0, 16);
     h->d.dirty = b.n1 + 2;
+    if ((e = cudaMalloc(&h->d.freelist, (size_t)cap_b * 8)) != cudaSuccess) return fail("cudaMalloc(freelist)", e);
+    if ((e = cudaMalloc(&h->d.fl, 8 * 4)) != cudaSuccess) return fail("cudaMalloc(freelist)", e);
+    if ((e = cudaMalloc(&h->rc_tiles, ((size_t)cap_b / RC_TILE + 2) * 4)) != cudaSuccess) return fail("cudaMalloc(reclaim)", e);
+    cudaMemset(h->d.fl, 0, 8 * 4);
   }
   cudaMemset(h->d.head, 0xFF, 32 * 4);
   cudaMemset(h->d.counter, 0, 32 * 4);

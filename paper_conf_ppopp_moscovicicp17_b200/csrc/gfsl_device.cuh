@@ -56,6 +56,9 @@ struct DevState {
   uint32_t key_max;      // largest valid internal key (= key_range)
   BatchCtl *ctl;         // the handle's per-batch control block
   uint32_t *dirty;       // set when a batch mutated the structure (-> upper-level rebuild)
+  uint32_t *freelist;    // 2 x cap_bottom: reclaimed level-0 chunks (double-buffered)
+  uint32_t *fl;          // [0] free chunks in the current list, [1] taken, [2] buffer,
+                         // [3..5] reclaim scratch
 };
 
 // Per-batch control block (device memory, zeroed before every batch).

@@ -30,11 +30,51 @@ struct RebuildBufs {
   uint32_t *order_key;    // [cap_bottom] min keys in key order
   uint32_t *order_chunk;  // [cap_bottom] their chunks
   uint32_t *n1;           // [4]          marked chunks; old upper bump; dirty; active
+  void *levels;           // RbLevels computed once per rebuild (scan_top kernel)
   uint32_t words, blocks;
   uint32_t fill;          // F: entries per rebuilt upper chunk
 };
 
 constexpr int RB_BLOCK_WORDS = 1024;
+
+// level geometry from n1 (identical in every thread)
+struct RbLevels {
+  uint32_t m[MAX_N];     // chunks of level l (l >= 1)
+  uint32_t base[MAX_N];  // index of chunk 1 of level l (chunk 0 is the head chunk l-1)
+  uint64_t pw[MAX_N];    // F^(l-1)
+  int top;               // highest rebuilt level (its m == 1)
+};
+
+template <int N>
+__device__ __forceinline__ void rb_levels(uint32_t n1, uint32_t F, RbLevels &L) {
+  uint32_t len = n1 + 1;  // |A_1| including -inf
+  uint32_t base = N - 1;
+  uint64_t pw = 1;
+  L.top = N - 1;
+  for (int l = 1; l < N; ++l) {
+    L.m[l] = (len + F - 1) / F;
+    L.base[l] = base;
+    L.pw[l] = pw;
+    base += L.m[l] - 1;
+    if (L.m[l] == 1) {
+      L.top = l;
+      for (int q = l + 1; q < N; ++q) {
+        L.m[q] = 1;
+        L.base[q] = base;
+        L.pw[q] = pw * F;
+      }
+      break;
+    }
+    len = L.m[l];
+    pw *= F;
+  }
+}
+
+template <int N>
+__device__ __forceinline__ uint32_t rb_chunk(const RbLevels &L, int l, uint32_t j) {
+  return j == 0 ? (uint32_t)(l - 1) : L.base[l] + j - 1;
+}
+
 
 __device__ __forceinline__ bool rb_candidate(const DevState &d, uint32_t c, int N, uint32_t &minkey) {
   const uint64_t *ch = d.pool + (size_t)c * N;
@@ -97,7 +137,8 @@ __global__ void __launch_bounds__(1024) rebuild_scan_kernel(RebuildBufs b) {
   if (w < b.words) b.word_prefix[w] = warp_tot[warp] + incl - v;
 }
 
-// (3) exclusive scan of the block sums (one block)
+// (3) exclusive scan of the block sums (one block); n1 = the total; the level geometry
+template <int N>
 __global__ void __launch_bounds__(1024) rebuild_scan_top_kernel(RebuildBufs b) {
   pdl_wait();
   if (!rb_active(b)) return;
@@ -130,7 +171,10 @@ __global__ void __launch_bounds__(1024) rebuild_scan_top_kernel(RebuildBufs b) {
     if (threadIdx.x == 1023) carry += warp_tot[warp] + incl;
     __syncthreads();
   }
-  if (threadIdx.x == 0) b.n1[0] = carry;  // marked chunks = total popcount
+  if (threadIdx.x == 0) {
+    b.n1[0] = carry;  // marked chunks = total popcount
+    rb_levels<N>(carry, b.fill, *(RbLevels *)b.levels);
+  }
 }
 
 // (4) each marked chunk writes itself at its rank
@@ -151,44 +195,6 @@ __global__ void __launch_bounds__(256) rebuild_rank_kernel(const __grid_constant
   }
 }
 
-// level geometry from n1 (identical in every thread)
-struct RbLevels {
-  uint32_t m[MAX_N];     // chunks of level l (l >= 1)
-  uint32_t base[MAX_N];  // index of chunk 1 of level l (chunk 0 is the head chunk l-1)
-  uint64_t pw[MAX_N];    // F^(l-1)
-  int top;               // highest rebuilt level (its m == 1)
-};
-
-template <int N>
-__device__ __forceinline__ void rb_levels(uint32_t n1, uint32_t F, RbLevels &L) {
-  uint32_t len = n1 + 1;  // |A_1| including -inf
-  uint32_t base = N - 1;
-  uint64_t pw = 1;
-  L.top = N - 1;
-  for (int l = 1; l < N; ++l) {
-    L.m[l] = (len + F - 1) / F;
-    L.base[l] = base;
-    L.pw[l] = pw;
-    base += L.m[l] - 1;
-    if (L.m[l] == 1) {
-      L.top = l;
-      for (int q = l + 1; q < N; ++q) {
-        L.m[q] = 1;
-        L.base[q] = base;
-        L.pw[q] = pw * F;
-      }
-      break;
-    }
-    len = L.m[l];
-    pw *= F;
-  }
-}
-
-template <int N>
-__device__ __forceinline__ uint32_t rb_chunk(const RbLevels &L, int l, uint32_t j) {
-  return j == 0 ? (uint32_t)(l - 1) : L.base[l] + j - 1;
-}
-
 // (5) write every chunk of levels >= 1; one warp per chunk, lane e writes entry e
 template <int N>
 __global__ void __launch_bounds__(256) rebuild_pack_kernel(const __grid_constant__ DevState d, RebuildBufs b) {
@@ -196,8 +202,9 @@ __global__ void __launch_bounds__(256) rebuild_pack_kernel(const __grid_constant
   if (!rb_active(b)) return;
   const uint32_t n1 = b.n1[0];
   const uint32_t F = b.fill;
-  RbLevels L;
-  rb_levels<N>(n1, F, L);
+  __shared__ RbLevels L;
+  if (threadIdx.x == 0) L = *(const RbLevels *)b.levels;
+  __syncthreads();
   uint32_t total = 0;
   for (int l = 1; l < N; ++l) total += L.m[l];
   const uint32_t head0 = d.head[0];
@@ -246,24 +253,144 @@ __global__ void __launch_bounds__(256) rebuild_pack_kernel(const __grid_constant
   if (blockIdx.x == 0 && threadIdx.x == 0) d.bump[1] = L.base[N - 1] + (L.top == N - 1 ? L.m[N - 1] - 1 : 0);
 }
 
-// (6) clear the bitmap marks; return the upper chunks past the new bump to the allocated
-// state; reset the counters for the next rebuild
+// ---- R25: reclaim the zombie level-0 chunks into the free list -------------------------
+// Right after a rebuild nothing points at a zombie any more: upkeep (R23) unlinked them
+// from level 0 and the rebuilt upper levels only point at live chunks.  So every zombie is
+// reset to the allocated state of P:237 and appended, in ascending chunk order, after the
+// still-unused part of the previous free list (reclamation between launches).
+constexpr int RC_TILE = 1024;  // chunks per tile: 256 threads x 4
+
+// (6+7) clear the bitmap marks, return the upper chunks past the new bump to the
+// allocated state, and count the zombies per tile
 template <int N>
-__global__ void __launch_bounds__(256) rebuild_clear_kernel(const __grid_constant__ DevState d, RebuildBufs b) {
+__global__ void __launch_bounds__(256) reclaim_count_kernel(const __grid_constant__ DevState d, RebuildBufs b,
+                                                            uint32_t *tile_cnt) {
   pdl_wait();
   if (!rb_active(b)) return;
-  const uint32_t n1 = b.n1[0];
-  const uint32_t old_used = b.n1[1];
-  const uint32_t new_used = d.bump[1];
-  const uint32_t stride = gridDim.x * blockDim.x;
-  const uint32_t tid = blockIdx.x * blockDim.x + threadIdx.x;
-  for (uint32_t i = tid; i < n1; i += stride) b.bitmap[b.order_key[i] >> 5] = 0u;
-  if (old_used > new_used) {
-    const uint64_t first = (uint64_t)new_used * N, lastx = (uint64_t)old_used * N;
-    for (uint64_t e = first + tid; e < lastx; e += stride)
-      d.pool[e] = ((e % N) == (uint64_t)(N - 1)) ? (uint64_t)LOCK_HELD : EMPTY_ENTRY;
+  {
+    const uint32_t n1 = b.n1[0];
+    const uint32_t old_used = b.n1[1];
+    const uint32_t new_used = d.bump[1];
+    const uint32_t stride = gridDim.x * blockDim.x;
+    const uint32_t tid = blockIdx.x * blockDim.x + threadIdx.x;
+    for (uint32_t i = tid; i < n1; i += stride) b.bitmap[b.order_key[i] >> 5] = 0u;
+    if (old_used > new_used) {
+      const uint64_t first = (uint64_t)new_used * N, lastx = (uint64_t)old_used * N;
+      for (uint64_t e = first + tid; e < lastx; e += stride)
+        d.pool[e] = ((e % N) == (uint64_t)(N - 1)) ? (uint64_t)LOCK_HELD : EMPTY_ENTRY;
+    }
+  }
+  const uint32_t used = min(d.bump[0], d.cap_bottom);
+  const uint32_t tiles = (used + RC_TILE - 1) / RC_TILE;
+  __shared__ uint32_t wsum[8];
+  for (uint32_t tile = blockIdx.x; tile < tiles; tile += gridDim.x) {
+    uint32_t cnt = 0;
+    for (int q = 0; q < 4; ++q) {
+      const uint32_t i = tile * RC_TILE + threadIdx.x * 4 + q;
+      if (i < used && lo32(d.pool[(size_t)(d.cap_upper + i) * N + N - 1]) == LOCK_ZOMBIE) ++cnt;
+    }
+    for (int o = 16; o; o >>= 1) cnt += __shfl_xor_sync(0xFFFFFFFFu, cnt, o);
+    if ((threadIdx.x & 31) == 0) wsum[threadIdx.x >> 5] = cnt;
+    __syncthreads();
+    if (threadIdx.x == 0) {
+      uint32_t t = 0;
+      for (int w = 0; w < 8; ++w) t += wsum[w];
+      tile_cnt[tile] = t;
+    }
+    __syncthreads();
   }
 }
 
+// (8) exclusive scan of the tile counts; the new list = old remainder + zombies
+__global__ void __launch_bounds__(1024) reclaim_scan_kernel(const __grid_constant__ DevState d, RebuildBufs b,
+                                                            uint32_t *tile_cnt) {
+  pdl_wait();
+  if (!rb_active(b)) return;
+  const uint32_t used = min(d.bump[0], d.cap_bottom);
+  const uint32_t tiles = (used + RC_TILE - 1) / RC_TILE;
+  __shared__ uint32_t carry, warp_tot[32];
+  if (threadIdx.x == 0) carry = 0;
+  __syncthreads();
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  for (uint32_t base = 0; base < tiles; base += 1024) {
+    const uint32_t i = base + threadIdx.x;
+    const uint32_t v = i < tiles ? tile_cnt[i] : 0u;
+    uint32_t incl = v;
+    for (int o = 1; o < 32; o <<= 1) {
+      const uint32_t y = __shfl_up_sync(0xFFFFFFFFu, incl, o);
+      if (lane >= o) incl += y;
+    }
+    if (lane == 31) warp_tot[warp] = incl;
+    __syncthreads();
+    if (warp == 0) {
+      uint32_t t = warp_tot[lane], ti = t;
+      for (int o = 1; o < 32; o <<= 1) {
+        const uint32_t y = __shfl_up_sync(0xFFFFFFFFu, ti, o);
+        if (lane >= o) ti += y;
+      }
+      warp_tot[lane] = ti - t;
+    }
+    __syncthreads();
+    if (i < tiles) tile_cnt[i] = carry + warp_tot[warp] + incl - v;
+    __syncthreads();
+    if (threadIdx.x == 1023) carry += warp_tot[warp] + incl;
+    __syncthreads();
+  }
+  if (threadIdx.x == 0) {
+    const uint32_t count = d.fl[0], taken = d.fl[1], sel = d.fl[2];
+    const uint32_t rem = taken < count ? count - taken : 0u;
+    d.fl[3] = rem;
+    d.fl[4] = sel;
+    d.fl[5] = taken;
+    d.fl[0] = rem + carry;
+    d.fl[1] = 0;
+    d.fl[2] = sel ^ 1u;
+  }
+}
+
+// (9) write the new list (old remainder first, then the zombies in chunk order) and reset
+// the zombies to the allocated state
+template <int N>
+__global__ void __launch_bounds__(256) reclaim_write_kernel(const __grid_constant__ DevState d, RebuildBufs b,
+                                                            const uint32_t *tile_off) {
+  pdl_wait();
+  if (!rb_active(b)) return;
+  const uint32_t rem = d.fl[3], oldsel = d.fl[4], taken = d.fl[5];
+  const uint32_t *oldl = d.freelist + (size_t)oldsel * d.cap_bottom;
+  uint32_t *newl = d.freelist + (size_t)(oldsel ^ 1u) * d.cap_bottom;
+  for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < rem; i += gridDim.x * blockDim.x)
+    newl[i] = oldl[taken + i];
+  const uint32_t used = min(d.bump[0], d.cap_bottom);
+  const uint32_t tiles = (used + RC_TILE - 1) / RC_TILE;
+  __shared__ uint32_t wsum[8];
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  for (uint32_t tile = blockIdx.x; tile < tiles; tile += gridDim.x) {
+    bool z[4];
+    uint32_t cnt = 0;
+    for (int q = 0; q < 4; ++q) {
+      const uint32_t i = tile * RC_TILE + threadIdx.x * 4 + q;
+      z[q] = i < used && lo32(d.pool[(size_t)(d.cap_upper + i) * N + N - 1]) == LOCK_ZOMBIE;
+      cnt += z[q];
+    }
+    uint32_t incl = cnt;
+    for (int o = 1; o < 32; o <<= 1) {
+      const uint32_t y = __shfl_up_sync(0xFFFFFFFFu, incl, o);
+      if (lane >= o) incl += y;
+    }
+    if (lane == 31) wsum[warp] = incl;
+    __syncthreads();
+    uint32_t pos = rem + tile_off[tile] + incl - cnt;
+    for (int w = 0; w < warp; ++w) pos += wsum[w];
+    for (int q = 0; q < 4; ++q) {
+      if (!z[q]) continue;
+      const uint32_t c = d.cap_upper + tile * RC_TILE + threadIdx.x * 4 + q;
+      newl[pos++] = c;
+      uint64_t *ch = d.pool + (size_t)c * N;
+      for (int e = 0; e < N - 1; ++e) ch[e] = EMPTY_ENTRY;
+      ch[N - 1] = (uint64_t)LOCK_HELD;
+    }
+    __syncthreads();
+  }
+}
 
 }  // namespace gfsl_dev

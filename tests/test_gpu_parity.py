@@ -176,3 +176,19 @@ def test_batch_host_matches_device_path():
     _, k1, v1 = g1.validate()
     _, k2, v2 = g2.validate()
     assert np.array_equal(k1, k2) and np.array_equal(v1, v2)
+
+
+def test_long_churn_reclaims_and_stays_exact():
+    """Concurrent 50/50 churn for many batches with rebuild + reclamation every batch:
+    results stay bit-exact and the level-0 pool stops growing."""
+    R = 20_000
+    g = GFSL(R, rebuild_every=1)
+    o = OracleMap(R)
+    prefill(g, o, R, R // 2)
+    used = []
+    for i, (op, key, val) in enumerate(workload_batches(R, 4_000, 60, (50, 50, 0))):
+        run_batch(g, o, op, key, val)
+        if i % 10 == 9:
+            rep = check_same_set(g, o)
+            used.append(rep.pool_used[0])
+    assert used[-1] <= used[1] * 1.02 + 8

@@ -141,3 +141,24 @@ def test_model_with_rebuild_matches_oracle_a(N, every):
             l0 = [c for c in m.level_chain(0) if not m.zombie(c)][1:]
             targets = {V(e) for c in m.level_chain(1) for e in m.pool[c][: m.DSIZE] if K(e) != INF}
             assert all(c in targets for c in l0 if m.keys(c)[0] != INF)
+
+
+def test_reclaimed_chunks_bound_the_pool():
+    """R25: with zombies recycled after each rebuild, sustained 50/50 churn stops growing
+    the level-0 pool; without reclamation (no rebuild) every merge leaks a chunk."""
+    R, N = 600, 16
+    o = OracleMap(R)
+    runs = {}
+    for every in (1, 0):
+        m = GFSLModel(N, R, cap_bottom=20000, cap_upper=4000, rebuild_every=every)
+        w = Workload(R, 200, mix=(50, 50, 0), seed=SEED_BASE + 99)
+        used = []
+        for b in range(120):
+            op, key, val, _ = w.make_batch(b)
+            m.batch(op.numpy().tolist(), key.numpy().astype(np.uint32).tolist(),
+                    val.numpy().astype(np.uint32).tolist())
+            used.append(m.bump[0])
+        assert m.check_invariants() == []
+        runs[every] = used
+    assert runs[1][-1] == runs[1][60]          # plateau with reclamation
+    assert runs[0][-1] > runs[0][60] + 20      # keeps leaking without it
