@@ -192,3 +192,20 @@ def test_long_churn_reclaims_and_stays_exact():
             rep = check_same_set(g, o)
             used.append(rep.pool_used[0])
     assert used[-1] <= used[1] * 1.02 + 8
+
+
+def test_pool_exhaustion_is_sticky():
+    """Inserting far more keys than `capacity` sizes the pool for exhausts it: the next
+    call reports GFSL_EPOOL, and so does every later one (the structure is undefined)."""
+    from paper_conf_ppopp_moscovicicp17_b200.gfsl import GFSLError, GFSL_EPOOL
+    R = 100_000
+    g = GFSL(R, capacity=100)
+    keys = np.random.default_rng(3).permutation(R)[:20_000].astype(np.uint32)
+    with pytest.raises(GFSLError) as ei:
+        for s in range(0, keys.size, 2_000):
+            k = keys[s:s + 2_000]
+            g.batch(*to_dev(np.ones(k.size, np.uint8), k, k))
+            torch.cuda.synchronize()
+    assert ei.value.status == GFSL_EPOOL
+    with pytest.raises(GFSLError):
+        g.batch(*to_dev(np.zeros(1, np.uint8), np.zeros(1, np.uint32), None))
