@@ -51,6 +51,12 @@ CONFIGS = {
     "C4-32": (100_000_000, 100_000_000, 50_000_000, 10, (0, 0, 100), "uniform", 32),
     "C4-16": (100_000_000, 100_000_000, 50_000_000, 10, (0, 0, 100), "uniform", 16),
     "C5": (1_000_000_000, 500_000_000, 125_000_000, 8, (10, 10, 80), "uniform", 16),
+    # NEXT-4: the paper's other workloads (Fig 5.3 mixes, Fig 5.4b/c single-op runs)
+    "M1-1-98": (1_000_000, 500_000, 625_000, 16, (1, 1, 98), "uniform", 16),
+    "M5-5-90": (1_000_000, 500_000, 625_000, 16, (5, 5, 90), "uniform", 16),
+    "M20-20-60-10M": (10_000_000, 5_000_000, 625_000, 16, (20, 20, 60), "uniform", 16),
+    "INS-1M": (1_000_000, 0, 125_000, 8, (100, 0, 0), "uniform", 16),     # R inserts, empty start
+    "DEL-1M": (1_000_000, 1_000_000, 125_000, 8, (0, 100, 0), "uniform", 16),  # R deletes, full start
 }
 L2_FLUSH_BYTES = 256 << 20
 
