@@ -8,6 +8,7 @@
 #include <cuda_runtime.h>
 
 #include <algorithm>
+#include <cstddef>
 #include <cstdlib>
 #include <array>
 #include <cstdio>
@@ -49,7 +50,9 @@ struct gfsl {
   DevState d{};
   BatchCtl *ctl = nullptr;
   uint2 *list_c = nullptr, *list_u = nullptr;
-  uint32_t *plan_path = nullptr, *mut_list = nullptr;
+  uint32_t *plan_path = nullptr;
+  uint4 *mut_rec = nullptr;
+  uint32_t *mut_u = nullptr, *list_v = nullptr;
   uint8_t *plan_top = nullptr;
   uint64_t list_cap = 0;
   uint32_t *h_error = nullptr;  // mapped host memory, device alias in d.error
@@ -106,7 +109,8 @@ __global__ void init_heads_kernel(DevState d, uint32_t N) {
 __global__ void __launch_bounds__(256)
 classify_kernel(const uint8_t *__restrict__ ops, const uint32_t *__restrict__ keys,
                 uint8_t *__restrict__ res, uint32_t n, uint64_t key_range,
-                uint2 *__restrict__ list_c, uint2 *__restrict__ list_u, BatchCtl *ctl) {
+                uint2 *__restrict__ list_c, uint2 *__restrict__ list_u, BatchCtl *ctl,
+                const uint32_t *__restrict__ vals, uint32_t *__restrict__ list_v) {
   __shared__ uint32_t wc[8], wu[8], base_c, base_u;
   const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
   const uint32_t stride = gridDim.x * blockDim.x;
@@ -145,7 +149,11 @@ classify_kernel(const uint8_t *__restrict__ ops, const uint32_t *__restrict__ ke
     __syncthreads();
     const uint32_t below = (1u << lane) - 1u;
     if (isc) list_c[base_c + wc[warp] + __popc(bc & below)] = e;
-    if (isu) list_u[base_u + wu[warp] + __popc(bu & below)] = e;
+    if (isu) {
+      const uint32_t pos = base_u + wu[warp] + __popc(bu & below);
+      list_u[pos] = e;
+      list_v[pos] = vals ? vals[i] : 0u;
+    }
     __syncthreads();
   }
 }
@@ -154,7 +162,8 @@ classify_kernel(const uint8_t *__restrict__ ops, const uint32_t *__restrict__ ke
 __global__ void classify_ordered_kernel(const uint8_t *__restrict__ ops, const uint32_t *__restrict__ keys,
                                         uint8_t *__restrict__ res, uint32_t n, uint64_t key_range,
                                         uint2 *__restrict__ list_c, uint2 *__restrict__ list_u,
-                                        BatchCtl *ctl) {
+                                        BatchCtl *ctl, const uint32_t *__restrict__ vals,
+                                        uint32_t *__restrict__ list_v) {
   __shared__ uint32_t wc[8], wu[8];
   __shared__ uint32_t base_c, base_u;
   const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
@@ -185,7 +194,10 @@ __global__ void classify_ordered_kernel(const uint8_t *__restrict__ ops, const u
     }
     const uint32_t below = (1u << lane) - 1u;
     if (isc) list_c[oc + __popc(bc & below)] = e;
-    if (isu) list_u[ou + __popc(bu & below)] = e;
+    if (isu) {
+      list_u[ou + __popc(bu & below)] = e;
+      list_v[ou + __popc(bu & below)] = vals ? vals[i] : 0u;
+    }
     __syncthreads();
     if (threadIdx.x == 0) {
       for (int w = 0; w < (int)(blockDim.x >> 5); ++w) {
@@ -212,7 +224,7 @@ static void set_pdl(gfsl *h, cudaLaunchAttribute &a) {
   a.val.programmaticStreamSerializationAllowed = h->cfg.no_pdl ? 0 : 1;
 }
 
-static SearchOut search_out(gfsl *h) { return SearchOut{h->plan_path, h->plan_top, h->mut_list}; }
+static SearchOut search_out(gfsl *h) { return SearchOut{h->plan_path, h->plan_top, h->mut_rec, h->mut_u, h->list_v}; }
 
 // The upper levels live in one contiguous range (the upper pool, chunks [0, cap_upper)),
 // so the search kernel is launched with an L2 access-policy window that marks the used
@@ -400,7 +412,9 @@ static void free_all(gfsl *h) {
   cudaFree(h->list_u);
   cudaFree(h->plan_path);
   cudaFree(h->plan_top);
-  cudaFree(h->mut_list);
+  cudaFree(h->mut_rec);
+  cudaFree(h->mut_u);
+  cudaFree(h->list_v);
   cudaFree(h->st_op);
   cudaFree(h->st_res);
   cudaFree(h->st_key);
@@ -505,6 +519,10 @@ extern "C" gfsl_t gfsl_create_ex(uint64_t key_range, uint64_t capacity, const gf
     if ((e = cudaMalloc(&h->d.fl, 8 * 4)) != cudaSuccess) return fail("cudaMalloc(freelist)", e);
     if ((e = cudaMalloc(&h->rc_tiles, ((size_t)cap_b / RC_TILE + 2) * 4)) != cudaSuccess) return fail("cudaMalloc(reclaim)", e);
     cudaMemset(h->d.fl, 0, 8 * 4);
+#ifdef GFSL_DEBUG_TIMING
+    if ((e = cudaMalloc(&h->d.debug_times, ((size_t)148 * 64 * 15 + 64) * 8)) != cudaSuccess) return fail("cudaMalloc", e);
+    cudaMemset(h->d.debug_times, 0, ((size_t)148 * 64 * 15 + 64) * 8);
+#endif
   }
   cudaMemset(h->d.head, 0xFF, 32 * 4);
   cudaMemset(h->d.counter, 0, 32 * 4);
@@ -573,9 +591,14 @@ static gfsl_status ensure_lists(gfsl *h, uint64_t n) {
   cudaFree(h->list_u);
   cudaFree(h->plan_path);
   cudaFree(h->plan_top);
-  cudaFree(h->mut_list);
+  cudaFree(h->mut_rec);
+  cudaFree(h->mut_u);
+  cudaFree(h->list_v);
   h->list_c = h->list_u = nullptr;
-  h->plan_path = h->mut_list = nullptr;
+  h->plan_path = nullptr;
+  h->mut_rec = nullptr;
+  h->mut_u = nullptr;
+  h->list_v = nullptr;
   h->plan_top = nullptr;
   h->list_cap = 0;
   const uint64_t cap = std::max<uint64_t>(n, 1024);
@@ -583,7 +606,9 @@ static gfsl_status ensure_lists(gfsl *h, uint64_t n) {
   CK(cudaMalloc(&h->list_u, cap * 8));
   CK(cudaMalloc(&h->plan_path, cap * 4 * PLAN_LEVELS));
   CK(cudaMalloc(&h->plan_top, cap));
-  CK(cudaMalloc(&h->mut_list, cap * 4));
+  CK(cudaMalloc(&h->mut_rec, cap * 16));
+  CK(cudaMalloc(&h->mut_u, cap * 4));
+  CK(cudaMalloc(&h->list_v, cap * 4));
   h->list_cap = cap;
   return GFSL_OK;
 }
@@ -597,14 +622,14 @@ static gfsl_status enqueue_batch(gfsl *h, const uint8_t *ops, const uint32_t *ke
     for (auto &e : ev) CK(cudaEventCreate(&e));
     CK(cudaEventRecord(ev[0], s));
   }
-  CK(cudaMemsetAsync(h->ctl, 0, sizeof(BatchCtl), s));
+  CK(cudaMemsetAsync(h->ctl, 0, offsetof(BatchCtl, uq) + (size_t)std::min(h->update_grid, BatchCtl::UQ_MAX) * 32, s));
   if (h->cfg.serial_updates) {
     classify_ordered_kernel<<<1, 256, 0, s>>>(ops, keys, res, (uint32_t)n, h->key_range, h->list_c,
-                                              h->list_u, h->ctl);
+                                              h->list_u, h->ctl, vals, h->list_v);
   } else {
     const int cgrid = (int)std::min<uint64_t>((n + 255) / 256, (uint64_t)h->sms * 16);
     classify_kernel<<<std::max(cgrid, 1), 256, 0, s>>>(ops, keys, res, (uint32_t)n, h->key_range,
-                                                      h->list_c, h->list_u, h->ctl);
+                                                      h->list_c, h->list_u, h->ctl, vals, h->list_v);
   }
   if (prof) CK(cudaEventRecord(ev[1], s));
   bool ok = dispatch_contains(h, ops, keys, res, s);
@@ -694,6 +719,14 @@ extern "C" gfsl_status gfsl_batch_host(gfsl_t h, const uint8_t *op_types, const 
   CK(cudaStreamSynchronize(s));
   return sticky(h);
 }
+
+#ifdef GFSL_DEBUG_TIMING
+extern "C" gfsl_status gfsl_debug_times(gfsl_t h, unsigned long long *out, uint64_t n) {
+  CK(cudaDeviceSynchronize());
+  CK(cudaMemcpy(out, h->d.debug_times, std::min<uint64_t>(n, (uint64_t)148 * 64 * 15 + 64) * 8, cudaMemcpyDeviceToHost));
+  return GFSL_OK;
+}
+#endif
 
 extern "C" gfsl_status gfsl_get_stats(gfsl_t h, gfsl_stats *out) {
   if (!h || !out) return GFSL_EINVAL;

@@ -59,6 +59,7 @@ struct DevState {
   uint32_t *freelist;    // 2 x cap_bottom: reclaimed level-0 chunks (double-buffered)
   uint32_t *fl;          // [0] free chunks in the current list, [1] taken, [2] buffer,
                          // [3..5] reclaim scratch
+  unsigned long long *debug_times;  // GFSL_DEBUG_TIMING builds: per-team (start, end, ops)
 };
 
 // Per-batch control block (device memory, zeroed before every batch).
@@ -66,10 +67,15 @@ struct BatchCtl {
   uint32_t n_contains;   // Contains ops of the batch (classify)
   uint32_t n_updates;    // Insert/Delete ops of the batch (classify)
   uint32_t n_mut;        // update ops that mutate (search kernel)
-  uint32_t next_update;  // dynamic work counter of the update kernel
+  uint32_t unused0;
   uint32_t snap_height;  // height seen by the search kernel
   uint32_t n_merges;     // merges of this batch (update kernel) -> upkeep sweep
   uint32_t pad[2];
+  // dynamic work queues of the update kernel (one per update block, at most UQ_MAX):
+  // queue j of Q hands out the mutation slots j, j + Q, j + 2Q, ... in order; one counter
+  // per 32-byte sector
+  static constexpr int UQ_MAX = 2048;
+  uint32_t uq[UQ_MAX * 8];
 };
 
 __device__ __forceinline__ uint32_t lo32(uint64_t x) { return (uint32_t)x; }

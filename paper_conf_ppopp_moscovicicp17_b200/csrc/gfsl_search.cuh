@@ -49,7 +49,9 @@ constexpr uint32_t F_EQUAL = 0x80000000u;    // on the down pointer: the winning
 struct SearchOut {
   uint32_t *plan_path;  // [n_updates * PLAN_LEVELS]
   uint8_t *plan_top;    // [n_updates]: highest level holding k (0 = bottom only), 0xFF = no-op
-  uint32_t *mut_list;   // [n_updates]: update slots that mutate
+  uint4 *mut_rec;       // [n_updates]: the ops that mutate, {op word, key, path[0], top | value}
+  uint32_t *mut_u;      // [n_updates]: their update slots (-> plan_path)
+  uint32_t *list_v;     // [n_updates]: the value of update slot u (classify kernel)
 };
 
 template <int N, int TEAM, bool COUNT = false>
@@ -99,9 +101,13 @@ search_kernel(DevState d, uint8_t *__restrict__ res, const uint2 *__restrict__ l
     if (!lane_live || sl >= n) return make_uint2(0xFFFFFFFFu, 0u);
     return sl < nc ? list_c[sl] : list_u[sl - nc];
   };
+  auto load_val = [&](uint32_t sl) -> uint32_t {
+    return (lane_live && sl < n && sl >= nc && t == 0) ? so.list_v[sl - nc] : 0u;
+  };
   uint32_t slot = warp_global * TPW + team_in_warp;  // this team's current op slot
   uint2 cur_op = load_op(slot);
   uint2 nxt_op = load_op(slot + total_teams);
+  uint32_t cur_val = load_val(slot), nxt_val = load_val(slot + total_teams);
   bool active = lane_live && slot < n;
   uint32_t k = cur_op.y;
   uint32_t cur = start;
@@ -185,7 +191,12 @@ search_kernel(DevState d, uint8_t *__restrict__ res, const uint2 *__restrict__ l
             res[opi] = mut ? 1 : 0;
             so.plan_path[(size_t)u * PLAN_LEVELS] = here;  // path[0] = enclosing chunk
             so.plan_top[u] = mut ? (uint8_t)seen_top : (uint8_t)0xFF;
-            if (mut) so.mut_list[atomicAdd(&ctl->n_mut, 1u)] = u;
+            if (mut) {
+              const uint32_t m = atomicAdd(&ctl->n_mut, 1u);
+              // {op word, key, path[0], top (Delete) | value (Insert)}
+              so.mut_rec[m] = make_uint4(cur_op.x, k, here, (cur_op.x & DELETE_FLAG) ? seen_top : cur_val);
+              so.mut_u[m] = u;
+            }
           }
         }
         if (COUNT) ++nops;
@@ -193,8 +204,10 @@ search_kernel(DevState d, uint8_t *__restrict__ res, const uint2 *__restrict__ l
         slot += total_teams;
         active = slot < n;
         cur_op = nxt_op;
+        cur_val = nxt_val;
         k = cur_op.y;
         nxt_op = load_op(slot + total_teams);
+        nxt_val = load_val(slot + total_teams);
         cur = start;
         level = height;
         bt = bt_c = NULL_CHUNK;

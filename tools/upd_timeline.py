@@ -1,0 +1,37 @@
+"""Per-warp timeline of the dual-op update kernel (needs a library built with
+-DGFSL_DEBUG_TIMING in place of libgfsl.so).  python tools/upd_timeline.py [config]"""
+import ctypes, os, sys
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+import numpy as np
+import torch
+from bench import CONFIGS, make_inputs, prefill_gpu
+from paper_conf_ppopp_moscovicicp17_b200 import gfsl as G
+from paper_conf_ppopp_moscovicicp17_b200.workload import SEED_BASE, Workload
+
+cfg = sys.argv[1] if len(sys.argv) > 1 else "C2"
+R, pre, B, nb, mix, dist, N = CONFIGS[cfg]
+dev = torch.device("cuda")
+g = G.GFSL(R, capacity=R, chunk_entries=N)
+prefill_gpu(g, R, pre, dev)
+w = Workload(R, B, mix=mix, dist=dist, seed=SEED_BASE + 1)
+lib = G.load_library()
+n = 148 * 64 * 15 + 64
+buf = (ctypes.c_ulonglong * n)()
+for b in range(4):
+    g.batch(*make_inputs(w, b, dev)[:3])
+torch.cuda.synchronize()
+lib.gfsl_debug_times(ctypes.c_void_p(g.h), buf, ctypes.c_uint64(n))
+a = np.frombuffer(buf, dtype=np.uint64)[:148 * 64 * 15].reshape(-1, 15).astype(np.float64)
+a = a[a[:, 0] > 0]
+t0 = a[:, 0].min()
+st, en, it = (a[:, 0] - t0) / 1e3, (a[:, 1] - t0) / 1e3, a[:, 2]
+oc = a[:, 3:7].sum(0)
+ser = a[:, 7]
+print(f"{cfg}: warps={len(a)} iterations={it.sum():.0f} kernel span={en.max():.1f} us")
+print("outcomes done/defer/cont/full:", oc.astype(int).tolist())
+print("start pct 0/50/90/100:", np.percentile(st, [0, 50, 90, 100]).round(1))
+print("end   pct 0/50/90/99/100:", np.percentile(en, [0, 50, 90, 99, 100]).round(1))
+print("iterations/warp pct 0/50/100:", np.percentile(it, [0, 50, 100]))
+dur = (en - st) * 1e3 * 1.965
+print(f"serial-section share {ser.sum() / dur.sum():.2f}; cycles per iteration excl. serial {(dur.sum() - ser.sum()) / it.sum():.0f};"
+      f" serial cycles per cont/full op {ser.sum() / max(oc[2] + oc[3], 1):.0f}")
