@@ -50,6 +50,10 @@ typedef enum gfsl_status {
 #define GFSL_REBUILD_DEFAULT_PERIOD 2u
 #define GFSL_REBUILD_NEVER 0xFFFFFFFFu
 
+/* Largest batch (ops per gfsl_batch call): the op index shares a 32-bit word with three
+ * flag bits on the device.  Larger batches are split by the caller. */
+#define GFSL_MAX_BATCH ((1u << 29) - 1u)
+
 /* Op codes (the "operation type" of the op array). */
 enum { GFSL_CONTAINS = 0, GFSL_INSERT = 1, GFSL_DELETE = 2 };
 /* Per-op result codes. */
@@ -110,6 +114,7 @@ void gfsl_destroy(gfsl_t h);
  * All arrays belong to the caller, must be on the handle's device, and must stay valid
  * until `stream` reaches the end of the batch.  Batches on one handle are serialized in
  * issue order (the handle makes each batch wait for the previous one).
+ * n <= GFSL_MAX_BATCH.
  * Returns GFSL_EINVAL for bad host arguments, or a sticky error (GFSL_EPOOL, GFSL_ECUDA)
  * raised by an earlier batch; on error nothing is enqueued.
  */

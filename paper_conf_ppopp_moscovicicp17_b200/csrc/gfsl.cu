@@ -1,7 +1,8 @@
 // gfsl.cu -- libgfsl: the C ABI of include/gfsl.h over the sm_100a kernels.
 //
 // A batch is enqueued as (DESIGN.md §Batch pipeline):
-//   memset(ctl) -> classify (a2) -> contains_kernel (B1, a3) -> update_kernel (B2, a4/a5)
+//   memset(ctl) -> search_kernel (intake + B1, a2/a3) -> update_kernel (B2, a4/a5)
+//   -> upkeep (-> rebuild every `rebuild_every` batches)
 // with no host synchronization.  The library owns the chunk pool, the head
 // array and per-level counters, the bump counters and the sticky error word; the
 // caller owns the op / key / value / result arrays.
@@ -49,11 +50,8 @@ struct gfsl {
   uint64_t key_range = 0;
   DevState d{};
   BatchCtl *ctl = nullptr;
-  uint2 *list_c = nullptr, *list_u = nullptr;
-  uint32_t *plan_path = nullptr;
+  uint32_t *plan_path = nullptr, *mut_of = nullptr;
   uint4 *mut_rec = nullptr;
-  uint32_t *mut_u = nullptr, *list_v = nullptr;
-  uint8_t *plan_top = nullptr;
   uint64_t list_cap = 0;
   uint32_t *h_error = nullptr;  // mapped host memory, device alias in d.error
   cudaEvent_t last = nullptr;
@@ -73,7 +71,7 @@ struct gfsl {
 };
 
 // ------------------------------------------------------------------------------------
-// kernels: pool init and classify (a2)
+// kernels: pool init
 
 // Every pool chunk starts in the "allocated" state of P:237: all entries +inf, max +inf,
 // locked.  Allocation is then only a bump of the counter.
@@ -103,116 +101,6 @@ __global__ void init_heads_kernel(DevState d, uint32_t N) {
   }
 }
 
-// Batch intake: range/op-code check (invalid -> 0xFF, no effect) and the split into the
-// Contains list and the Insert/Delete list.  Appends are aggregated per block (one global
-// atomic per list per 256-op tile) so the two list counters do not serialize at L2.
-__global__ void __launch_bounds__(256)
-classify_kernel(const uint8_t *__restrict__ ops, const uint32_t *__restrict__ keys,
-                uint8_t *__restrict__ res, uint32_t n, uint64_t key_range,
-                uint2 *__restrict__ list_c, uint2 *__restrict__ list_u, BatchCtl *ctl,
-                const uint32_t *__restrict__ vals, uint32_t *__restrict__ list_v) {
-  __shared__ uint32_t wc[8], wu[8], base_c, base_u;
-  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-  const uint32_t stride = gridDim.x * blockDim.x;
-  for (uint32_t base = blockIdx.x * blockDim.x; base < n; base += stride) {
-    const uint32_t i = base + threadIdx.x;
-    bool isc = false, isu = false;
-    uint2 e = make_uint2(0, 0);
-    if (i < n) {
-      const uint8_t op = ops[i];
-      const uint32_t k = keys[i];
-      const bool valid = op <= 2 && (uint64_t)k < key_range;
-      if (!valid) res[i] = 0xFF;
-      isc = valid && op == 0;
-      isu = valid && op != 0;
-      e = make_uint2(i | (op == 2 ? DELETE_FLAG : 0u), k + 1u);  // internal key (R3)
-    }
-    const uint32_t bc = __ballot_sync(0xFFFFFFFFu, isc);
-    const uint32_t bu = __ballot_sync(0xFFFFFFFFu, isu);
-    if (lane == 0) {
-      wc[warp] = __popc(bc);
-      wu[warp] = __popc(bu);
-    }
-    __syncthreads();
-    if (threadIdx.x == 0) {
-      uint32_t tc = 0, tu = 0;
-      for (int w = 0; w < 8; ++w) {
-        const uint32_t c = wc[w], u = wu[w];
-        wc[w] = tc;
-        wu[w] = tu;
-        tc += c;
-        tu += u;
-      }
-      base_c = tc ? atomicAdd(&ctl->n_contains, tc) : 0;
-      base_u = tu ? atomicAdd(&ctl->n_updates, tu) : 0;
-    }
-    __syncthreads();
-    const uint32_t below = (1u << lane) - 1u;
-    if (isc) list_c[base_c + wc[warp] + __popc(bc & below)] = e;
-    if (isu) {
-      const uint32_t pos = base_u + wu[warp] + __popc(bu & below);
-      list_u[pos] = e;
-      list_v[pos] = vals ? vals[i] : 0u;
-    }
-    __syncthreads();
-  }
-}
-
-// Serial (test) mode: the same split, in op-index order (one block, tile by tile).
-__global__ void classify_ordered_kernel(const uint8_t *__restrict__ ops, const uint32_t *__restrict__ keys,
-                                        uint8_t *__restrict__ res, uint32_t n, uint64_t key_range,
-                                        uint2 *__restrict__ list_c, uint2 *__restrict__ list_u,
-                                        BatchCtl *ctl, const uint32_t *__restrict__ vals,
-                                        uint32_t *__restrict__ list_v) {
-  __shared__ uint32_t wc[8], wu[8];
-  __shared__ uint32_t base_c, base_u;
-  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-  if (threadIdx.x == 0) base_c = base_u = 0;
-  __syncthreads();
-  for (uint32_t base = 0; base < n; base += blockDim.x) {
-    const uint32_t i = base + threadIdx.x;
-    bool isc = false, isu = false;
-    uint2 e = make_uint2(0, 0);
-    if (i < n) {
-      const uint8_t op = ops[i];
-      const bool valid = op <= 2 && (uint64_t)keys[i] < key_range;
-      if (!valid) res[i] = 0xFF;
-      isc = valid && op == 0;
-      isu = valid && op != 0;
-      e = make_uint2(i | (op == 2 ? DELETE_FLAG : 0u), keys[i] + 1u);
-    }
-    const uint32_t bc = __ballot_sync(0xFFFFFFFFu, isc), bu = __ballot_sync(0xFFFFFFFFu, isu);
-    if (lane == 0) {
-      wc[warp] = __popc(bc);
-      wu[warp] = __popc(bu);
-    }
-    __syncthreads();
-    uint32_t oc = base_c, ou = base_u;
-    for (int w = 0; w < warp; ++w) {
-      oc += wc[w];
-      ou += wu[w];
-    }
-    const uint32_t below = (1u << lane) - 1u;
-    if (isc) list_c[oc + __popc(bc & below)] = e;
-    if (isu) {
-      list_u[ou + __popc(bu & below)] = e;
-      list_v[ou + __popc(bu & below)] = vals ? vals[i] : 0u;
-    }
-    __syncthreads();
-    if (threadIdx.x == 0) {
-      for (int w = 0; w < (int)(blockDim.x >> 5); ++w) {
-        base_c += wc[w];
-        base_u += wu[w];
-      }
-    }
-    __syncthreads();
-  }
-  if (threadIdx.x == 0) {
-    ctl->n_contains = base_c;
-    ctl->n_updates = base_u;
-  }
-}
-
 // ------------------------------------------------------------------------------------
 // template dispatch
 
@@ -224,7 +112,9 @@ static void set_pdl(gfsl *h, cudaLaunchAttribute &a) {
   a.val.programmaticStreamSerializationAllowed = h->cfg.no_pdl ? 0 : 1;
 }
 
-static SearchOut search_out(gfsl *h) { return SearchOut{h->plan_path, h->plan_top, h->mut_rec, h->mut_u, h->list_v}; }
+static SearchOut search_out(gfsl *h) {
+  return SearchOut{h->mut_rec, h->plan_path, h->cfg.serial_updates ? h->mut_of : nullptr};
+}
 
 // The upper levels live in one contiguous range (the upper pool, chunks [0, cap_upper)),
 // so the search kernel is launched with an L2 access-policy window that marks the used
@@ -242,10 +132,7 @@ static void fill_window(gfsl *h, cudaLaunchAttribute &a) {
 }
 
 template <int N, int TEAM>
-static void launch_contains(gfsl *h, const uint8_t *ops, const uint32_t *keys, uint8_t *res,
-                            cudaStream_t s) {
-  (void)ops;
-  (void)keys;
+static void launch_contains(gfsl *h, const BatchIn &in, cudaStream_t s) {
   cudaLaunchConfig_t lc{};
   lc.gridDim = dim3(h->contains_grid);
   lc.blockDim = dim3(256);
@@ -255,21 +142,18 @@ static void launch_contains(gfsl *h, const uint8_t *ops, const uint32_t *keys, u
   if (h->persist_max && h->window_max) fill_window(h, attr[lc.numAttrs++]);
   set_pdl(h, attr[lc.numAttrs++]);
   if (h->cfg.count_reads)
-    cudaLaunchKernelEx(&lc, search_kernel<N, TEAM, true>, h->d, res, (const uint2 *)h->list_c,
-                       (const uint2 *)h->list_u, h->ctl, search_out(h));
+    cudaLaunchKernelEx(&lc, search_kernel<N, TEAM, true>, h->d, in, h->ctl, search_out(h));
   else
-    cudaLaunchKernelEx(&lc, search_kernel<N, TEAM, false>, h->d, res, (const uint2 *)h->list_c,
-                       (const uint2 *)h->list_u, h->ctl, search_out(h));
+    cudaLaunchKernelEx(&lc, search_kernel<N, TEAM, false>, h->d, in, h->ctl, search_out(h));
 }
 
 #define GFSL_CONTAINS_CONFIGS(X) \
   X(32, 2) X(32, 4) X(32, 8) X(32, 16) X(32, 32) X(16, 1) X(16, 2) X(16, 4) X(16, 8) X(16, 16) \
   X(12, 12) X(6, 6)
 
-static bool dispatch_contains(gfsl *h, const uint8_t *ops, const uint32_t *keys, uint8_t *res,
-                              cudaStream_t s) {
+static bool dispatch_contains(gfsl *h, const BatchIn &in, cudaStream_t s) {
   switch (h->N * 100 + h->team) {
-#define X(n, t) case n * 100 + t: launch_contains<n, t>(h, ops, keys, res, s); return true;
+#define X(n, t) case n * 100 + t: launch_contains<n, t>(h, in, s); return true;
     GFSL_CONTAINS_CONFIGS(X)
 #undef X
   }
@@ -277,9 +161,7 @@ static bool dispatch_contains(gfsl *h, const uint8_t *ops, const uint32_t *keys,
 }
 
 template <int N>
-static void launch_update(gfsl *h, const uint8_t *ops, const uint32_t *keys, const uint32_t *vals,
-                          uint8_t *res, uint32_t n, cudaStream_t s, cudaEvent_t after_update) {
-  (void)n;
+static void launch_update(gfsl *h, const BatchIn &in, cudaStream_t s, cudaEvent_t after_update) {
   cudaLaunchConfig_t lc{};
   cudaLaunchAttribute attr[1];
   set_pdl(h, attr[0]);
@@ -289,8 +171,7 @@ static void launch_update(gfsl *h, const uint8_t *ops, const uint32_t *keys, con
   lc.blockDim = dim3(h->cfg.serial_updates ? 32 : 256);
   lc.gridDim = dim3(h->cfg.serial_updates ? 1 : h->update_grid);
   const int serial = h->cfg.serial_updates ? 1 : 0;
-  cudaLaunchKernelEx(&lc, update_kernel<N>, h->d, vals, res, (const uint2 *)h->list_u, h->ctl,
-                     search_out(h), serial);
+  cudaLaunchKernelEx(&lc, update_kernel<N>, h->d, in, h->ctl, search_out(h), serial);
   if (after_update) cudaEventRecord(after_update, s);
   lc.blockDim = dim3(256);
   lc.gridDim = dim3(h->sms * 4);
@@ -408,13 +289,9 @@ static void free_all(gfsl *h) {
   cudaFree(h->d.bump);
   cudaFree(h->d.stats);
   cudaFree(h->ctl);
-  cudaFree(h->list_c);
-  cudaFree(h->list_u);
   cudaFree(h->plan_path);
-  cudaFree(h->plan_top);
+  cudaFree(h->mut_of);
   cudaFree(h->mut_rec);
-  cudaFree(h->mut_u);
-  cudaFree(h->list_v);
   cudaFree(h->st_op);
   cudaFree(h->st_res);
   cudaFree(h->st_key);
@@ -520,8 +397,8 @@ extern "C" gfsl_t gfsl_create_ex(uint64_t key_range, uint64_t capacity, const gf
     if ((e = cudaMalloc(&h->rc_tiles, ((size_t)cap_b / RC_TILE + 2) * 4)) != cudaSuccess) return fail("cudaMalloc(reclaim)", e);
     cudaMemset(h->d.fl, 0, 8 * 4);
 #ifdef GFSL_DEBUG_TIMING
-    if ((e = cudaMalloc(&h->d.debug_times, ((size_t)148 * 64 * 15 + 64) * 8)) != cudaSuccess) return fail("cudaMalloc", e);
-    cudaMemset(h->d.debug_times, 0, ((size_t)148 * 64 * 15 + 64) * 8);
+    if ((e = cudaMalloc(&h->d.debug_times, ((size_t)148 * 64 * 48 + 64) * 8)) != cudaSuccess) return fail("cudaMalloc", e);
+    cudaMemset(h->d.debug_times, 0, ((size_t)148 * 64 * 48 + 64) * 8);
 #endif
   }
   cudaMemset(h->d.head, 0xFF, 32 * 4);
@@ -587,28 +464,17 @@ static gfsl_status sticky(gfsl *h) {
 static gfsl_status ensure_lists(gfsl *h, uint64_t n) {
   if (n <= h->list_cap) return GFSL_OK;
   cudaDeviceSynchronize();
-  cudaFree(h->list_c);
-  cudaFree(h->list_u);
   cudaFree(h->plan_path);
-  cudaFree(h->plan_top);
+  cudaFree(h->mut_of);
   cudaFree(h->mut_rec);
-  cudaFree(h->mut_u);
-  cudaFree(h->list_v);
-  h->list_c = h->list_u = nullptr;
   h->plan_path = nullptr;
+  h->mut_of = nullptr;
   h->mut_rec = nullptr;
-  h->mut_u = nullptr;
-  h->list_v = nullptr;
-  h->plan_top = nullptr;
   h->list_cap = 0;
   const uint64_t cap = std::max<uint64_t>(n, 1024);
-  CK(cudaMalloc(&h->list_c, cap * 8));
-  CK(cudaMalloc(&h->list_u, cap * 8));
   CK(cudaMalloc(&h->plan_path, cap * 4 * PLAN_LEVELS));
-  CK(cudaMalloc(&h->plan_top, cap));
+  CK(cudaMalloc(&h->mut_of, cap * 4));
   CK(cudaMalloc(&h->mut_rec, cap * 16));
-  CK(cudaMalloc(&h->mut_u, cap * 4));
-  CK(cudaMalloc(&h->list_v, cap * 4));
   h->list_cap = cap;
   return GFSL_OK;
 }
@@ -623,26 +489,19 @@ static gfsl_status enqueue_batch(gfsl *h, const uint8_t *ops, const uint32_t *ke
     CK(cudaEventRecord(ev[0], s));
   }
   CK(cudaMemsetAsync(h->ctl, 0, offsetof(BatchCtl, uq) + (size_t)std::min(h->update_grid, BatchCtl::UQ_MAX) * 32, s));
-  if (h->cfg.serial_updates) {
-    classify_ordered_kernel<<<1, 256, 0, s>>>(ops, keys, res, (uint32_t)n, h->key_range, h->list_c,
-                                              h->list_u, h->ctl, vals, h->list_v);
-  } else {
-    const int cgrid = (int)std::min<uint64_t>((n + 255) / 256, (uint64_t)h->sms * 16);
-    classify_kernel<<<std::max(cgrid, 1), 256, 0, s>>>(ops, keys, res, (uint32_t)n, h->key_range,
-                                                      h->list_c, h->list_u, h->ctl, vals, h->list_v);
-  }
   if (prof) CK(cudaEventRecord(ev[1], s));
-  bool ok = dispatch_contains(h, ops, keys, res, s);
+  const BatchIn in{ops, keys, vals, res, (uint32_t)n, h->key_range};
+  bool ok = dispatch_contains(h, in, s);
   if (prof) CK(cudaEventRecord(ev[2], s));
   if (!ok) {
     set_last_error("no contains kernel for this (N, team)");
     return GFSL_EINVAL;
   }
   switch (h->N) {
-    case 32: launch_update<32>(h, ops, keys, vals, res, (uint32_t)n, s, prof ? ev[3] : nullptr); break;
-    case 16: launch_update<16>(h, ops, keys, vals, res, (uint32_t)n, s, prof ? ev[3] : nullptr); break;
-    case 12: launch_update<12>(h, ops, keys, vals, res, (uint32_t)n, s, prof ? ev[3] : nullptr); break;
-    case 6: launch_update<6>(h, ops, keys, vals, res, (uint32_t)n, s, prof ? ev[3] : nullptr); break;
+    case 32: launch_update<32>(h, in, s, prof ? ev[3] : nullptr); break;
+    case 16: launch_update<16>(h, in, s, prof ? ev[3] : nullptr); break;
+    case 12: launch_update<12>(h, in, s, prof ? ev[3] : nullptr); break;
+    case 6: launch_update<6>(h, in, s, prof ? ev[3] : nullptr); break;
   }
   cudaError_t e = cudaGetLastError();
   if (e != cudaSuccess) {
@@ -671,7 +530,7 @@ extern "C" gfsl_status gfsl_batch(gfsl_t h, const uint8_t *op_types, const uint3
   gfsl_status st = sticky(h);
   if (st != GFSL_OK) return st;
   if (n == 0) return GFSL_OK;
-  if (!op_types || !keys || !results || n > 0xFFFFFFFFull) {
+  if (!op_types || !keys || !results || n > GFSL_MAX_BATCH) {
     set_last_error("bad batch arguments");
     return GFSL_EINVAL;
   }
@@ -689,7 +548,7 @@ extern "C" gfsl_status gfsl_batch_host(gfsl_t h, const uint8_t *op_types, const 
   gfsl_status st = sticky(h);
   if (st != GFSL_OK) return st;
   if (n == 0) return GFSL_OK;
-  if (!op_types || !keys || !results || n > 0xFFFFFFFFull) {
+  if (!op_types || !keys || !results || n > GFSL_MAX_BATCH) {
     set_last_error("bad batch arguments");
     return GFSL_EINVAL;
   }
@@ -723,7 +582,7 @@ extern "C" gfsl_status gfsl_batch_host(gfsl_t h, const uint8_t *op_types, const 
 #ifdef GFSL_DEBUG_TIMING
 extern "C" gfsl_status gfsl_debug_times(gfsl_t h, unsigned long long *out, uint64_t n) {
   CK(cudaDeviceSynchronize());
-  CK(cudaMemcpy(out, h->d.debug_times, std::min<uint64_t>(n, (uint64_t)148 * 64 * 15 + 64) * 8, cudaMemcpyDeviceToHost));
+  CK(cudaMemcpy(out, h->d.debug_times, std::min<uint64_t>(n, (uint64_t)148 * 64 * 48 + 64) * 8, cudaMemcpyDeviceToHost));
   return GFSL_OK;
 }
 #endif

@@ -64,8 +64,8 @@ struct DevState {
 
 // Per-batch control block (device memory, zeroed before every batch).
 struct BatchCtl {
-  uint32_t n_contains;   // Contains ops of the batch (classify)
-  uint32_t n_updates;    // Insert/Delete ops of the batch (classify)
+  uint32_t unused1;
+  uint32_t unused2;
   uint32_t n_mut;        // update ops that mutate (search kernel)
   uint32_t unused0;
   uint32_t snap_height;  // height seen by the search kernel

@@ -23,6 +23,9 @@
 // kernel (B2), which starts from the recorded path ("the enclosing chunk must
 // either be in the path or reachable from it").
 //
+// The kernel also does the batch intake: it reads the caller's op/key/value arrays
+// directly (op i is team slot i), so no separate classify pass or op lists exist.
+//
 // B200 design: a team is TEAM lanes (TEAM | 32, TEAM <= N); each lane
 // holds EPL = N/TEAM consecutive entries loaded with one vector load (8/16/32 B), so a
 // warp runs 32/TEAM independent traversals in lockstep (P:205 allows teams smaller than
@@ -37,27 +40,38 @@ namespace gfsl_dev {
 
 constexpr int PLAN_LEVELS = 16;  // path levels recorded per update op (height < 16)
 
-// Op lists built by the classify kernel: {op index | DELETE_FLAG if Delete, internal key}.
-constexpr uint32_t DELETE_FLAG = 0x80000000u;
-constexpr uint32_t OPI_MASK = 0x7FFFFFFFu;
+// Op word: {op index | flags}.  A batch holds at most OPI_MASK + 1 = 2^29 ops.
+constexpr uint32_t DELETE_FLAG = 0x80000000u;   // Delete
+constexpr uint32_t UPDATE_FLAG = 0x40000000u;   // Insert or Delete
+constexpr uint32_t INVALID_FLAG = 0x20000000u;  // bad op code or key: result 0xFF, no effect
+constexpr uint32_t OPI_MASK = 0x1FFFFFFFu;
 // Chunk indices are < 2^30, so a shuffled pointer carries two flag bits.
 constexpr uint32_t PTR_MASK = 0x3FFFFFFFu;
 constexpr uint32_t F_ZOMBIE = 0x80000000u;   // on the NEXT pointer: the chunk is a zombie
 constexpr uint32_t F_LATERAL = 0x40000000u;  // on the NEXT pointer: max < k
 constexpr uint32_t F_EQUAL = 0x80000000u;    // on the down pointer: the winning key == k
 
+// The batch's input arrays (caller-owned device memory, input order).
+struct BatchIn {
+  const uint8_t *ops;
+  const uint32_t *keys;
+  const uint32_t *vals;  // may be NULL (= 0)
+  uint8_t *res;
+  uint32_t n;
+  uint64_t key_range;
+};
+
+// The mutations a batch's search phase hands to the update phase, compact: mutation m
+// (in completion order) has its record and its path.
 struct SearchOut {
-  uint32_t *plan_path;  // [n_updates * PLAN_LEVELS]
-  uint8_t *plan_top;    // [n_updates]: highest level holding k (0 = bottom only), 0xFF = no-op
-  uint4 *mut_rec;       // [n_updates]: the ops that mutate, {op word, key, path[0], top | value}
-  uint32_t *mut_u;      // [n_updates]: their update slots (-> plan_path)
-  uint32_t *list_v;     // [n_updates]: the value of update slot u (classify kernel)
+  uint4 *mut_rec;       // [n]: {op index | DELETE_FLAG, internal key, path[0], top (Delete) | value (Insert)}
+  uint32_t *plan_path;  // [n * PLAN_LEVELS]: mutation m's path, lane l = chunk at level l
+  uint32_t *mut_of;     // [n] or NULL: op i -> its mutation index, 0xFFFFFFFF if none (serial mode)
 };
 
 template <int N, int TEAM, bool COUNT = false>
 __global__ void __launch_bounds__(256)
-search_kernel(DevState d, uint8_t *__restrict__ res, const uint2 *__restrict__ list_c,
-              const uint2 *__restrict__ list_u, BatchCtl *__restrict__ ctl, SearchOut so) {
+search_kernel(DevState d, const BatchIn in, BatchCtl *__restrict__ ctl, SearchOut so) {
   constexpr int EPL = N / TEAM;
   static_assert(EPL * TEAM == N, "TEAM must divide N");
   constexpr int TPW = 32 / TEAM;                    // teams per warp
@@ -68,6 +82,9 @@ search_kernel(DevState d, uint8_t *__restrict__ res, const uint2 *__restrict__ l
   constexpr uint32_t FULL = 0xFFFFFFFFu;
 
   __shared__ uint32_t s_start, s_height;
+  // the path of the team's current op (written by its lane 0 only), copied out compactly
+  // at the end if the op mutates (about 1 op in 10)
+  __shared__ __align__(16) uint32_t s_path[(256 / 32) * TPW][PLAN_LEVELS];
   const int lane = threadIdx.x & 31;
   pdl_wait();
   pdl_trigger();
@@ -85,8 +102,8 @@ search_kernel(DevState d, uint8_t *__restrict__ res, const uint2 *__restrict__ l
   __syncthreads();
   const uint32_t start = s_start;
   const int height = (int)s_height;
-  const uint32_t nc = ctl->n_contains;
-  const uint32_t n = nc + ctl->n_updates;
+  const uint32_t n = in.n;
+  uint8_t *__restrict__ res = in.res;
 
   const int team_in_warp = lane / TEAM;
   const int t = lane - team_in_warp * TEAM;          // tId
@@ -95,19 +112,38 @@ search_kernel(DevState d, uint8_t *__restrict__ res, const uint2 *__restrict__ l
   const uint32_t warp_global = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   const uint32_t total_teams = (gridDim.x * blockDim.x >> 5) * TPW;
   const int next_src = lane_live ? team_base + NEXT_LANE : lane;
+  uint32_t *const my_path = s_path[((threadIdx.x >> 5) * TPW + (lane_live ? team_in_warp : 0)) % ((256 / 32) * TPW)];
 
-  // op slot s: s < nc -> list_c[s]; else update op list_u[s - nc].  One op prefetched.
-  auto load_op = [&](uint32_t sl) -> uint2 {
-    if (!lane_live || sl >= n) return make_uint2(0xFFFFFFFFu, 0u);
-    return sl < nc ? list_c[sl] : list_u[sl - nc];
+  // Batch intake, fused: op slot i is input op i, read straight from the caller's arrays
+  // (range/op-code check; an invalid op is traversed as a Contains of key 0 and answered
+  // 0xFF).  Internal key = key + 1 (R3).  One op prefetched.
+  // The prefetched op stays raw (loaded, not yet looked at) until it becomes current, so
+  // its loads overlap the current traversal.
+  // An Insert's value is loaded when the op becomes current (it is needed only at its end).
+  struct RawOp {
+    uint32_t op, key;
   };
-  auto load_val = [&](uint32_t sl) -> uint32_t {
-    return (lane_live && sl < n && sl >= nc && t == 0) ? so.list_v[sl - nc] : 0u;
+  auto load_raw = [&](uint32_t i) -> RawOp {
+    RawOp r{3u, 0u};
+    if (lane_live && i < n) {
+      r.op = __ldg(in.ops + i);
+      r.key = __ldg(in.keys + i);
+    }
+    return r;
+  };
+  auto load_val = [&](uint32_t i, const RawOp &r) -> uint32_t {
+    return (t == 0 && in.vals && r.op == 1 && lane_live && i < n) ? __ldg(in.vals + i) : 0u;
+  };
+  auto decode = [&](uint32_t i, const RawOp &r) -> uint2 {
+    const bool valid = r.op <= 2 && (uint64_t)r.key < in.key_range;
+    const uint32_t fl = !valid ? INVALID_FLAG : (r.op == 2 ? (DELETE_FLAG | UPDATE_FLAG) : (r.op == 1 ? UPDATE_FLAG : 0u));
+    return make_uint2(i | fl, valid ? r.key + 1u : 1u);
   };
   uint32_t slot = warp_global * TPW + team_in_warp;  // this team's current op slot
-  uint2 cur_op = load_op(slot);
-  uint2 nxt_op = load_op(slot + total_teams);
-  uint32_t cur_val = load_val(slot), nxt_val = load_val(slot + total_teams);
+  RawOp raw = load_raw(slot);
+  uint2 cur_op = decode(slot, raw);
+  uint32_t cur_val = load_val(slot, raw);
+  RawOp nxt = load_raw(slot + total_teams);
   bool active = lane_live && slot < n;
   uint32_t k = cur_op.y;
   uint32_t cur = start;
@@ -163,10 +199,10 @@ search_kernel(DevState d, uint8_t *__restrict__ res, const uint2 *__restrict__ l
       const bool done = !lat && level == 0;                 // bottom enclosing chunk (Alg 4.4)
       const bool down = !lat && level > 0;                  // down step (l.19-23) / backtrack
       const bool restart = down && !tb && bt == NULL_CHUNK; // (l.25) impossible when quiescent
-      const bool upd = slot >= nc;
+      const bool upd = (cur_op.x & UPDATE_FLAG) != 0;
       const uint32_t here = cur;
       if (down && upd && t == 0 && level < PLAN_LEVELS)     // searchSlow's path (Alg 4.6 l.28-37)
-        so.plan_path[(size_t)(slot - nc) * PLAN_LEVELS + level] = tb ? cur : bt_c;
+        my_path[level] = tb ? cur : bt_c;
       if (down && tb && (dptr & F_EQUAL) && seen_top == 0) seen_top = level;
       const bool set_bt = lat && !(np & F_ZOMBIE) && level > 0;  // prevKv = currKv (l.16)
       const uint32_t next_cur = lat ? (np & PTR_MASK) : (tb ? (dptr & PTR_MASK) : bt);
@@ -182,32 +218,35 @@ search_kernel(DevState d, uint8_t *__restrict__ res, const uint2 *__restrict__ l
         const bool te = tb != 0;
         const uint32_t opi = cur_op.x & OPI_MASK;
         if (t == 0) {
+          uint32_t m = 0xFFFFFFFFu;
           if (!upd) {
-            res[opi] = te ? 1 : 0;
+            res[opi] = (cur_op.x & INVALID_FLAG) ? 0xFF : (te ? 1 : 0);
           } else {
             // Alg 4.5 l.3-4 / Alg 4.11 l.4-5 on the snapshot: exact under the contract
-            const uint32_t u = slot - nc;
             const bool mut = (cur_op.x & DELETE_FLAG) ? te : !te;
             res[opi] = mut ? 1 : 0;
-            so.plan_path[(size_t)u * PLAN_LEVELS] = here;  // path[0] = enclosing chunk
-            so.plan_top[u] = mut ? (uint8_t)seen_top : (uint8_t)0xFF;
             if (mut) {
-              const uint32_t m = atomicAdd(&ctl->n_mut, 1u);
-              // {op word, key, path[0], top (Delete) | value (Insert)}
-              so.mut_rec[m] = make_uint4(cur_op.x, k, here, (cur_op.x & DELETE_FLAG) ? seen_top : cur_val);
-              so.mut_u[m] = u;
+              m = atomicAdd(&ctl->n_mut, 1u);
+              // {op index | DELETE_FLAG, key, path[0], top (Delete) | value (Insert)}
+              const uint32_t w = opi | (cur_op.x & DELETE_FLAG);
+              so.mut_rec[m] = make_uint4(w, k, here, (cur_op.x & DELETE_FLAG) ? seen_top : cur_val);
+              my_path[0] = here;  // path[0] = the enclosing bottom chunk
+              const uint4 *src = reinterpret_cast<const uint4 *>(my_path);
+              uint4 *dst = reinterpret_cast<uint4 *>(so.plan_path + (size_t)m * PLAN_LEVELS);
+#pragma unroll
+              for (int q = 0; q < PLAN_LEVELS / 4; ++q) dst[q] = src[q];
             }
           }
+          if (so.mut_of) so.mut_of[opi] = m;
         }
         if (COUNT) ++nops;
         // next op of this team (prefetched one ahead)
         slot += total_teams;
         active = slot < n;
-        cur_op = nxt_op;
-        cur_val = nxt_val;
+        cur_op = decode(slot, nxt);
+        cur_val = load_val(slot, nxt);
         k = cur_op.y;
-        nxt_op = load_op(slot + total_teams);
-        nxt_val = load_val(slot + total_teams);
+        nxt = load_raw(slot + total_teams);
         cur = start;
         level = height;
         bt = bt_c = NULL_CHUNK;

@@ -15,14 +15,21 @@ g = G.GFSL(R, capacity=R, chunk_entries=N)
 prefill_gpu(g, R, pre, dev)
 w = Workload(R, B, mix=mix, dist=dist, seed=SEED_BASE + 1)
 lib = G.load_library()
-n = 148 * 64 * 15 + 64
+n = 148 * 64 * 48 + 64
 buf = (ctypes.c_ulonglong * n)()
+buf0 = (ctypes.c_ulonglong * n)()
 for b in range(4):
+    if b == 3:
+        torch.cuda.synchronize()
+        lib.gfsl_debug_times(ctypes.c_void_p(g.h), buf0, ctypes.c_uint64(n))
     g.batch(*make_inputs(w, b, dev)[:3])
 torch.cuda.synchronize()
 lib.gfsl_debug_times(ctypes.c_void_p(g.h), buf, ctypes.c_uint64(n))
-a = np.frombuffer(buf, dtype=np.uint64)[:148 * 64 * 15].reshape(-1, 15).astype(np.float64)
+
+a = np.frombuffer(buf, dtype=np.uint64)[:148 * 64 * 48].reshape(-1, 48).astype(np.float64)
 a = a[a[:, 0] > 0]
+cnt = np.zeros(100, np.int64)
+cnt[40:72] = a[:, 16:48].sum(0).astype(np.int64)
 t0 = a[:, 0].min()
 st, en, it = (a[:, 0] - t0) / 1e3, (a[:, 1] - t0) / 1e3, a[:, 2]
 oc = a[:, 3:7].sum(0)
@@ -35,3 +42,9 @@ print("iterations/warp pct 0/50/100:", np.percentile(it, [0, 50, 100]))
 dur = (en - st) * 1e3 * 1.965
 print(f"serial-section share {ser.sum() / dur.sum():.2f}; cycles per iteration excl. serial {(dur.sum() - ser.sum()) / it.sum():.0f};"
       f" serial cycles per cont/full op {ser.sum() / max(oc[2] + oc[3], 1):.0f}")
+for name, i in (("insert_locked: split_insert(0)", 40), ("  .. split_chunk(0)", 46), ("  .. update_down_ptrs(0)", 48),
+                ("  raise_levels", 42), ("  unlocks", 44), ("delete_upper: exact checks", 50), ("  upper levels", 52),
+                ("  bottom remove", 54), ("full ops", 58), ("cont delete", 60), ("cont insert", 62)):
+    c = cnt[i + 1]
+    print(f"  {name:34s} n={c:7d}  cycles/call {cnt[i] / max(c, 1):8.0f}")
+print("  merges:", cnt[56])
