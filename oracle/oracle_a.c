@@ -24,6 +24,12 @@
  * Invalid ops (op code > 2 or key >= key_range) get result 0xFF and no effect
  * (reading R5).
  *
+ * oa_batch_seq() is the combining semantics of SURVEY 8(f) NEXT-1 (R26), exact
+ * for ANY batch: every Contains is answered against M (as in S1); then the mutating ops
+ * are applied one by one in input order, each answered against the map as it is at that
+ * point.  Under the contract it equals oa_batch() (the mutations of distinct keys
+ * commute).
+ *
  * How: a sequential Pugh skiplist (levels of sorted linked lists, each a
  * random sublist of the one below, a node's height drawn with p = 1/2), MAX_LEVEL 32,
  * xorshift64 RNG.  This is the textbook structure of P:191, not GFSL: the two share
@@ -227,6 +233,30 @@ int oa_batch(oa_map *m, const uint8_t *op, const uint32_t *key, const uint32_t *
       if (oa_insert(m, key[i], val ? val[i] : 0) < 0) return OA_ENOMEM;
     } else {
       oa_erase(m, key[i]);
+    }
+  }
+  return OA_OK;
+}
+
+/*
+ * Combining batch (R26): pass 1 answers the Contains ops
+ * against the pre-batch map; pass 2 applies every valid Insert/Delete sequentially in
+ * input order, each result taken from the map at that moment.  No contract.
+ */
+int oa_batch_seq(oa_map *m, const uint8_t *op, const uint32_t *key, const uint32_t *val,
+                 uint8_t *res, uint64_t n, uint64_t key_range) {
+  for (uint64_t i = 0; i < n; i++) {
+    if (!oa_valid(op[i], key[i], key_range)) { res[i] = OA_INVALID; continue; }
+    if (op[i] == OA_CONTAINS) res[i] = oa_contains(m, key[i]) ? OA_TRUE : OA_FALSE;
+  }
+  for (uint64_t i = 0; i < n; i++) {
+    if (!oa_valid(op[i], key[i], key_range) || op[i] == OA_CONTAINS) continue;
+    if (op[i] == OA_INSERT) {
+      int r = oa_insert(m, key[i], val ? val[i] : 0);
+      if (r < 0) return OA_ENOMEM;
+      res[i] = r ? OA_TRUE : OA_FALSE;
+    } else {
+      res[i] = oa_erase(m, key[i]) ? OA_TRUE : OA_FALSE;
     }
   }
   return OA_OK;

@@ -53,6 +53,8 @@ def _load():
         lib.oa_export.argtypes = [vp, vp, vp, u64]
         lib.oa_batch.restype = ctypes.c_int
         lib.oa_batch.argtypes = [vp, vp, vp, vp, vp, u64, u64]
+        lib.oa_batch_seq.restype = ctypes.c_int
+        lib.oa_batch_seq.argtypes = [vp, vp, vp, vp, vp, u64, u64]
         _lib = lib
     return _lib
 
@@ -101,13 +103,16 @@ class OracleMap:
     def erase(self, k: int) -> bool:
         return bool(self.lib.oa_erase(self.h, k))
 
-    def batch(self, op: np.ndarray, key: np.ndarray, val: np.ndarray | None) -> np.ndarray:
+    def batch(self, op: np.ndarray, key: np.ndarray, val: np.ndarray | None,
+              combine: bool = False) -> np.ndarray:
+        """S1 batch (R1; contract enforced), or with combine=True the combining
+        semantics of R26 (Contains on the pre-batch map, mutations in input order)."""
         op = np.ascontiguousarray(op, dtype=np.uint8)
         key = np.ascontiguousarray(key, dtype=np.uint32)
         val = None if val is None else np.ascontiguousarray(val, dtype=np.uint32)
         res = np.empty(op.shape[0], dtype=np.uint8)
-        rc = self.lib.oa_batch(self.h, _ptr(op), _ptr(key), _ptr(val), _ptr(res),
-                               op.shape[0], self.key_range)
+        fn = self.lib.oa_batch_seq if combine else self.lib.oa_batch
+        rc = fn(self.h, _ptr(op), _ptr(key), _ptr(val), _ptr(res), op.shape[0], self.key_range)
         if rc == OA_ECONTRACT:
             raise ValueError("batch violates the <=1-mutating-op-per-key contract")
         if rc != OA_OK:

@@ -157,3 +157,73 @@ def test_paper_contains_examples():
     q = np.array(g["query"], np.uint32)
     r = o.batch(np.zeros(q.size, np.uint8), q, None)
     assert r.tolist() == g["expect"]
+
+
+# ---- combining semantics (R26) ----
+
+def brute_batch_seq(M: dict, op, key, val, R):
+    """Plain definition of R26 over a Python dict: Contains against the pre-batch map,
+    then every Insert/Delete one at a time in input order."""
+    pre = set(M)
+    res = []
+    for o, k in zip(op, key):
+        res.append(INVALID if (o > 2 or k >= R) else (int(k in pre) if o == 0 else None))
+    for i, (o, k, v) in enumerate(zip(op, key, val)):
+        if res[i] is not None:
+            continue
+        if o == 1:
+            res[i] = int(k not in M)
+            if k not in M:
+                M[k] = v
+        else:
+            res[i] = int(k in M)
+            M.pop(k, None)
+    return np.array(res, dtype=np.uint8)
+
+
+@pytest.mark.parametrize("R", [1, 3, 16, 200])
+def test_oracle_seq_vs_dict_with_duplicates(R):
+    rng = np.random.default_rng(100 + R)
+    o = OracleMap(R, seed=5)
+    M = {}
+    for _ in range(300):
+        B = int(rng.integers(0, 40))
+        op = rng.integers(0, 3, size=B).astype(np.uint8)
+        key = rng.integers(0, R + 1, size=B).astype(np.uint32)  # R = invalid
+        val = rng.integers(0, 2**32, size=B, dtype=np.uint64).astype(np.uint32)
+        r = o.batch(op, key, val, combine=True)
+        e = brute_batch_seq(M, op.tolist(), key.tolist(), val.tolist(), R)
+        assert np.array_equal(r, e)
+        ks, vs = o.export()
+        assert ks.tolist() == sorted(M)
+        assert vs.tolist() == [M[k] for k in sorted(M)]
+
+
+def test_oracle_seq_equals_s1_under_contract():
+    R, B = 3000, 2000
+    rng = np.random.default_rng(21)
+    a, b = OracleMap(R), OracleMap(R)
+    for _ in range(10):
+        op, key, val = random_batch(rng, R, B)
+        assert np.array_equal(a.batch(op, key, val), b.batch(op, key, val, combine=True))
+    assert np.array_equal(a.export()[0], b.export()[0])
+    assert np.array_equal(a.export()[1], b.export()[1])
+
+
+def test_oracle_seq_per_key_automaton():
+    """Hand-worked chains on one key (Insert false iff present, Delete false iff absent,
+    Alg 4.5 l.2-4 / Alg 4.11 l.3-5; a present key's value is never overwritten)."""
+    I, D, C = 1, 2, 0
+    o = OracleMap(10)
+    # absent: I(5) I(6) D I(7) C -> 1 0 1 1 | C sees the pre-batch map -> 0; final 7
+    r = o.batch(np.array([I, I, D, I, C], np.uint8), np.full(5, 4, np.uint32),
+                np.array([5, 6, 0, 7, 0], np.uint32), combine=True)
+    assert r.tolist() == [1, 0, 1, 1, 0] and o.get(4) == 7
+    # present (7): D D I(8) I(9) -> 1 0 1 0; final 8
+    r = o.batch(np.array([D, D, I, I], np.uint8), np.full(4, 4, np.uint32),
+                np.array([0, 0, 8, 9], np.uint32), combine=True)
+    assert r.tolist() == [1, 0, 1, 0] and o.get(4) == 8
+    # present: I(1) D C -> 0 1 1; final absent
+    r = o.batch(np.array([I, D, C], np.uint8), np.full(3, 4, np.uint32),
+                np.array([1, 0, 0], np.uint32), combine=True)
+    assert r.tolist() == [0, 1, 1] and o.get(4) is None and len(o) == 0
