@@ -57,7 +57,16 @@ CONFIGS = {
     "M20-20-60-10M": (10_000_000, 5_000_000, 625_000, 16, (20, 20, 60), "uniform", 16),
     "INS-1M": (1_000_000, 0, 125_000, 8, (100, 0, 0), "uniform", 16),     # R inserts, empty start
     "DEL-1M": (1_000_000, 1_000_000, 125_000, 8, (0, 100, 0), "uniform", 16),  # R deletes, full start
+    # NEXT-1: raw Zipf(0.99) -- mutating keys i.i.d. too (no redraws), so hot keys carry
+    # long Insert/Delete chains; run in combining mode (R26), exact for any batch
+    "C2-zipf-raw": (1_000_000, 500_000, 625_000, 16, (10, 10, 80), "zipf", 16),
+    "C3-zipf-raw": (10_000_000, 5_000_000, 6_250_000, 16, (10, 10, 80), "zipf", 16),
 }
+COMBINE_CONFIGS = {"C2-zipf-raw", "C3-zipf-raw"}
+
+
+def combine_mode(args) -> bool:
+    return args.config in COMBINE_CONFIGS or getattr(args, "combine", False)
 L2_FLUSH_BYTES = 256 << 20
 
 
@@ -171,7 +180,7 @@ def max_over_ranks(x: float, world: int) -> float:
 # --------------------------------------------------------------------------------------
 # reference arm / cpu baseline: the oracle as it stands, on this host's cores
 
-def oracle_sample(cfg_name, steps, warmup, budget_s=20.0, per_step_ops=1_000_000):
+def oracle_sample(cfg_name, steps, warmup, budget_s=20.0, per_step_ops=1_000_000, combine=False):
     """Times Oracle-A on a bounded sample of the config's own batches (1 host thread)."""
     from oracle.oracle_a import OracleMap
     R, pre, B, nb, mix, dist, N = CONFIGS[cfg_name]
@@ -189,17 +198,17 @@ def oracle_sample(cfg_name, steps, warmup, budget_s=20.0, per_step_ops=1_000_000
     o.batch(np.ones(pre_s, np.uint8), k.numpy().astype(np.uint32),
             prefill_values(SEED_BASE, k).numpy().astype(np.uint32))
     Bs = min(B, per_step_ops)
-    w = Workload(Rs, Bs, mix=mix, dist=dist, seed=SEED_BASE + 1)
+    w = Workload(Rs, Bs, mix=mix, dist=dist, seed=SEED_BASE + 1, dedup=not combine)
     batches = []
     for b in range(warmup + steps):
         op, key, val, _ = w.make_batch(b)
         batches.append((op.numpy(), key.numpy().astype(np.uint32), val.numpy().astype(np.uint32)))
     for b in range(warmup):
-        o.batch(*batches[b])
+        o.batch(*batches[b], combine=combine)
     t_total, n_total, done = 0.0, 0, 0
     for b in range(warmup, warmup + steps):
         t0 = time.perf_counter()
-        o.batch(*batches[b])
+        o.batch(*batches[b], combine=combine)
         t_total += time.perf_counter() - t0
         n_total += Bs
         done += 1
@@ -214,7 +223,8 @@ def run_reference(args, world, rank):
     cfg = args.config
     if rank != 0:
         return
-    mops, t, done, Bs, note = oracle_sample(cfg, args.steps, args.warmup, budget_s=60.0)
+    mops, t, done, Bs, note = oracle_sample(cfg, args.steps, args.warmup, budget_s=60.0,
+                                            combine=combine_mode(args))
     line = {
         "impl": "reference", "metric": METRIC, "value": round(mops, 4), "unit": "Mops/s",
         "n_gpus": args.gpus, "steps": done, "warmup": args.warmup,
@@ -274,6 +284,8 @@ def run_gpu(args, world, rank, local):
     else:
         g = GFSL(R, capacity=R, chunk_entries=N, contains_team=args.team)
         prefill_gpu(g, R, pre1, dev)
+    if combine_mode(args):
+        (g.local if world > 1 else g).configure(combine=1)
     if args.l2_window:
         (g.local if world > 1 else g).configure(l2_window=1)
     if args.no_pdl:
@@ -281,7 +293,8 @@ def run_gpu(args, world, rank, local):
     (g.local if world > 1 else g).configure(
         rebuild_every=0xFFFFFFFF if args.rebuild_every < 0 else args.rebuild_every)
     PROF = 3  # extra batches after the timed region, for the per-kernel breakdown
-    w = Workload(R, B1, mix=mix, dist=dist, seed=SEED_BASE + 1 + 7919 * rank)
+    w = Workload(R, B1, mix=mix, dist=dist, seed=SEED_BASE + 1 + 7919 * rank,
+                 dedup=not combine_mode(args))
     inputs = [make_inputs(w, b, dev) for b in range(W + steps + PROF)]
     redraws = sum(x[3] for x in inputs)
     flush = torch.empty(L2_FLUSH_BYTES, dtype=torch.uint8, device=dev)
@@ -292,7 +305,8 @@ def run_gpu(args, world, rank, local):
     torch.cuda.synchronize()
     barrier(world)
     local_g = g.local if world > 1 else g
-    mut0 = local_g.stats()["mutations"]
+    st0 = local_g.stats()
+    mut0 = st0["mutations"]
 
     starts = [torch.cuda.Event(enable_timing=True) for _ in range(steps)]
     ends = [torch.cuda.Event(enable_timing=True) for _ in range(steps)]
@@ -315,7 +329,12 @@ def run_gpu(args, world, rank, local):
     total_ms = max_over_ranks(local_ms, world)
     ops_total = B1 * steps * world
     mops = ops_total / (total_ms / 1e3) / 1e6
-    n_mut = (local_g.stats()["mutations"] - mut0) / max(steps, 1)
+    st_t = local_g.stats()
+    n_mut = (st_t["mutations"] - mut0) / max(steps, 1)
+    # our kernels launched inside the timed region (counted by libgfsl at enqueue), plus the
+    # route kernels of the multi-GPU path (3 plan + pack + unpack per step)
+    launches = int(st_t["kernel_launches"] - st0["kernel_launches"]) + (5 * steps if world > 1 else 0)
+    lib_launches = int(st_t["library_launches"] - st0["library_launches"])
     # per-kernel breakdown: CUDA events between the kernels of PROF extra batches (events
     # between kernels would defeat the programmatic dependent launch of the timed steps)
     local_g.configure(profile_phases=1)
@@ -394,6 +413,8 @@ def run_gpu(args, world, rank, local):
     if not args.no_e2e and world == 1:
         g2 = GFSL(R, capacity=R, chunk_entries=N, contains_team=args.team)
         prefill_gpu(g2, R, pre1, dev)
+        if combine_mode(args):
+            g2.configure(combine=1)
         host = [(x[0].cpu().pin_memory(), x[1].cpu().pin_memory(), x[2].cpu().pin_memory())
                 for x in inputs]
         out = torch.empty(B1, dtype=torch.uint8).pin_memory()
@@ -412,7 +433,8 @@ def run_gpu(args, world, rank, local):
 
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
-        cm, ct, cdone, cBs, note = oracle_sample(args.config, min(steps, 16), 1, budget_s=15.0)
+        cm, ct, cdone, cBs, note = oracle_sample(args.config, min(steps, 16), 1, budget_s=15.0,
+                                                combine=combine_mode(args))
         cpu = {"value": round(cm, 4), "unit": "Mops/s", "cores": 1, "kind": "oracle",
                "sample": f"{cdone} batches of {cBs} ops ({ct:.1f} s); {note}"}
 
@@ -430,6 +452,8 @@ def run_gpu(args, world, rank, local):
             "config": {"workload": args.config, "key_range": R,
                        "rebuild_every": "never" if args.rebuild_every < 0 else (args.rebuild_every or 2), "prefill": pre1 * world,
                        "batch_ops": B1 * world, "mix_ins_del_con": list(mix), "keys": dist,
+                       "semantics": "combining (R26): mutations in input order, any batch" if combine_mode(args)
+                       else "S1 snapshot, <=1 mutation per key (R1/R2)",
                        "chunk_entries": N, "contains_team": local_g.cfg.contains_team or (4 if N == 32 else 2),
                        "l2": "flushed (256 MiB write) between timed steps",
                        "parallelism": f"range-shard x{world}" if world > 1 else "1 GPU"},
@@ -444,7 +468,8 @@ def run_gpu(args, world, rank, local):
             "chunk_reads_l0_per_contains": round(reads_l0_per_op, 3),
             "cpu_baseline": cpu,
             "e2e": e2e,
-            "gpu_launches": 4 * steps + (5 * steps if world > 1 else 0),  # classify, search, update, upkeep (+ route plan x3, pack, unpack)
+            "gpu_launches": launches,
+            "library_launches": lib_launches,  # CUB radix-sort kernels (combining mode only)
             "clocks": clk,
             "wall_s_timed_region": round(wall, 4),
             "generator_redraws": int(redraws),
@@ -467,6 +492,8 @@ def main():
     ap.add_argument("--validate", action="store_true")
     ap.add_argument("--no-ubench", action="store_true", help="skip the B6 roofline microbenchmark")
     ap.add_argument("--no-pdl", action="store_true", help="no programmatic dependent launch (ablation)")
+    ap.add_argument("--combine", action="store_true",
+                    help="combining mode (R26) for any config (always on for *-raw configs)")
     ap.add_argument("--rebuild-every", type=int, default=0,
                     help="rebuild the upper levels after every k-th batch (R24); "
                          "0 = library default (2), -1 = never (the paper's dynamics only)")

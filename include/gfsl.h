@@ -19,7 +19,8 @@
  * batch is  M + {successful inserts} - {successful deletes}.  Contract: at most one
  * mutating op (Insert/Delete) per key per batch.  Outside the contract every result is
  * still the result of SOME linearization of the batch, but parity with the
- * oracle is only promised inside it.
+ * oracle is only promised inside it -- unless the handle runs in combining mode
+ * (gfsl_config.combine, reading R26), which is exact for any batch.
  *
  * Keys are valid in [0, key_range), key_range <= 2^32 - 2 (the two extremes of the
  * 32-bit internal key space are the -inf / +inf sentinels of P:203).  Any uint32 is a
@@ -82,6 +83,16 @@ typedef struct gfsl_config {
                                (R24: "compact the structure between kernel
                                launches").  0 = GFSL_REBUILD_DEFAULT_PERIOD;
                                GFSL_REBUILD_NEVER = the paper's structure dynamics only */
+  uint32_t combine;         /* 1 = combining mode (R26): exact
+                               for ANY batch, with no <=1-mutation-per-key contract.  The
+                               Contains of a batch still see the map before the batch (S1);
+                               the Insert/Delete ops are linearized in input order, so each
+                               one's result follows the paper's Insert (false iff present,
+                               Alg 4.5 l.2-4; no overwrite) and Delete (false iff absent,
+                               Alg 4.11 l.3-5) applied one after another.  Each key's chain
+                               is reduced to at most one net structural op (or an in-place
+                               value write) before the update kernel.  Costs a radix sort of
+                               the batch's keys.  0 = the contract mode of R1. */
 } gfsl_config;
 
 /*
@@ -174,7 +185,9 @@ typedef struct gfsl_stats {
   uint64_t contains_reads_l0; /* ... of which on the bottom level */
   uint64_t contains_ops;    /* Contains ops counted (count_reads=1) */
   uint64_t mutations;       /* Insert/Delete ops that changed the map */
-  uint64_t reserved[4];
+  uint64_t kernel_launches; /* libgfsl kernels enqueued by gfsl_batch calls so far */
+  uint64_t library_launches;/* library (CUB radix sort, combining mode) kernels, estimated */
+  uint64_t reserved[2];
 } gfsl_stats;
 gfsl_status gfsl_get_stats(gfsl_t h, gfsl_stats *out);
 

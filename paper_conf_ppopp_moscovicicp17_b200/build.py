@@ -15,7 +15,7 @@ ROOT = os.path.dirname(HERE)
 CSRC = os.path.join(HERE, "csrc")
 LIB = os.path.join(HERE, "libgfsl.so")
 SOURCES = ["gfsl.cu"]
-HEADERS = ["gfsl_device.cuh", "gfsl_search.cuh", "gfsl_update.cuh", "gfsl_ubench.cuh", "gfsl_rebuild.cuh"]
+HEADERS = ["gfsl_device.cuh", "gfsl_search.cuh", "gfsl_update.cuh", "gfsl_ubench.cuh", "gfsl_rebuild.cuh", "gfsl_combine.cuh"]
 
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]

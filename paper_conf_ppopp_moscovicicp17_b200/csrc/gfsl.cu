@@ -23,6 +23,9 @@
 #include "gfsl_update.cuh"
 #include "gfsl_ubench.cuh"
 #include "gfsl_rebuild.cuh"
+#include "gfsl_combine.cuh"
+
+#include <cub/device/device_radix_sort.cuh>
 
 using namespace gfsl_dev;
 
@@ -62,12 +65,22 @@ struct gfsl {
   uint32_t *st_key = nullptr, *st_val = nullptr;
   uint64_t st_cap = 0;
   uint64_t batches = 0, ops = 0;
+  uint64_t launches = 0, lib_launches = 0;  // our kernels / CUB's (combining sort) enqueued by batches
   std::vector<std::array<cudaEvent_t, 5>> phase_ev;  // profile_phases
   // L2 persistence for the upper pool (the search kernel's access-policy window)
   size_t persist_max = 0, window_max = 0;
   uint32_t *h_bump = nullptr;  // pinned copy of the bump counters, refreshed every batch
   RebuildBufs rb{};            // upper-level rebuild (R24)
   uint32_t *rc_tiles = nullptr;  // zombie reclamation scratch (R25)
+  // combining mode (R26): sort double buffers, net mutations, value writes, CUB scratch
+  uint32_t *ck[2] = {nullptr, nullptr}, *cw[2] = {nullptr, nullptr};
+  uint4 *net_rec = nullptr;
+  uint32_t *net_path = nullptr;
+  uint2 *vw = nullptr;
+  void *cub_tmp = nullptr;
+  size_t cub_bytes = 0;
+  uint64_t comb_cap = 0;
+  int sort_bits = 32;
 };
 
 // ------------------------------------------------------------------------------------
@@ -112,8 +125,19 @@ static void set_pdl(gfsl *h, cudaLaunchAttribute &a) {
   a.val.programmaticStreamSerializationAllowed = h->cfg.no_pdl ? 0 : 1;
 }
 
+// What the search kernel writes: the records of the ops whose snapshot answer mutates
+// (numbered by ctl->n_mut, or by ctl->n_cand when the combine kernel picks the net ones).
 static SearchOut search_out(gfsl *h) {
-  return SearchOut{h->mut_rec, h->plan_path, h->cfg.serial_updates ? h->mut_of : nullptr};
+  if (h->cfg.combine)
+    return SearchOut{h->mut_rec, h->plan_path, h->mut_of, &h->ctl->n_cand, h->ck[0], h->cw[0]};
+  return SearchOut{h->mut_rec, h->plan_path, h->cfg.serial_updates ? h->mut_of : nullptr,
+                   &h->ctl->n_mut, nullptr, nullptr};
+}
+// What the update kernel reads: the same records, or the net mutations of combining mode.
+static SearchOut update_in(gfsl *h) {
+  if (h->cfg.combine)
+    return SearchOut{h->net_rec, h->net_path, h->mut_of, &h->ctl->n_mut, nullptr, nullptr};
+  return search_out(h);
 }
 
 // The upper levels live in one contiguous range (the upper pool, chunks [0, cap_upper)),
@@ -145,6 +169,7 @@ static void launch_contains(gfsl *h, const BatchIn &in, cudaStream_t s) {
     cudaLaunchKernelEx(&lc, search_kernel<N, TEAM, true>, h->d, in, h->ctl, search_out(h));
   else
     cudaLaunchKernelEx(&lc, search_kernel<N, TEAM, false>, h->d, in, h->ctl, search_out(h));
+  h->launches += 1;
 }
 
 #define GFSL_CONTAINS_CONFIGS(X) \
@@ -171,15 +196,22 @@ static void launch_update(gfsl *h, const BatchIn &in, cudaStream_t s, cudaEvent_
   lc.blockDim = dim3(h->cfg.serial_updates ? 32 : 256);
   lc.gridDim = dim3(h->cfg.serial_updates ? 1 : h->update_grid);
   const int serial = h->cfg.serial_updates ? 1 : 0;
-  cudaLaunchKernelEx(&lc, update_kernel<N>, h->d, in, h->ctl, search_out(h), serial);
-  if (after_update) cudaEventRecord(after_update, s);
+  cudaLaunchKernelEx(&lc, update_kernel<N>, h->d, in, h->ctl, update_in(h), serial);
+  h->launches += 2;  // update + upkeep
   lc.blockDim = dim3(256);
+  if (h->cfg.combine) {  // R26: keys deleted and re-inserted in this batch get their new value
+    lc.gridDim = dim3(h->sms * 2);
+    cudaLaunchKernelEx(&lc, value_write_kernel<N>, h->d, (const BatchCtl *)h->ctl, (const uint2 *)h->vw);
+    h->launches += 1;
+  }
+  if (after_update) cudaEventRecord(after_update, s);
   lc.gridDim = dim3(h->sms * 4);
   cudaLaunchKernelEx(&lc, upkeep_kernel<N>, h->d);
   // R24: rebuild the upper levels from level 0 after every `rebuild_every`-th batch
   const uint32_t every = h->cfg.rebuild_every == 0 ? GFSL_REBUILD_DEFAULT_PERIOD : h->cfg.rebuild_every;
   if (every != GFSL_REBUILD_NEVER && (h->batches + 1) % every == 0) {
     const RebuildBufs &b = h->rb;
+    h->launches += 9;
     lc.gridDim = dim3(1);
     lc.blockDim = dim3(32);
     cudaLaunchKernelEx(&lc, rebuild_begin_kernel, b);
@@ -304,6 +336,14 @@ static void free_all(gfsl *h) {
   cudaFree(h->rb.n1);
   cudaFree(h->rb.levels);
   cudaFree(h->rc_tiles);
+  for (int b = 0; b < 2; ++b) {
+    cudaFree(h->ck[b]);
+    cudaFree(h->cw[b]);
+  }
+  cudaFree(h->net_rec);
+  cudaFree(h->net_path);
+  cudaFree(h->vw);
+  cudaFree(h->cub_tmp);
   cudaFree(h->d.freelist);
   cudaFree(h->d.fl);
   if (h->h_error) cudaFreeHost(h->h_error);
@@ -443,6 +483,14 @@ extern "C" void gfsl_destroy(gfsl_t h) {
   free_all(h);
 }
 
+// bits of the combining sort: internal keys are in [1, key_range]; the all-ones key of
+// Contains / invalid ops must compare above every real key within the sorted bits
+static int sort_bits_for(uint64_t key_range) {
+  int b = 1;
+  while (b < 32 && (1ull << b) - 1 <= key_range) ++b;
+  return b;
+}
+
 // ------------------------------------------------------------------------------------
 // batch
 
@@ -479,6 +527,70 @@ static gfsl_status ensure_lists(gfsl *h, uint64_t n) {
   return GFSL_OK;
 }
 
+// Combining-mode buffers (R26), grown on demand like the lists.
+static gfsl_status ensure_combine(gfsl *h, uint64_t n) {
+  h->sort_bits = sort_bits_for(h->key_range);
+  size_t need = 0;
+  {
+    cub::DoubleBuffer<uint32_t> kb(nullptr, nullptr), vb(nullptr, nullptr);
+    CK(cub::DeviceRadixSort::SortPairs(nullptr, need, kb, vb, (int)std::max<uint64_t>(n, h->comb_cap), 0, h->sort_bits));
+  }
+  if (n <= h->comb_cap && need <= h->cub_bytes) return GFSL_OK;
+  cudaDeviceSynchronize();
+  if (n > h->comb_cap) {
+    for (int b = 0; b < 2; ++b) {
+      cudaFree(h->ck[b]);
+      cudaFree(h->cw[b]);
+      h->ck[b] = h->cw[b] = nullptr;
+    }
+    cudaFree(h->net_rec);
+    cudaFree(h->net_path);
+    cudaFree(h->vw);
+    h->net_rec = nullptr;
+    h->net_path = nullptr;
+    h->vw = nullptr;
+    h->comb_cap = 0;
+    const uint64_t cap = std::max<uint64_t>(n, 1024);
+    for (int b = 0; b < 2; ++b) {
+      CK(cudaMalloc(&h->ck[b], cap * 4));
+      CK(cudaMalloc(&h->cw[b], cap * 4));
+    }
+    CK(cudaMalloc(&h->net_rec, cap * 16));
+    CK(cudaMalloc(&h->net_path, cap * 4 * PLAN_LEVELS));
+    CK(cudaMalloc(&h->vw, cap * 8));
+    h->comb_cap = cap;
+  }
+  if (need > h->cub_bytes) {
+    cudaFree(h->cub_tmp);
+    h->cub_tmp = nullptr;
+    h->cub_bytes = 0;
+    CK(cudaMalloc(&h->cub_tmp, need));
+    h->cub_bytes = need;
+  }
+  return GFSL_OK;
+}
+
+// R26: sort the batch's (key, op) pairs so that each key's Insert/Delete chain is
+// contiguous and in input order (LSD radix sort is stable), then reduce the chains.
+static gfsl_status enqueue_combine(gfsl *h, const BatchIn &in, cudaStream_t s) {
+  cub::DoubleBuffer<uint32_t> kb(h->ck[0], h->ck[1]), vb(h->cw[0], h->cw[1]);
+  size_t bytes = h->cub_bytes;
+  CK(cub::DeviceRadixSort::SortPairs(h->cub_tmp, bytes, kb, vb, (int)in.n, 0, h->sort_bits, s));
+  h->lib_launches += 1 + (uint64_t)(h->sort_bits + 7) / 8;  // onesweep: histogram + one pass per 8-bit digit
+  h->launches += 1;  // combine_kernel
+  cudaLaunchConfig_t lc{};
+  cudaLaunchAttribute attr[1];
+  set_pdl(h, attr[0]);
+  lc.attrs = attr;
+  lc.numAttrs = 1;
+  lc.stream = s;
+  lc.blockDim = dim3(256);
+  lc.gridDim = dim3((unsigned)std::min<uint64_t>((in.n + 255) / 256, (uint64_t)h->sms * 8));
+  CK(cudaLaunchKernelEx(&lc, combine_kernel, in, h->ctl, (const uint32_t *)kb.Current(),
+                        (const uint32_t *)vb.Current(), search_out(h), update_in(h), h->vw));
+  return GFSL_OK;
+}
+
 static gfsl_status enqueue_batch(gfsl *h, const uint8_t *ops, const uint32_t *keys,
                                  const uint32_t *vals, uint8_t *res, uint64_t n, cudaStream_t s) {
   CK(cudaStreamWaitEvent(s, h->last, 0));
@@ -492,11 +604,15 @@ static gfsl_status enqueue_batch(gfsl *h, const uint8_t *ops, const uint32_t *ke
   if (prof) CK(cudaEventRecord(ev[1], s));
   const BatchIn in{ops, keys, vals, res, (uint32_t)n, h->key_range};
   bool ok = dispatch_contains(h, in, s);
-  if (prof) CK(cudaEventRecord(ev[2], s));
   if (!ok) {
     set_last_error("no contains kernel for this (N, team)");
     return GFSL_EINVAL;
   }
+  if (h->cfg.combine) {
+    gfsl_status cs = enqueue_combine(h, in, s);
+    if (cs != GFSL_OK) return cs;
+  }
+  if (prof) CK(cudaEventRecord(ev[2], s));
   switch (h->N) {
     case 32: launch_update<32>(h, in, s, prof ? ev[3] : nullptr); break;
     case 16: launch_update<16>(h, in, s, prof ? ev[3] : nullptr); break;
@@ -535,6 +651,7 @@ extern "C" gfsl_status gfsl_batch(gfsl_t h, const uint8_t *op_types, const uint3
     return GFSL_EINVAL;
   }
   if ((st = ensure_lists(h, n)) != GFSL_OK) return st;
+  if (h->cfg.combine && (st = ensure_combine(h, n)) != GFSL_OK) return st;
   return enqueue_batch(h, op_types, keys, values, results, n, (cudaStream_t)stream);
 }
 
@@ -568,6 +685,7 @@ extern "C" gfsl_status gfsl_batch_host(gfsl_t h, const uint8_t *op_types, const 
     h->st_cap = n;
   }
   if ((st = ensure_lists(h, n)) != GFSL_OK) return st;
+  if (h->cfg.combine && (st = ensure_combine(h, n)) != GFSL_OK) return st;
   cudaStream_t s = (cudaStream_t)stream;
   CK(cudaMemcpyAsync(h->st_op, op_types, n, cudaMemcpyHostToDevice, s));
   CK(cudaMemcpyAsync(h->st_key, keys, n * 4, cudaMemcpyHostToDevice, s));
@@ -604,6 +722,8 @@ extern "C" gfsl_status gfsl_get_stats(gfsl_t h, gfsl_stats *out) {
   out->contains_reads_l0 = s[ST_CREADS_L0];
   out->contains_ops = s[ST_COPS];
   out->mutations = s[ST_MUTATIONS];
+  out->kernel_launches = h->launches;
+  out->library_launches = h->lib_launches;
   return GFSL_OK;
 }
 

@@ -64,9 +64,9 @@ struct DevState {
 
 // Per-batch control block (device memory, zeroed before every batch).
 struct BatchCtl {
-  uint32_t unused1;
-  uint32_t unused2;
-  uint32_t n_mut;        // update ops that mutate (search kernel)
+  uint32_t n_cand;       // combining mode (R26): records written by the search kernel
+  uint32_t n_vw;         // combining mode: value writes (combine kernel)
+  uint32_t n_mut;        // update ops that mutate (search kernel, or the combine kernel)
   uint32_t unused0;
   uint32_t snap_height;  // height seen by the search kernel
   uint32_t n_merges;     // merges of this batch (update kernel) -> upkeep sweep

@@ -66,8 +66,19 @@ struct BatchIn {
 struct SearchOut {
   uint4 *mut_rec;       // [n]: {op index | DELETE_FLAG, internal key, path[0], top (Delete) | value (Insert)}
   uint32_t *plan_path;  // [n * PLAN_LEVELS]: mutation m's path, lane l = chunk at level l
-  uint32_t *mut_of;     // [n] or NULL: op i -> its mutation index, 0xFFFFFFFF if none (serial mode)
+  uint32_t *mut_of;     // [n] or NULL: op i -> its mutation index, 0xFFFFFFFF if none (serial
+                        // and combining modes)
+  uint32_t *mut_count;  // the counter that numbers the records (ctl->n_mut, or ctl->n_cand
+                        // when a combining pass selects the net mutations, R26)
+  uint32_t *comb_key;   // [n] or NULL (combining mode, R26): op i's sort key = internal key
+                        // for a valid Insert/Delete, else all ones
+  uint32_t *comb_w;     // [n]: op i | CW_* flags (the sort's payload)
 };
+
+// Combining-mode payload flags (R26); the op index is < 2^29.
+constexpr uint32_t CW_P0 = 0x80000000u;      // k was present in the snapshot
+constexpr uint32_t CW_DEL = 0x40000000u;     // Delete (else Insert)
+constexpr uint32_t CW_NOTMUT = 0x20000000u;  // Contains or invalid: not part of any chain
 
 template <int N, int TEAM, bool COUNT = false>
 __global__ void __launch_bounds__(256)
@@ -226,7 +237,7 @@ search_kernel(DevState d, const BatchIn in, BatchCtl *__restrict__ ctl, SearchOu
             const bool mut = (cur_op.x & DELETE_FLAG) ? te : !te;
             res[opi] = mut ? 1 : 0;
             if (mut) {
-              m = atomicAdd(&ctl->n_mut, 1u);
+              m = atomicAdd(so.mut_count, 1u);
               // {op index | DELETE_FLAG, key, path[0], top (Delete) | value (Insert)}
               const uint32_t w = opi | (cur_op.x & DELETE_FLAG);
               so.mut_rec[m] = make_uint4(w, k, here, (cur_op.x & DELETE_FLAG) ? seen_top : cur_val);
@@ -238,6 +249,11 @@ search_kernel(DevState d, const BatchIn in, BatchCtl *__restrict__ ctl, SearchOu
             }
           }
           if (so.mut_of) so.mut_of[opi] = m;
+          if (so.comb_key) {  // R26: the op's place in its key's chain
+            const bool chain = upd && !(cur_op.x & INVALID_FLAG);
+            so.comb_key[opi] = chain ? k : 0xFFFFFFFFu;
+            so.comb_w[opi] = opi | (chain ? ((te ? CW_P0 : 0u) | ((cur_op.x & DELETE_FLAG) ? CW_DEL : 0u)) : CW_NOTMUT);
+          }
         }
         if (COUNT) ++nops;
         // next op of this team (prefetched one ahead)

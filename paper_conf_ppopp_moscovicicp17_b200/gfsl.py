@@ -33,7 +33,7 @@ class gfsl_config(ctypes.Structure):
                 ("serial_updates", ctypes.c_uint32), ("count_reads", ctypes.c_uint32),
                 ("profile_phases", ctypes.c_uint32), ("l2_window", ctypes.c_uint32),
                 ("no_pdl", ctypes.c_uint32),
-                ("rebuild_every", ctypes.c_uint32)]
+                ("rebuild_every", ctypes.c_uint32), ("combine", ctypes.c_uint32)]
 
 
 class gfsl_report(ctypes.Structure):
@@ -52,7 +52,8 @@ class gfsl_stats(ctypes.Structure):
                 ("merges", ctypes.c_uint64), ("zombie_unlinks", ctypes.c_uint64),
                 ("lock_retries", ctypes.c_uint64), ("contains_reads", ctypes.c_uint64),
                 ("contains_reads_l0", ctypes.c_uint64), ("contains_ops", ctypes.c_uint64),
-                ("mutations", ctypes.c_uint64), ("reserved", ctypes.c_uint64 * 4)]
+                ("mutations", ctypes.c_uint64), ("kernel_launches", ctypes.c_uint64),
+                ("library_launches", ctypes.c_uint64), ("reserved", ctypes.c_uint64 * 2)]
 
 
 class gfsl_meta(ctypes.Structure):
@@ -167,7 +168,7 @@ class GFSL:
                  contains_team: int = 0, serial_updates: bool = False,
                  contains_blocks_per_sm: int = 0, update_blocks_per_sm: int = 0,
                  count_reads: bool = False, profile_phases: bool = False,
-                 rebuild_every: int = 0):
+                 rebuild_every: int = 0, combine: bool = False):
         import torch
         if not torch.cuda.is_available():
             raise RuntimeError("GFSL needs a CUDA device (there is no CPU fallback)")
@@ -175,7 +176,7 @@ class GFSL:
         cfg = gfsl_config(chunk_entries, contains_team, contains_blocks_per_sm,
                           update_blocks_per_sm, 1 if serial_updates else 0,
                           1 if count_reads else 0, 1 if profile_phases else 0, 0, 0,
-                          rebuild_every)
+                          rebuild_every, 1 if combine else 0)
         self.key_range = int(key_range)
         self.chunk_entries = int(chunk_entries)
         self.cfg = cfg

@@ -15,7 +15,8 @@ Recipe (the paper's workloads):
   the mix exact.
 * mutating keys of one batch are drawn WITHOUT replacement (the <=1-mutating-op-per-key
   contract, R2): a colliding draw is redrawn from the next counter value, up to
-  64 tries, then uniformly.
+  64 tries, then uniformly.  ``dedup=False`` keeps the i.i.d. draws (for combining mode,
+  DESIGN.md R26, which has no contract).
 * value = ``h(seed, VAL, i) mod 2^32`` (the paper inserts NULL; random values make
   the export check meaningful).
 * prefill = the first P elements of a keyed Feistel permutation of [0, R) (cycle walking),
@@ -137,6 +138,7 @@ class Workload:
     dist: str = "uniform"          # "uniform" | "zipf"
     zipf_s: float = 0.99
     seed: int = SEED_BASE
+    dedup: bool = True             # False: mutating keys i.i.d. too (combining mode, R26)
     _zipf: ZipfTable | None = field(default=None, repr=False)
 
     def n_ins_del(self):
@@ -167,7 +169,7 @@ class Workload:
         val = uniform_u32(self.seed, VAL, gidx)
         redraws = 0
         mut = (op != CONTAINS).nonzero().flatten()
-        if mut.numel():
+        if mut.numel() and self.dedup:
             key, redraws = self._dedup_mutating(key, mut, gidx, device)
         return op, key, val, redraws
 
