@@ -346,6 +346,8 @@ static void free_all(gfsl *h) {
   cudaFree(h->cub_tmp);
   cudaFree(h->d.freelist);
   cudaFree(h->d.fl);
+  cudaFree(h->d.dir);
+  cudaFree(h->d.dir_hdr);
   if (h->h_error) cudaFreeHost(h->h_error);
   if (h->h_bump) cudaFreeHost(h->h_bump);
   if (h->last) cudaEventDestroy(h->last);
@@ -436,6 +438,13 @@ extern "C" gfsl_t gfsl_create_ex(uint64_t key_range, uint64_t capacity, const gf
     if ((e = cudaMalloc(&h->d.fl, 8 * 4)) != cudaSuccess) return fail("cudaMalloc(freelist)", e);
     if ((e = cudaMalloc(&h->rc_tiles, ((size_t)cap_b / RC_TILE + 2) * 4)) != cudaSuccess) return fail("cudaMalloc(reclaim)", e);
     cudaMemset(h->d.fl, 0, 8 * 4);
+    // R27: level-1 directory, about one bucket per level-1 key, at most 2^22 (16 MiB)
+    uint32_t dcap = 1024;
+    while (dcap < (1u << 22) && (uint64_t)dcap < key_range + 1) dcap <<= 1;
+    h->d.dir_cap = dcap;
+    if ((e = cudaMalloc(&h->d.dir, (size_t)dcap * 4)) != cudaSuccess) return fail("cudaMalloc(dir)", e);
+    if ((e = cudaMalloc(&h->d.dir_hdr, 4 * 4)) != cudaSuccess) return fail("cudaMalloc(dir)", e);
+    cudaMemset(h->d.dir_hdr, 0, 4 * 4);
 #ifdef GFSL_DEBUG_TIMING
     if ((e = cudaMalloc(&h->d.debug_times, ((size_t)148 * 64 * 48 + 64) * 8)) != cudaSuccess) return fail("cudaMalloc", e);
     cudaMemset(h->d.debug_times, 0, ((size_t)148 * 64 * 48 + 64) * 8);
@@ -797,6 +806,7 @@ extern "C" gfsl_status gfsl_load(gfsl_t h, const gfsl_meta *meta, const uint64_t
   CK(cudaMemcpy(h->d.counter, meta->counters, 32 * 4, cudaMemcpyHostToDevice));
   uint32_t bump[2] = {meta->used_bottom, meta->used_upper};
   CK(cudaMemcpy(h->d.bump, bump, 8, cudaMemcpyHostToDevice));
+  CK(cudaMemset(h->d.dir_hdr, 0, 4 * 4));  // the directory describes the old structure
   return GFSL_OK;
 }
 

@@ -60,6 +60,12 @@ struct DevState {
   uint32_t *fl;          // [0] free chunks in the current list, [1] taken, [2] buffer,
                          // [3..5] reclaim scratch
   unsigned long long *debug_times;  // GFSL_DEBUG_TIMING builds: per-team (start, end, ops)
+  // Level-1 directory (R27): dir[b] = the level-1 chunk holding the largest level-1 key
+  // <= (b << shift), written by each upper-level rebuild.  dir_hdr = {shift, valid,
+  // buckets}; valid = 0 until the first rebuild (and after gfsl_load).
+  uint32_t *dir;
+  uint32_t *dir_hdr;
+  uint32_t dir_cap;      // entries allocated (a power of two)
 };
 
 // Per-batch control block (device memory, zeroed before every batch).

@@ -177,11 +177,42 @@ __global__ void __launch_bounds__(1024) rebuild_scan_top_kernel(RebuildBufs b) {
   }
 }
 
-// (4) each marked chunk writes itself at its rank
+// rank of key k among the marked min keys: how many are <= k
+__device__ __forceinline__ uint32_t rb_rank_le(const RebuildBufs &b, uint32_t k) {
+  const uint32_t w = k >> 5, bit = k & 31;
+  const uint32_t mask = bit == 31 ? 0xFFFFFFFFu : ((2u << bit) - 1u);
+  return b.block_sum[w / RB_BLOCK_WORDS] + b.word_prefix[w] + __popc(b.bitmap[w] & mask);
+}
+
+// (4) each marked chunk writes itself at its rank; the level-1 directory (R27)
 template <int N>
 __global__ void __launch_bounds__(256) rebuild_rank_kernel(const __grid_constant__ DevState d, RebuildBufs b) {
   pdl_wait();
   if (!rb_active(b)) return;
+  {
+    // R27: bucket q = keys [q << shift, (q+1) << shift); its entry is the level-1 chunk
+    // that holds the largest level-1 key <= q << shift.  Level-1 entry i >= 1 is the i-th
+    // marked min key, so that entry is number rank(q << shift), in chunk rank / F of the
+    // packed level 1 (rebuild_pack_kernel).  About one bucket per level-1 key.
+    const uint32_t n1 = b.n1[0];
+    uint32_t target = 1024;
+    while (target < 2u * n1 && target < d.dir_cap) target <<= 1;
+    target = min(target, d.dir_cap);
+    int shift = 0;
+    while (((uint64_t)d.key_max >> shift) + 1 > target) ++shift;
+    const uint32_t buckets = (uint32_t)((uint64_t)d.key_max >> shift) + 1;
+    const RbLevels *L = (const RbLevels *)b.levels;
+    const uint32_t base1 = L->base[1];
+    for (uint32_t q = blockIdx.x * blockDim.x + threadIdx.x; q < buckets; q += gridDim.x * blockDim.x) {
+      const uint32_t j = rb_rank_le(b, q << shift) / b.fill;
+      d.dir[q] = j == 0 ? 0u : base1 + j - 1;  // rb_chunk(L, 1, j)
+    }
+    if (blockIdx.x == 0 && threadIdx.x == 0) {
+      d.dir_hdr[0] = (uint32_t)shift;
+      d.dir_hdr[1] = 1u;
+      d.dir_hdr[2] = buckets;
+    }
+  }
   const uint32_t used = min(d.bump[0], d.cap_bottom);
   for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < used; i += gridDim.x * blockDim.x) {
     const uint32_t c = d.cap_upper + i;

@@ -80,8 +80,12 @@ constexpr uint32_t CW_P0 = 0x80000000u;      // k was present in the snapshot
 constexpr uint32_t CW_DEL = 0x40000000u;     // Delete (else Insert)
 constexpr uint32_t CW_NOTMUT = 0x20000000u;  // Contains or invalid: not part of any chain
 
+#ifndef GFSL_SEARCH_MIN_BLOCKS
+#define GFSL_SEARCH_MIN_BLOCKS 1
+#endif
+
 template <int N, int TEAM, bool COUNT = false>
-__global__ void __launch_bounds__(256)
+__global__ void __launch_bounds__(256, GFSL_SEARCH_MIN_BLOCKS)
 search_kernel(DevState d, const BatchIn in, BatchCtl *__restrict__ ctl, SearchOut so) {
   constexpr int EPL = N / TEAM;
   static_assert(EPL * TEAM == N, "TEAM must divide N");
@@ -92,7 +96,7 @@ search_kernel(DevState d, const BatchIn in, BatchCtl *__restrict__ ctl, SearchOu
   constexpr int LOCK_LANE = LOCK_E / EPL, LOCK_J = LOCK_E % EPL;
   constexpr uint32_t FULL = 0xFFFFFFFFu;
 
-  __shared__ uint32_t s_start, s_height;
+  __shared__ uint32_t s_start, s_height, s_dir_shift;
   // the path of the team's current op (written by its lane 0 only), copied out compactly
   // at the end if the op mutates (about 1 op in 10)
   __shared__ __align__(16) uint32_t s_path[(256 / 32) * TPW][PLAN_LEVELS];
@@ -107,12 +111,21 @@ search_kernel(DevState d, const BatchIn in, BatchCtl *__restrict__ ctl, SearchOu
     if (lane == 0) {
       s_height = h;
       s_start = d.head[h];
+      // R27: Contains enter at level 1 through the directory when there are levels above
+      s_dir_shift = (h >= 2 && d.dir_hdr[1]) ? d.dir_hdr[0] : 32u;
       if (blockIdx.x == 0) ctl->snap_height = h;
     }
   }
   __syncthreads();
   const uint32_t start = s_start;
   const int height = (int)s_height;
+  const uint32_t dir_shift = s_dir_shift;
+  const bool use_dir = dir_shift < 32u;
+  // where a traversal starts: searchDown from the top (Alg 4.2 l.2-4), or -- for a
+  // Contains when the directory is valid -- at level 1, in the chunk the directory names
+  // for k's bucket (R27).  Insert/Delete always start at the top: searchSlow records the
+  // whole path (Alg 4.6).
+  auto dir_op = [&](uint32_t opw) { return use_dir && !(opw & (UPDATE_FLAG | INVALID_FLAG)); };
   const uint32_t n = in.n;
   uint8_t *__restrict__ res = in.res;
 
@@ -157,8 +170,12 @@ search_kernel(DevState d, const BatchIn in, BatchCtl *__restrict__ ctl, SearchOu
   RawOp nxt = load_raw(slot + total_teams);
   bool active = lane_live && slot < n;
   uint32_t k = cur_op.y;
-  uint32_t cur = start;
-  int level = height;
+  uint32_t cur = dir_op(cur_op.x) ? __ldg(d.dir + (k >> dir_shift)) : start;
+  int level = dir_op(cur_op.x) ? 1 : height;
+  // the next op's directory word is loaded one loop iteration after its raw op (so that
+  // its key has arrived), and is ready when the op becomes current
+  uint32_t nxt_dir = start;
+  bool pf_dir = use_dir;
   uint32_t bt = NULL_CHUNK, bt_c = NULL_CHUNK;       // prevKv, reduced
   int seen_top = 0;                                  // highest level where k was seen
   unsigned long long restarts = 0;
@@ -167,6 +184,10 @@ search_kernel(DevState d, const BatchIn in, BatchCtl *__restrict__ ctl, SearchOu
   while (__any_sync(FULL, active)) {
     ChunkSlice<EPL> s;
     ld_slice_nc<EPL>(d.pool + (size_t)cur * N + t * EPL, s);  // idle teams re-read `cur`
+    if (pf_dir) {
+      if (nxt.op == 0 && (uint64_t)nxt.key < in.key_range) nxt_dir = __ldg(d.dir + ((nxt.key + 1u) >> dir_shift));
+      pf_dir = false;
+    }
     if (COUNT && active) {
       ++reads;
       reads_l0 += (level == 0);
@@ -209,7 +230,9 @@ search_kernel(DevState d, const BatchIn in, BatchCtl *__restrict__ ctl, SearchOu
       const bool lat = (np & (F_ZOMBIE | F_LATERAL)) != 0;  // zombie (l.9-11) / lateral (l.15-18)
       const bool done = !lat && level == 0;                 // bottom enclosing chunk (Alg 4.4)
       const bool down = !lat && level > 0;                  // down step (l.19-23) / backtrack
-      const bool restart = down && !tb && bt == NULL_CHUNK; // (l.25) impossible when quiescent
+      // (l.25): only from a directory entry made stale by the batches since the last
+      // rebuild (R27: level-1 keys <= k deleted from that chunk); never from the top
+      const bool restart = down && !tb && bt == NULL_CHUNK;
       const bool upd = (cur_op.x & UPDATE_FLAG) != 0;
       const uint32_t here = cur;
       if (down && upd && t == 0 && level < PLAN_LEVELS)     // searchSlow's path (Alg 4.6 l.28-37)
@@ -263,8 +286,9 @@ search_kernel(DevState d, const BatchIn in, BatchCtl *__restrict__ ctl, SearchOu
         cur_val = load_val(slot, nxt);
         k = cur_op.y;
         nxt = load_raw(slot + total_teams);
-        cur = start;
-        level = height;
+        cur = dir_op(cur_op.x) ? nxt_dir : start;
+        level = dir_op(cur_op.x) ? 1 : height;
+        pf_dir = use_dir;
         bt = bt_c = NULL_CHUNK;
         seen_top = 0;
       }

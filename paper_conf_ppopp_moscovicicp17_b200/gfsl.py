@@ -17,7 +17,8 @@ from dataclasses import dataclass
 import numpy as np
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "libgfsl.so")
+# GFSL_LIB: an alternative build of the same library (tools/ experiments only)
+LIB_PATH = os.environ.get("GFSL_LIB") or os.path.join(_HERE, "libgfsl.so")
 
 GFSL_OK, GFSL_EINVAL, GFSL_ENOMEM, GFSL_EPOOL, GFSL_ECUDA, GFSL_ECORRUPT = range(6)
 CONTAINS, INSERT, DELETE = 0, 1, 2
