@@ -81,6 +81,7 @@ struct gfsl {
   size_t cub_bytes = 0;
   uint64_t comb_cap = 0;
   int sort_bits = 32;
+  uint32_t region_cap = 1;  // record slots per region for the current batch
 };
 
 // ------------------------------------------------------------------------------------
@@ -129,15 +130,28 @@ static void set_pdl(gfsl *h, cudaLaunchAttribute &a) {
 // (numbered by ctl->n_mut, or by ctl->n_cand when the combine kernel picks the net ones).
 static SearchOut search_out(gfsl *h) {
   if (h->cfg.combine)
-    return SearchOut{h->mut_rec, h->plan_path, h->mut_of, &h->ctl->n_cand, h->ck[0], h->cw[0]};
+    return SearchOut{h->mut_rec, h->plan_path, h->mut_of, h->ctl->ccnt, h->region_cap, h->ck[0], h->cw[0]};
   return SearchOut{h->mut_rec, h->plan_path, h->cfg.serial_updates ? h->mut_of : nullptr,
-                   &h->ctl->n_mut, nullptr, nullptr};
+                   h->ctl->mcnt, h->region_cap, nullptr, nullptr};
 }
 // What the update kernel reads: the same records, or the net mutations of combining mode.
 static SearchOut update_in(gfsl *h) {
   if (h->cfg.combine)
-    return SearchOut{h->net_rec, h->net_path, h->mut_of, &h->ctl->n_mut, nullptr, nullptr};
+    return SearchOut{h->net_rec, h->net_path, h->mut_of, h->ctl->mcnt, h->region_cap, nullptr, nullptr};
   return search_out(h);
+}
+
+// Record slots per region (BatchCtl::mcnt) for a batch of n ops: a region collects the
+// records of the blocks b with b % MUT_REGIONS == r, of the search kernel (each block
+// answers at most teams_per_block * ceil(n / teams) ops) and of the combine kernel.
+static uint32_t region_cap_for(const gfsl *h, uint64_t n) {
+  const uint64_t R = BatchCtl::MUT_REGIONS;
+  const uint64_t tpb = (256 / 32) * (32 / h->team);
+  const uint64_t teams = (uint64_t)h->contains_grid * tpb;
+  const uint64_t s_cap = (((uint64_t)h->contains_grid + R - 1) / R) * tpb * ((n + teams - 1) / teams);
+  const uint64_t cg = std::max<uint64_t>(1, std::min<uint64_t>((n + 255) / 256, (uint64_t)h->sms * 8));
+  const uint64_t c_cap = ((cg + R - 1) / R) * 256 * ((n + 256 * cg - 1) / (256 * cg));
+  return (uint32_t)std::max<uint64_t>(1, std::max(s_cap, c_cap));
 }
 
 // The upper levels live in one contiguous range (the upper pool, chunks [0, cap_upper)),
@@ -519,6 +533,9 @@ static gfsl_status sticky(gfsl *h) {
 }
 
 static gfsl_status ensure_lists(gfsl *h, uint64_t n) {
+  h->region_cap = region_cap_for(h, n);
+  // mut_of is indexed by op; records and paths by region slot
+  n = std::max<uint64_t>(n, (uint64_t)BatchCtl::MUT_REGIONS * h->region_cap);
   if (n <= h->list_cap) return GFSL_OK;
   cudaDeviceSynchronize();
   cudaFree(h->plan_path);
@@ -539,10 +556,12 @@ static gfsl_status ensure_lists(gfsl *h, uint64_t n) {
 // Combining-mode buffers (R26), grown on demand like the lists.
 static gfsl_status ensure_combine(gfsl *h, uint64_t n) {
   h->sort_bits = sort_bits_for(h->key_range);
+  const uint64_t n_sort = n;
+  n = std::max<uint64_t>(n, (uint64_t)BatchCtl::MUT_REGIONS * h->region_cap);  // net records
   size_t need = 0;
   {
     cub::DoubleBuffer<uint32_t> kb(nullptr, nullptr), vb(nullptr, nullptr);
-    CK(cub::DeviceRadixSort::SortPairs(nullptr, need, kb, vb, (int)std::max<uint64_t>(n, h->comb_cap), 0, h->sort_bits));
+    CK(cub::DeviceRadixSort::SortPairs(nullptr, need, kb, vb, (int)std::max<uint64_t>(n_sort, h->comb_cap), 0, h->sort_bits));
   }
   if (n <= h->comb_cap && need <= h->cub_bytes) return GFSL_OK;
   cudaDeviceSynchronize();

@@ -32,7 +32,7 @@ namespace gfsl_dev {
 
 // One thread per sorted element.  sk/sw: the sorted keys and payloads (n elements).
 // cand: the search kernel's records (and mut_of: op -> record); net: where the net
-// mutations go (counted by ctl->n_mut).  vw: value writes {internal key, value} (ctl->n_vw).
+// mutations go (numbered per region in ctl->mcnt).  vw: value writes {internal key, value} (ctl->n_vw).
 __global__ void __launch_bounds__(256)
 combine_kernel(const BatchIn in, BatchCtl *__restrict__ ctl, const uint32_t *__restrict__ sk,
                const uint32_t *__restrict__ sw, SearchOut cand, SearchOut net, uint2 *__restrict__ vw) {
@@ -65,7 +65,7 @@ combine_kernel(const BatchIn in, BatchCtl *__restrict__ ctl, const uint32_t *__r
     const uint32_t v_new = fin && in.vals ? in.vals[sw[r] & OPI_MASK] : 0u;
     if (p0 != fin) {  // net Insert (absent -> present) or net Delete (present -> absent)
       const uint32_t m = cand.mut_of[i];  // the last op's snapshot answer mutates: recorded
-      q = atomicAdd(&ctl->n_mut, 1u);
+      q = mut_slot(net);
       uint4 rec = cand.mut_rec[m];
       if (fin) rec.w = v_new;
       net.mut_rec[q] = rec;

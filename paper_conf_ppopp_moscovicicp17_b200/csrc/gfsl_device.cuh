@@ -70,13 +70,21 @@ struct DevState {
 
 // Per-batch control block (device memory, zeroed before every batch).
 struct BatchCtl {
-  uint32_t n_cand;       // combining mode (R26): records written by the search kernel
+  uint32_t unused1;
   uint32_t n_vw;         // combining mode: value writes (combine kernel)
-  uint32_t n_mut;        // update ops that mutate (search kernel, or the combine kernel)
+  uint32_t unused2;
   uint32_t unused0;
   uint32_t snap_height;  // height seen by the search kernel
   uint32_t n_merges;     // merges of this batch (update kernel) -> upkeep sweep
   uint32_t pad[2];
+  // Mutation records are numbered per region: region r (= the writing block's index mod
+  // MUT_REGIONS) owns record slots [r * region_cap, (r+1) * region_cap) and counts them
+  // in mcnt[r] (records the update kernel applies) or ccnt[r] (combining mode: the search
+  // kernel's candidates).  32 counters instead of one keep the appends of all blocks from
+  // serialising on one L2 atomic.
+  static constexpr int MUT_REGIONS = 32;
+  uint32_t mcnt[MUT_REGIONS];
+  uint32_t ccnt[MUT_REGIONS];
   // dynamic work queues of the update kernel (one per update block, at most UQ_MAX):
   // queue j of Q hands out the mutation slots j, j + Q, j + 2Q, ... in order; one counter
   // per 32-byte sector

@@ -68,12 +68,19 @@ struct SearchOut {
   uint32_t *plan_path;  // [n * PLAN_LEVELS]: mutation m's path, lane l = chunk at level l
   uint32_t *mut_of;     // [n] or NULL: op i -> its mutation index, 0xFFFFFFFF if none (serial
                         // and combining modes)
-  uint32_t *mut_count;  // the counter that numbers the records (ctl->n_mut, or ctl->n_cand
-                        // when a combining pass selects the net mutations, R26)
+  uint32_t *mut_count;  // the MUT_REGIONS counters that number the records (ctl->mcnt, or
+                        // ctl->ccnt when a combining pass selects the net mutations, R26)
+  uint32_t region_cap;  // record slots per region (BatchCtl::mcnt)
   uint32_t *comb_key;   // [n] or NULL (combining mode, R26): op i's sort key = internal key
                         // for a valid Insert/Delete, else all ones
   uint32_t *comb_w;     // [n]: op i | CW_* flags (the sort's payload)
 };
+
+// A record slot in the writing block's region (BatchCtl::mcnt).
+__device__ __forceinline__ uint32_t mut_slot(const SearchOut &so) {
+  const uint32_t rg = blockIdx.x % BatchCtl::MUT_REGIONS;
+  return rg * so.region_cap + atomicAdd(so.mut_count + rg, 1u);
+}
 
 // Combining-mode payload flags (R26); the op index is < 2^29.
 constexpr uint32_t CW_P0 = 0x80000000u;      // k was present in the snapshot
@@ -260,7 +267,7 @@ search_kernel(DevState d, const BatchIn in, BatchCtl *__restrict__ ctl, SearchOu
             const bool mut = (cur_op.x & DELETE_FLAG) ? te : !te;
             res[opi] = mut ? 1 : 0;
             if (mut) {
-              m = atomicAdd(so.mut_count, 1u);
+              m = mut_slot(so);
               // {op index | DELETE_FLAG, key, path[0], top (Delete) | value (Insert)}
               const uint32_t w = opi | (cur_op.x & DELETE_FLAG);
               so.mut_rec[m] = make_uint4(w, k, here, (cur_op.x & DELETE_FLAG) ? seen_top : cur_val);
@@ -299,6 +306,38 @@ search_kernel(DevState d, const BatchIn in, BatchCtl *__restrict__ ctl, SearchOu
     stat_add(d, ST_CREADS, reads);
     stat_add(d, ST_CREADS_L0, reads_l0);
     stat_add(d, ST_COPS, nops);
+  }
+}
+
+// The update kernel's view of the region-numbered records: slot s in [0, total) ->
+// record index.  Built once per block from the MUT_REGIONS counters (shared memory).
+struct MutMap {
+  const uint32_t *excl;  // [MUT_REGIONS + 1] exclusive prefix of the counts (shared)
+  uint32_t cap;
+  __device__ __forceinline__ uint32_t total() const { return excl[BatchCtl::MUT_REGIONS]; }
+  __device__ __forceinline__ uint32_t rec(uint32_t s) const {
+    int r = 0;  // the last region whose prefix is <= s (empty regions are skipped)
+#pragma unroll
+    for (int step = BatchCtl::MUT_REGIONS / 2; step >= 1; step >>= 1)
+      if (excl[r + step] <= s) r += step;
+    return (uint32_t)r * cap + (s - excl[r]);
+  }
+};
+
+// Fills s_excl (MUT_REGIONS + 1 entries) from the counters; call from every thread of
+// the block before any thread returns, then __syncthreads().
+__device__ __forceinline__ void mutmap_build(const uint32_t *cnt, uint32_t *s_excl) {
+  if (threadIdx.x < 32) {
+    const int lane = threadIdx.x;
+    const uint32_t v = cnt[lane];
+    uint32_t incl = v;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      const uint32_t y = __shfl_up_sync(0xFFFFFFFFu, incl, o);
+      if (lane >= o) incl += y;
+    }
+    s_excl[lane] = incl - v;
+    if (lane == 31) s_excl[32] = incl;
   }
 }
 
