@@ -43,10 +43,25 @@ class PoolExhausted(Exception):
     pass
 
 
+def raise_draw(rkey: int, level: int) -> int:
+    """isKeyRaised's random draw: a counter-based 32-bit
+    hash of (raised key, level of the split) -- the murmur3 finalizer of
+    rkey ^ level * 0x9E3779B9 ^ 0x2545F491.  The key is raised iff the draw < p * 2^32."""
+    x = (rkey ^ (level * 0x9E3779B9) ^ 0x2545F491) & 0xFFFFFFFF
+    x ^= x >> 16
+    x = (x * 0x85EBCA6B) & 0xFFFFFFFF
+    x ^= x >> 13
+    x = (x * 0xC2B2AE35) & 0xFFFFFFFF
+    x ^= x >> 16
+    return x
+
+
 class GFSLModel:
     def __init__(self, N: int, key_range: int, cap_bottom: int, cap_upper: int,
-                 rebuild_every: int = 0):
+                 rebuild_every: int = 0, p_chunk_q32: int = 0):
         assert N >= 6
+        # p_chunk (P:471, P:1068-1072) as a 32-bit fraction; 0 = p_chunk = 1 (R16)
+        self.p_chunk_q32 = p_chunk_q32
         self.rebuild_every = rebuild_every
         self.batches = 0
         self.dirty = False
@@ -348,7 +363,10 @@ class GFSLModel:
         if not hold:
             self.unlock(other)                            # Alg 4.9 l.6-9
         self.update_down_ptrs(level, moved, pnew)         # Alg 4.9 l.12
-        return True, pins, pextra, True, rkey, rptr       # p_chunk = 1 (R16)
+        # isKeyRaised (Alg 4.5 l.15): always at p_chunk = 1 (R16), else with
+        # probability p_chunk (the counter-based draw of R28)
+        up = self.p_chunk_q32 == 0 or raise_draw(rkey, level) < self.p_chunk_q32
+        return True, pins, pextra, up, rkey, rptr
 
     def insert(self, k, v, path):
         ok, pins, pextra, raise_, rkey, rptr = self.insert_to_level(0, path[0], k, v)

@@ -162,3 +162,36 @@ def test_reclaimed_chunks_bound_the_pool():
         runs[every] = used
     assert runs[1][-1] == runs[1][60]          # plateau with reclamation
     assert runs[0][-1] > runs[0][60] + 20      # keeps leaking without it
+
+
+@pytest.mark.parametrize("N,p", [(6, 0.5), (16, 0.25), (32, 0.5)])
+def test_model_with_p_chunk_matches_oracle_a(N, p):
+    """p_chunk < 1 (R28): results, final set and invariants unchanged; fewer
+    keys reach the upper levels than at p_chunk = 1 (the raise is a coin flip per split)."""
+    R = 400 if N <= 12 else 2000
+    q = int(p * 2**32)
+    m = GFSLModel(N, R, cap_bottom=4000, cap_upper=1000, p_chunk_q32=q)
+    m1 = GFSLModel(N, R, cap_bottom=4000, cap_upper=1000)
+    o = OracleMap(R)
+    w = Workload(R, 150, mix=(45, 25, 30), seed=SEED_BASE + 7 * N)
+    for b in range(30):
+        op, key, val, _ = w.make_batch(b)
+        opn, kn, vn = op.numpy(), key.numpy().astype(np.uint32), val.numpy().astype(np.uint32)
+        r = m.batch(opn.tolist(), kn.tolist(), vn.tolist())
+        m1.batch(opn.tolist(), kn.tolist(), vn.tolist())
+        assert r == o.batch(opn, kn, vn).tolist()
+        assert m.check_invariants() == []
+    ks, vs = m.export()
+    ok, ov = o.export()
+    assert ks == ok.tolist() and vs == ov.tolist()
+    upper = lambda mm: sum(len(mm.level_keys(l)) for l in range(1, mm.N))  # noqa: E731
+    assert upper(m) < upper(m1)
+
+
+def test_raise_draw_is_uniform():
+    """The draw of R28 is a fixed bijective mix of its input: about p of all (key, level)
+    pairs are raised, and the fraction is monotone in p."""
+    from oracle.oracle_b import raise_draw
+    d = np.array([raise_draw(k, lv) for k in range(1, 20001) for lv in range(3)], np.uint64)
+    for p in (0.25, 0.5, 0.75):
+        assert abs(float((d < int(p * 2**32)).mean()) - p) < 0.01
