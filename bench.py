@@ -284,14 +284,14 @@ def run_gpu(args, world, rank, local):
     else:
         g = GFSL(R, capacity=R, chunk_entries=N, contains_team=args.team)
         prefill_gpu(g, R, pre1, dev)
-    if combine_mode(args):
-        (g.local if world > 1 else g).configure(combine=1)
-    if args.l2_window:
-        (g.local if world > 1 else g).configure(l2_window=1)
-    if args.no_pdl:
-        (g.local if world > 1 else g).configure(no_pdl=1)
-    (g.local if world > 1 else g).configure(
-        rebuild_every=0xFFFFFFFF if args.rebuild_every < 0 else args.rebuild_every)
+    def apply_options(h):
+        """The run's library options (identical for the timed and the e2e handles)."""
+        h.configure(combine=1 if combine_mode(args) else 0,
+                    p_chunk_q32=int(args.p_chunk * 2**32) if args.p_chunk < 1.0 else 0,
+                    l2_window=1 if args.l2_window else 0, no_pdl=1 if args.no_pdl else 0,
+                    rebuild_every=0xFFFFFFFF if args.rebuild_every < 0 else args.rebuild_every)
+
+    apply_options(g.local if world > 1 else g)
     PROF = 3  # extra batches after the timed region, for the per-kernel breakdown
     w = Workload(R, B1, mix=mix, dist=dist, seed=SEED_BASE + 1 + 7919 * rank,
                  dedup=not combine_mode(args))
@@ -413,23 +413,48 @@ def run_gpu(args, world, rank, local):
     if not args.no_e2e and world == 1:
         g2 = GFSL(R, capacity=R, chunk_entries=N, contains_team=args.team)
         prefill_gpu(g2, R, pre1, dev)
-        if combine_mode(args):
-            g2.configure(combine=1)
+        apply_options(g2)
         host = [(x[0].cpu().pin_memory(), x[1].cpu().pin_memory(), x[2].cpu().pin_memory())
                 for x in inputs]
         out = torch.empty(B1, dtype=torch.uint8).pin_memory()
+        outs = [torch.empty(B1, dtype=torch.uint8).pin_memory() for _ in range(steps)]
         for b in range(W):
             g2.batch_host(*host[b], out=out)
-        t_e2e = 0.0
+        # (a) synchronous calls, one per step, L2 flushed before each (outside the timer)
+        t_sync = 0.0
         for j in range(steps):
             flush.zero_()
             torch.cuda.synchronize()
             t0 = time.perf_counter()
             g2.batch_host(*host[W + j], out=out)
-            t_e2e += time.perf_counter() - t0
-        e2e = {"value": round(B1 * steps / t_e2e / 1e6, 3), "unit": "Mops/s",
-               "h2d_bytes_per_step": B1 * 9, "d2h_bytes_per_step": B1}
+            t_sync += time.perf_counter() - t0
+        # (b) the headline: the K steps back to back through gfsl_batch_host_async, as a
+        # user streams batches (copy-in of step j+1 overlaps the kernels of step j), from
+        # the first call until every step's results are in host memory; wall clock
+        g3 = GFSL(R, capacity=R, chunk_entries=N, contains_team=args.team)
+        prefill_gpu(g3, R, pre1, dev)
+        apply_options(g3)
+        out_w = torch.empty(B1, dtype=torch.uint8).pin_memory()
+        for b in range(W):
+            g3.batch_host(*host[b], out=out_w)
+        torch.cuda.synchronize()
+        t0 = time.perf_counter()
+        for j in range(steps):
+            g3.batch_host_async(*host[W + j], out=outs[j])
+        torch.cuda.synchronize()
+        t_pipe = time.perf_counter() - t0
+        e2e = {"value": round(B1 * steps / t_pipe / 1e6, 3), "unit": "Mops/s",
+               "h2d_bytes_per_step": B1 * 9, "d2h_bytes_per_step": B1,
+               "how": "gfsl_batch_host_async, K steps back to back from pinned host buffers, wall "
+                      "clock from the first call to the last result in host memory; L2 not "
+                      "flushed between these steps",
+               "sync_per_step": {"value": round(B1 * steps / t_sync / 1e6, 3), "unit": "Mops/s",
+                                 "how": "gfsl_batch_host (synchronous) per step, L2 flushed before "
+                                        "each step, summed wall time of the calls"}}
+        # both handles ran the same sequence: their answers must agree
+        assert torch.equal(out, outs[-1]), "e2e paths disagree"
         g2.close()
+        g3.close()
 
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
@@ -454,7 +479,7 @@ def run_gpu(args, world, rank, local):
                        "batch_ops": B1 * world, "mix_ins_del_con": list(mix), "keys": dist,
                        "semantics": "combining (R26): mutations in input order, any batch" if combine_mode(args)
                        else "S1 snapshot, <=1 mutation per key (R1/R2)",
-                       "chunk_entries": N, "contains_team": local_g.cfg.contains_team or (4 if N == 32 else 2),
+                       "chunk_entries": N, "p_chunk": args.p_chunk, "contains_team": local_g.cfg.contains_team or (4 if N == 32 else 2),
                        "l2": "flushed (256 MiB write) between timed steps",
                        "parallelism": f"range-shard x{world}" if world > 1 else "1 GPU"},
             "roofline": roofline,
@@ -492,6 +517,8 @@ def main():
     ap.add_argument("--validate", action="store_true")
     ap.add_argument("--no-ubench", action="store_true", help="skip the B6 roofline microbenchmark")
     ap.add_argument("--no-pdl", action="store_true", help="no programmatic dependent launch (ablation)")
+    ap.add_argument("--p-chunk", type=float, default=1.0,
+                    help="isKeyRaised probability (P:1068-1072, R28) for the timed batches; 1 = the default")
     ap.add_argument("--combine", action="store_true",
                     help="combining mode (R26) for any config (always on for *-raw configs)")
     ap.add_argument("--rebuild-every", type=int, default=0,

@@ -93,6 +93,13 @@ typedef struct gfsl_config {
                                is reduced to at most one net structural op (or an in-place
                                value write) before the update kernel.  Costs a radix sort of
                                the batch's keys.  0 = the contract mode of R1. */
+  uint32_t p_chunk_q32;     /* p_chunk, the probability that a split raises a key to the
+                               level above (isKeyRaised; swept in P:1068-1072), as a
+                               32-bit fraction p * 2^32.  0 = p_chunk = 1, the paper's best
+                               and the default (R16, R28).  The draw is a hash of
+                               (raised key, level), so runs are reproducible.  The periodic
+                               upper-level rebuild (rebuild_every) replaces what the raises
+                               built; combine with GFSL_REBUILD_NEVER to study p_chunk. */
 } gfsl_config;
 
 /*
@@ -142,6 +149,19 @@ gfsl_status gfsl_batch(gfsl_t h, const uint8_t *op_types, const uint32_t *keys,
 gfsl_status gfsl_batch_host(gfsl_t h, const uint8_t *op_types, const uint32_t *keys,
                             const uint32_t *values, uint8_t *results, uint64_t n,
                             void *stream);
+
+/*
+ * The same, asynchronous: returns once the copies and kernels are enqueued.  The inputs
+ * are copied on a library-owned copy stream into one of two device staging slots, so
+ * the copy-in of the next batch overlaps the kernels of this one; the batch and the
+ * copy-out of the results run on `stream`.  `results` holds the answers once `stream`
+ * has reached this point (e.g. after cudaStreamSynchronize).  The host buffers must stay
+ * valid and unmodified until then, and must be pinned (page-locked) for the copies to
+ * be asynchronous (pageable buffers still work, with synchronous copies).
+ */
+gfsl_status gfsl_batch_host_async(gfsl_t h, const uint8_t *op_types, const uint32_t *keys,
+                                  const uint32_t *values, uint8_t *results, uint64_t n,
+                                  void *stream);
 
 /* Result of gfsl_validate: the invariants of PAPER.md §4.3 and P:203. */
 typedef struct gfsl_report {

@@ -60,10 +60,14 @@ struct gfsl {
   cudaEvent_t last = nullptr;
   bool sticky_cuda = false;
   int contains_grid = 0, update_grid = 0;
-  // staging for gfsl_batch_host
-  uint8_t *st_op = nullptr, *st_res = nullptr;
-  uint32_t *st_key = nullptr, *st_val = nullptr;
+  // staging for gfsl_batch_host(_async): two slots, so that the host->device copy of
+  // batch b+1 (on the copy stream) overlaps the kernels of batch b
+  uint8_t *st_op[2] = {nullptr, nullptr}, *st_res[2] = {nullptr, nullptr};
+  uint32_t *st_key[2] = {nullptr, nullptr}, *st_val[2] = {nullptr, nullptr};
   uint64_t st_cap = 0;
+  int st_slot = 0;
+  cudaStream_t copy_stream = nullptr;
+  cudaEvent_t ev_in[2] = {nullptr, nullptr}, ev_used[2] = {nullptr, nullptr};
   uint64_t batches = 0, ops = 0;
   uint64_t launches = 0, lib_launches = 0;  // our kernels / CUB's (combining sort) enqueued by batches
   std::vector<std::array<cudaEvent_t, 5>> phase_ev;  // profile_phases
@@ -338,10 +342,15 @@ static void free_all(gfsl *h) {
   cudaFree(h->plan_path);
   cudaFree(h->mut_of);
   cudaFree(h->mut_rec);
-  cudaFree(h->st_op);
-  cudaFree(h->st_res);
-  cudaFree(h->st_key);
-  cudaFree(h->st_val);
+  for (int b = 0; b < 2; ++b) {
+    cudaFree(h->st_op[b]);
+    cudaFree(h->st_res[b]);
+    cudaFree(h->st_key[b]);
+    cudaFree(h->st_val[b]);
+    if (h->ev_in[b]) cudaEventDestroy(h->ev_in[b]);
+    if (h->ev_used[b]) cudaEventDestroy(h->ev_used[b]);
+  }
+  if (h->copy_stream) cudaStreamDestroy(h->copy_stream);
   cudaFree(h->rb.bitmap);
   cudaFree(h->rb.word_prefix);
   cudaFree(h->rb.block_sum);
@@ -417,6 +426,7 @@ extern "C" gfsl_t gfsl_create_ex(uint64_t key_range, uint64_t capacity, const gf
   h->d.cap_bottom = (uint32_t)cap_b;
   h->d.cap_upper = (uint32_t)cap_u;
   h->d.key_max = (uint32_t)key_range;
+  h->d.p_chunk_q32 = cfg.p_chunk_q32;
   const uint64_t total_entries = (cap_b + cap_u) * N;
   if ((e = cudaMalloc(&h->d.pool, total_entries * 8)) != cudaSuccess) return fail("cudaMalloc(pool)", e);
   if ((e = cudaMalloc(&h->d.head, 32 * 4)) != cudaSuccess) return fail("cudaMalloc", e);
@@ -493,6 +503,7 @@ extern "C" gfsl_status gfsl_configure(gfsl_t h, const gfsl_config *cfg) {
   }
   h->cfg = *cfg;
   h->cfg.chunk_entries = h->N;
+  h->d.p_chunk_q32 = cfg->p_chunk_q32;
   h->cfg.contains_team = team;
   h->team = team;
   apply_launch_shape(h);
@@ -683,13 +694,42 @@ extern "C" gfsl_status gfsl_batch(gfsl_t h, const uint8_t *op_types, const uint3
   return enqueue_batch(h, op_types, keys, values, results, n, (cudaStream_t)stream);
 }
 
-extern "C" gfsl_status gfsl_batch_host(gfsl_t h, const uint8_t *op_types, const uint32_t *keys,
-                                       const uint32_t *values, uint8_t *results, uint64_t n,
-                                       void *stream) {
-  if (!h) {
-    set_last_error("NULL handle");
-    return GFSL_EINVAL;
+static gfsl_status ensure_staging(gfsl *h, uint64_t n) {
+  if (!h->copy_stream) {
+    CK(cudaStreamCreateWithFlags(&h->copy_stream, cudaStreamNonBlocking));
+    for (int b = 0; b < 2; ++b) {
+      CK(cudaEventCreateWithFlags(&h->ev_in[b], cudaEventDisableTiming));
+      CK(cudaEventCreateWithFlags(&h->ev_used[b], cudaEventDisableTiming));
+    }
   }
+  if (n <= h->st_cap) return GFSL_OK;
+  cudaDeviceSynchronize();
+  h->st_cap = 0;
+  for (int b = 0; b < 2; ++b) {
+    cudaFree(h->st_op[b]);
+    cudaFree(h->st_res[b]);
+    cudaFree(h->st_key[b]);
+    cudaFree(h->st_val[b]);
+    h->st_op[b] = h->st_res[b] = nullptr;
+    h->st_key[b] = h->st_val[b] = nullptr;
+  }
+  for (int b = 0; b < 2; ++b) {
+    CK(cudaMalloc(&h->st_op[b], n));
+    CK(cudaMalloc(&h->st_res[b], n));
+    CK(cudaMalloc(&h->st_key[b], n * 4));
+    CK(cudaMalloc(&h->st_val[b], n * 4));
+  }
+  h->st_cap = n;
+  return GFSL_OK;
+}
+
+// The host-buffer batch, asynchronous: the inputs go to staging slot b on the copy stream
+// (after the kernels of the batch that last used the slot have read it), the batch runs
+// on `stream` once they have arrived, and the results come back on `stream`.  So with
+// pinned host memory the copy-in of the next batch overlaps this batch's kernels.
+static gfsl_status batch_host_async(gfsl *h, const uint8_t *op_types, const uint32_t *keys,
+                                    const uint32_t *values, uint8_t *results, uint64_t n,
+                                    cudaStream_t s) {
   gfsl_status st = sticky(h);
   if (st != GFSL_OK) return st;
   if (n == 0) return GFSL_OK;
@@ -697,32 +737,47 @@ extern "C" gfsl_status gfsl_batch_host(gfsl_t h, const uint8_t *op_types, const 
     set_last_error("bad batch arguments");
     return GFSL_EINVAL;
   }
-  if (n > h->st_cap) {
-    cudaDeviceSynchronize();
-    cudaFree(h->st_op);
-    cudaFree(h->st_res);
-    cudaFree(h->st_key);
-    cudaFree(h->st_val);
-    h->st_op = h->st_res = nullptr;
-    h->st_key = h->st_val = nullptr;
-    h->st_cap = 0;
-    CK(cudaMalloc(&h->st_op, n));
-    CK(cudaMalloc(&h->st_res, n));
-    CK(cudaMalloc(&h->st_key, n * 4));
-    CK(cudaMalloc(&h->st_val, n * 4));
-    h->st_cap = n;
-  }
+  if ((st = ensure_staging(h, n)) != GFSL_OK) return st;
   if ((st = ensure_lists(h, n)) != GFSL_OK) return st;
   if (h->cfg.combine && (st = ensure_combine(h, n)) != GFSL_OK) return st;
-  cudaStream_t s = (cudaStream_t)stream;
-  CK(cudaMemcpyAsync(h->st_op, op_types, n, cudaMemcpyHostToDevice, s));
-  CK(cudaMemcpyAsync(h->st_key, keys, n * 4, cudaMemcpyHostToDevice, s));
-  if (values) CK(cudaMemcpyAsync(h->st_val, values, n * 4, cudaMemcpyHostToDevice, s));
-  st = enqueue_batch(h, h->st_op, h->st_key, values ? h->st_val : nullptr, h->st_res, n, s);
+  const int b = h->st_slot;
+  h->st_slot ^= 1;
+  cudaStream_t c = h->copy_stream;
+  CK(cudaStreamWaitEvent(c, h->ev_used[b], 0));  // the slot's previous batch has read it
+  CK(cudaMemcpyAsync(h->st_op[b], op_types, n, cudaMemcpyHostToDevice, c));
+  CK(cudaMemcpyAsync(h->st_key[b], keys, n * 4, cudaMemcpyHostToDevice, c));
+  if (values) CK(cudaMemcpyAsync(h->st_val[b], values, n * 4, cudaMemcpyHostToDevice, c));
+  CK(cudaEventRecord(h->ev_in[b], c));
+  CK(cudaStreamWaitEvent(s, h->ev_in[b], 0));
+  st = enqueue_batch(h, h->st_op[b], h->st_key[b], values ? h->st_val[b] : nullptr, h->st_res[b], n, s);
   if (st != GFSL_OK) return st;
-  CK(cudaMemcpyAsync(results, h->st_res, n, cudaMemcpyDeviceToHost, s));
+  CK(cudaEventRecord(h->ev_used[b], s));
+  CK(cudaMemcpyAsync(results, h->st_res[b], n, cudaMemcpyDeviceToHost, s));
+  return GFSL_OK;
+}
+
+extern "C" gfsl_status gfsl_batch_host(gfsl_t h, const uint8_t *op_types, const uint32_t *keys,
+                                       const uint32_t *values, uint8_t *results, uint64_t n,
+                                       void *stream) {
+  if (!h) {
+    set_last_error("NULL handle");
+    return GFSL_EINVAL;
+  }
+  cudaStream_t s = (cudaStream_t)stream;
+  gfsl_status st = batch_host_async(h, op_types, keys, values, results, n, s);
+  if (st != GFSL_OK) return st;
   CK(cudaStreamSynchronize(s));
   return sticky(h);
+}
+
+extern "C" gfsl_status gfsl_batch_host_async(gfsl_t h, const uint8_t *op_types, const uint32_t *keys,
+                                             const uint32_t *values, uint8_t *results, uint64_t n,
+                                             void *stream) {
+  if (!h) {
+    set_last_error("NULL handle");
+    return GFSL_EINVAL;
+  }
+  return batch_host_async(h, op_types, keys, values, results, n, (cudaStream_t)stream);
 }
 
 #ifdef GFSL_DEBUG_TIMING

@@ -66,7 +66,21 @@ struct DevState {
   uint32_t *dir;
   uint32_t *dir_hdr;
   uint32_t dir_cap;      // entries allocated (a power of two)
+  uint32_t p_chunk_q32;  // isKeyRaised probability as a 32-bit fraction; 0 = 1 (R16)
 };
+
+// isKeyRaised's draw (R28): a counter-based hash of (raised key, level of the split), the
+// murmur3 finalizer; the key is raised iff p_chunk = 1 or draw < p_chunk * 2^32.
+__device__ __forceinline__ bool raise_key(const DevState &d, uint32_t rkey, int level) {
+  if (d.p_chunk_q32 == 0) return true;
+  uint32_t x = rkey ^ ((uint32_t)level * 0x9E3779B9u) ^ 0x2545F491u;
+  x ^= x >> 16;
+  x *= 0x85EBCA6Bu;
+  x ^= x >> 13;
+  x *= 0xC2B2AE35u;
+  x ^= x >> 16;
+  return x < d.p_chunk_q32;
+}
 
 // Per-batch control block (device memory, zeroed before every batch).
 struct BatchCtl {

@@ -34,7 +34,8 @@ class gfsl_config(ctypes.Structure):
                 ("serial_updates", ctypes.c_uint32), ("count_reads", ctypes.c_uint32),
                 ("profile_phases", ctypes.c_uint32), ("l2_window", ctypes.c_uint32),
                 ("no_pdl", ctypes.c_uint32),
-                ("rebuild_every", ctypes.c_uint32), ("combine", ctypes.c_uint32)]
+                ("rebuild_every", ctypes.c_uint32), ("combine", ctypes.c_uint32),
+                ("p_chunk_q32", ctypes.c_uint32)]
 
 
 class gfsl_report(ctypes.Structure):
@@ -67,6 +68,7 @@ class gfsl_meta(ctypes.Structure):
 # Every symbol include/gfsl.h declares (checked by tests/test_abi.py).
 EXPORTS = [
     "gfsl_create", "gfsl_create_ex", "gfsl_destroy", "gfsl_batch", "gfsl_batch_host",
+    "gfsl_batch_host_async",
     "gfsl_validate", "gfsl_last_error", "gfsl_get_stats", "gfsl_dump", "gfsl_load",
     "gfsl_route_plan", "gfsl_route_pack", "gfsl_route_unpack", "gfsl_phase_times",
     "gfsl_configure", "gfsl_ubench",
@@ -96,6 +98,8 @@ def load_library(path: str = LIB_PATH):
     lib.gfsl_batch.argtypes = [vp, vp, vp, vp, vp, u64, vp]
     lib.gfsl_batch_host.restype = i32
     lib.gfsl_batch_host.argtypes = [vp, vp, vp, vp, vp, u64, vp]
+    lib.gfsl_batch_host_async.restype = i32
+    lib.gfsl_batch_host_async.argtypes = [vp, vp, vp, vp, vp, u64, vp]
     lib.gfsl_validate.restype = i32
     lib.gfsl_validate.argtypes = [vp, ctypes.POINTER(gfsl_report), vp, vp, u64,
                                   ctypes.POINTER(u64)]
@@ -169,7 +173,7 @@ class GFSL:
                  contains_team: int = 0, serial_updates: bool = False,
                  contains_blocks_per_sm: int = 0, update_blocks_per_sm: int = 0,
                  count_reads: bool = False, profile_phases: bool = False,
-                 rebuild_every: int = 0, combine: bool = False):
+                 rebuild_every: int = 0, combine: bool = False, p_chunk: float = 1.0):
         import torch
         if not torch.cuda.is_available():
             raise RuntimeError("GFSL needs a CUDA device (there is no CPU fallback)")
@@ -177,7 +181,8 @@ class GFSL:
         cfg = gfsl_config(chunk_entries, contains_team, contains_blocks_per_sm,
                           update_blocks_per_sm, 1 if serial_updates else 0,
                           1 if count_reads else 0, 1 if profile_phases else 0, 0, 0,
-                          rebuild_every, 1 if combine else 0)
+                          rebuild_every, 1 if combine else 0,
+                          0 if p_chunk >= 1.0 else int(p_chunk * 2**32))
         self.key_range = int(key_range)
         self.chunk_entries = int(chunk_entries)
         self.cfg = cfg
@@ -221,6 +226,19 @@ class GFSL:
             out = torch.empty(n, dtype=torch.uint8, pin_memory=op.is_pinned())
         _check(self.lib.gfsl_batch_host(self.h, _ptr(op), _ptr(key), _ptr(val), _ptr(out), n,
                                         _stream(stream)), "gfsl_batch_host")
+        return out
+
+    def batch_host_async(self, op, key, val=None, out=None, stream=None):
+        """Asynchronous batch on (pinned) HOST tensors: `out` holds the results once
+        `stream` (default: the current one) has completed this batch."""
+        import torch
+        n = op.numel()
+        assert not op.is_cuda and op.dtype == torch.uint8 and op.is_contiguous()
+        assert not key.is_cuda and key.element_size() == 4 and key.is_contiguous()
+        if out is None:
+            out = torch.empty(n, dtype=torch.uint8, pin_memory=op.is_pinned())
+        _check(self.lib.gfsl_batch_host_async(self.h, _ptr(op), _ptr(key), _ptr(val), _ptr(out),
+                                              n, _stream(stream)), "gfsl_batch_host_async")
         return out
 
     # ---- inspection ----------------------------------------------------------------

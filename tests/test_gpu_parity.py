@@ -178,6 +178,37 @@ def test_batch_host_matches_device_path():
     assert np.array_equal(k1, k2) and np.array_equal(v1, v2)
 
 
+def test_batch_host_async_pipelined():
+    """Many gfsl_batch_host_async calls in flight (two staging slots reused in turn, the
+    copy-in of batch b+1 overlapping batch b) give the oracle's answers for every batch."""
+    R = 30_000
+    g = GFSL(R)
+    o = OracleMap(R)
+    batches = list(workload_batches(R, 7_001, 9, (20, 20, 60)))
+    host = [tuple(torch.from_numpy(np.ascontiguousarray(a).view(np.int32) if a.dtype == np.uint32 else a).pin_memory()
+                  for a in b) for b in batches]
+    outs = [torch.empty(7_001, dtype=torch.uint8).pin_memory() for _ in batches]
+    for h, out in zip(host, outs):
+        g.batch_host_async(*h, out=out)
+    torch.cuda.synchronize()
+    for (op, key, val), out in zip(batches, outs):
+        assert np.array_equal(out.numpy(), o.batch(op, key, val))
+    check_same_set(g, o)
+
+
+@pytest.mark.parametrize("p", [0.25, 0.5])
+def test_p_chunk_concurrent(p):
+    """p_chunk < 1 with the concurrent update kernel and the paper's structure dynamics."""
+    from paper_conf_ppopp_moscovicicp17_b200.gfsl import REBUILD_NEVER
+    R = 30_000
+    g = GFSL(R, p_chunk=p, rebuild_every=REBUILD_NEVER)
+    o = OracleMap(R)
+    prefill(g, o, R, R // 2, chunk=5000)
+    for op, key, val in workload_batches(R, 6_000 + 3, 6, (20, 20, 60)):
+        run_batch(g, o, op, key, val)
+        check_same_set(g, o)
+
+
 def test_long_churn_reclaims_and_stays_exact():
     """Concurrent 50/50 churn for many batches with rebuild + reclamation every batch:
     results stay bit-exact and the level-0 pool stops growing."""

@@ -19,7 +19,7 @@ pytestmark = pytest.mark.gpu
 def model_like(g: GFSL, key_range, rebuild_every=0):
     meta, _ = g.dump()
     return GFSLModel(meta["chunk_entries"], key_range, meta["cap_bottom"], meta["cap_upper"],
-                     rebuild_every=rebuild_every)
+                     rebuild_every=rebuild_every, p_chunk_q32=g.cfg.p_chunk_q32)
 
 
 def assert_same_structure(g: GFSL, m: GFSLModel, where=""):
@@ -68,6 +68,23 @@ def test_serial_mode_is_byte_identical_to_oracle_b(N, R, B, nb, mix):
     assert st["splits"] > 0
     if mix[2] == 0:
         assert st["merges"] > 0
+
+
+@pytest.mark.parametrize("N,p", [(6, 0.5), (16, 0.25), (32, 0.5)])
+def test_serial_p_chunk_byte_identical_to_oracle_b(N, p):
+    """p_chunk < 1 (isKeyRaised; R28): same pool as Oracle-B."""
+    R = 400 if N == 6 else 3000
+    g = GFSL(R, chunk_entries=N, serial_updates=True, rebuild_every=REBUILD_NEVER, p_chunk=p)
+    m = model_like(g, R)
+    assert m.p_chunk_q32 == int(p * 2**32)
+    w = Workload(R, 300, mix=(40, 30, 30), seed=SEED_BASE + 29 * N)
+    for b in range(16):
+        op, key, val, _ = w.make_batch(b)
+        opn, kn, vn = op.numpy(), key.numpy().astype(np.uint32), val.numpy().astype(np.uint32)
+        r_gpu = g.batch(*dev(opn, kn, vn)).cpu().numpy()
+        r_ora = np.array(m.batch(opn.tolist(), kn.tolist(), vn.tolist()), np.uint8)
+        assert np.array_equal(r_gpu, r_ora), f"batch {b}"
+        assert_same_structure(g, m, f"after batch {b}")
 
 
 @pytest.mark.parametrize("N", [16, 32])
