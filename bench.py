@@ -408,9 +408,16 @@ def run_gpu(args, world, rank, local):
               "gather_GBps": round(n_search * reads_per_op * Cb / (c_ms / 1e3) / 1e9, 1) if c_ms > 0 else None,
               "note": "all chunk gathers of the search kernel incl. L1/L2-resident upper levels"}
 
+    rep = None
+    if args.validate:
+        rep_obj, _, _ = local_g.validate(export=False)
+        rep = {"keys": rep_obj.keys, "height": rep_obj.height, "violations": rep_obj.violations}
+    contains_team = local_g.cfg.contains_team or (4 if N == 32 else 2)
+
     # end to end through the C ABI with host buffers (fresh handle, same sequence)
     e2e = None
     if not args.no_e2e and world == 1:
+        g.close()  # the timed handle is done: free its pool for the e2e handles
         g2 = GFSL(R, capacity=R, chunk_entries=N, contains_team=args.team)
         prefill_gpu(g2, R, pre1, dev)
         apply_options(g2)
@@ -428,6 +435,8 @@ def run_gpu(args, world, rank, local):
             t0 = time.perf_counter()
             g2.batch_host(*host[W + j], out=out)
             t_sync += time.perf_counter() - t0
+        last_sync = out.clone()
+        g2.close()  # one extra handle at a time (a 1B-key pool is ~72 GB)
         # (b) the headline: the K steps back to back through gfsl_batch_host_async, as a
         # user streams batches (copy-in of step j+1 overlaps the kernels of step j), from
         # the first call until every step's results are in host memory; wall clock
@@ -452,8 +461,7 @@ def run_gpu(args, world, rank, local):
                                  "how": "gfsl_batch_host (synchronous) per step, L2 flushed before "
                                         "each step, summed wall time of the calls"}}
         # both handles ran the same sequence: their answers must agree
-        assert torch.equal(out, outs[-1]), "e2e paths disagree"
-        g2.close()
+        assert torch.equal(last_sync, outs[-1]), "e2e paths disagree"
         g3.close()
 
     cpu = None
@@ -462,11 +470,6 @@ def run_gpu(args, world, rank, local):
                                                 combine=combine_mode(args))
         cpu = {"value": round(cm, 4), "unit": "Mops/s", "cores": 1, "kind": "oracle",
                "sample": f"{cdone} batches of {cBs} ops ({ct:.1f} s); {note}"}
-
-    rep = None
-    if args.validate:
-        rep_obj, _, _ = local_g.validate(export=False)
-        rep = {"keys": rep_obj.keys, "height": rep_obj.height, "violations": rep_obj.violations}
 
     if rank == 0:
         line = {
@@ -479,7 +482,7 @@ def run_gpu(args, world, rank, local):
                        "batch_ops": B1 * world, "mix_ins_del_con": list(mix), "keys": dist,
                        "semantics": "combining (R26): mutations in input order, any batch" if combine_mode(args)
                        else "S1 snapshot, <=1 mutation per key (R1/R2)",
-                       "chunk_entries": N, "p_chunk": args.p_chunk, "contains_team": local_g.cfg.contains_team or (4 if N == 32 else 2),
+                       "chunk_entries": N, "p_chunk": args.p_chunk, "contains_team": contains_team,
                        "l2": "flushed (256 MiB write) between timed steps",
                        "parallelism": f"range-shard x{world}" if world > 1 else "1 GPU"},
             "roofline": roofline,

@@ -22,3 +22,22 @@ for N, serial in [(16, False), (32, False), (16, True)]:
     rep, ks, vs = g.validate()
     assert rep.violations == 0 and np.array_equal(ks, o.export()[0])
     print("ok", N, serial, g.stats())
+
+# combining mode (R26) with duplicate keys, and the async host entry point
+R = 2000
+g = GFSL(R, combine=True, rebuild_every=1)
+o = OracleMap(R)
+rng = np.random.default_rng(5)
+outs = []
+for b in range(6):
+    op = rng.integers(0, 3, 1500).astype(np.uint8)
+    key = rng.integers(0, R, 1500).astype(np.uint32)
+    val = rng.integers(0, 2**32, 1500, dtype=np.uint64).astype(np.uint32)
+    h = (torch.from_numpy(op).pin_memory(), torch.from_numpy(key.view(np.int32)).pin_memory(),
+         torch.from_numpy(val.view(np.int32)).pin_memory())
+    outs.append((g.batch_host_async(*h), o.batch(op, key, val, combine=True), h))
+torch.cuda.synchronize()
+assert all(np.array_equal(r.numpy(), e) for r, e, _ in outs)
+rep, ks, vs = g.validate()
+assert rep.violations == 0 and np.array_equal(ks, o.export()[0]) and np.array_equal(vs, o.export()[1])
+print("ok combine+async", g.stats())

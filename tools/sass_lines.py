@@ -1,6 +1,7 @@
 """Attribute an ncu report's per-SASS instruction counts and stall samples to CUDA source
 lines (nvdisasm -g line info of the same libgfsl.so build).
-python tools/sass_lines.py REPORT.ncu-rep KERNEL_MANGLED_PREFIX NCU_NAME_REGEX [lib.so]"""
+python tools/sass_lines.py REPORT.ncu-rep KERNEL_MANGLED_PREFIX NCU_NAME_REGEX [lib.so]
+(SRC_DIR = the csrc/ tree the library was built from, default the working tree)"""
 import collections
 import csv
 import io
@@ -60,7 +61,7 @@ srcs = {}
 for ln, c in agg.most_common(45):
     s = ""
     if ln:
-        p = os.path.join("paper_conf_ppopp_moscovicicp17_b200/csrc", ln[0])
+        p = os.path.join(os.environ.get("SRC_DIR", "paper_conf_ppopp_moscovicicp17_b200/csrc"), ln[0])
         if os.path.exists(p):
             srcs.setdefault(p, open(p).read().split("\n"))
             s = srcs[p][ln[1] - 1].strip()[:80]
