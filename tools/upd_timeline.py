@@ -48,3 +48,7 @@ for name, i in (("insert_locked: split_insert(0)", 40), ("  .. split_chunk(0)", 
     c = cnt[i + 1]
     print(f"  {name:34s} n={c:7d}  cycles/call {cnt[i] / max(c, 1):8.0f}")
 print("  merges:", cnt[56])
+
+ph = cnt[[64, 69, 65, 66, 67, 68]].astype(np.float64)
+nit = max(it.sum(), 1)
+print("per-iteration phase cycles (lane 0 of each warp): staging wait %.0f, take/stage records %.0f, CAS %.0f, read %.0f, decide+write %.0f, fence+release %.0f" % tuple(ph / nit))
