@@ -478,7 +478,7 @@ def run_gpu(args, world, rank, local):
             "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
             "dtype": "u32", "data": "synthetic",
             "config": {"workload": args.config, "key_range": R,
-                       "rebuild_every": "never" if args.rebuild_every < 0 else (args.rebuild_every or 2), "prefill": pre1 * world,
+                       "rebuild_every": "never" if args.rebuild_every < 0 else (args.rebuild_every or 4), "prefill": pre1 * world,
                        "batch_ops": B1 * world, "mix_ins_del_con": list(mix), "keys": dist,
                        "semantics": "combining (R26): mutations in input order, any batch" if combine_mode(args)
                        else "S1 snapshot, <=1 mutation per key (R1/R2)",
@@ -526,7 +526,7 @@ def main():
                     help="combining mode (R26) for any config (always on for *-raw configs)")
     ap.add_argument("--rebuild-every", type=int, default=0,
                     help="rebuild the upper levels after every k-th batch (R24); "
-                         "0 = library default (2), -1 = never (the paper's dynamics only)")
+                         "0 = library default (4), -1 = never (the paper's dynamics only)")
     ap.add_argument("--dist-backend", default="nccl", choices=["nccl", "gloo"],
                     help="gloo: exercise the multi-rank path with ranks sharing a GPU (no timing value)")
     ap.add_argument("--l2-window", action="store_true",

@@ -48,7 +48,7 @@ typedef enum gfsl_status {
   GFSL_ECORRUPT = 5  /* gfsl_validate found an invariant violation */
 } gfsl_status;
 
-#define GFSL_REBUILD_DEFAULT_PERIOD 2u
+#define GFSL_REBUILD_DEFAULT_PERIOD 4u
 #define GFSL_REBUILD_NEVER 0xFFFFFFFFu
 
 /* Largest batch (ops per gfsl_batch call): the op index shares a 32-bit word with three

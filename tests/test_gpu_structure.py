@@ -115,7 +115,7 @@ def test_serial_with_rebuild_byte_identical(N, every):
     """R24 on the GPU (rebuild kernels) equals Oracle-B's rebuild, entry for entry."""
     R = 3000 if N >= 16 else 500
     g = GFSL(R, chunk_entries=N, serial_updates=True, rebuild_every=every)
-    m = model_like(g, R, rebuild_every=every or 2)  # 0 = the library default period (2)
+    m = model_like(g, R, rebuild_every=every or 4)  # 0 = the library default period (4)
     w = Workload(R, R // 4, mix=(30, 30, 40), seed=SEED_BASE + 5 * N)
     for b in range(14):
         op, key, val, _ = w.make_batch(b)

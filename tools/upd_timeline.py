@@ -52,3 +52,4 @@ print("  merges:", cnt[56])
 ph = cnt[[64, 69, 65, 66, 67, 68]].astype(np.float64)
 nit = max(it.sum(), 1)
 print("per-iteration phase cycles (lane 0 of each warp): staging wait %.0f, take/stage records %.0f, CAS %.0f, read %.0f, decide+write %.0f, fence+release %.0f" % tuple(ph / nit))
+print("  of which: take a staged record %.0f, queue-item wait %.0f, stage_pair %.0f" % (cnt[70] / nit, (int(cnt[71]) & 0xFFFFFFFF) / nit, (int(cnt[71]) >> 32) / nit))
