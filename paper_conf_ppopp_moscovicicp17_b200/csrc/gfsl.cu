@@ -133,15 +133,16 @@ static void set_pdl(gfsl *h, cudaLaunchAttribute &a) {
 // What the search kernel writes: the records of the ops whose snapshot answer mutates
 // (numbered by ctl->n_mut, or by ctl->n_cand when the combine kernel picks the net ones).
 static SearchOut search_out(gfsl *h) {
+  const uint32_t full = h->cfg.serial_updates ? 1u : 0u;  // serial mode: traversals from the top
   if (h->cfg.combine)
-    return SearchOut{h->mut_rec, h->plan_path, h->mut_of, h->ctl->ccnt, h->region_cap, h->ck[0], h->cw[0]};
+    return SearchOut{h->mut_rec, h->plan_path, h->mut_of, h->ctl->ccnt, h->region_cap, h->ck[0], h->cw[0], full};
   return SearchOut{h->mut_rec, h->plan_path, h->cfg.serial_updates ? h->mut_of : nullptr,
-                   h->ctl->mcnt, h->region_cap, nullptr, nullptr};
+                   h->ctl->mcnt, h->region_cap, nullptr, nullptr, full};
 }
 // What the update kernel reads: the same records, or the net mutations of combining mode.
 static SearchOut update_in(gfsl *h) {
   if (h->cfg.combine)
-    return SearchOut{h->net_rec, h->net_path, h->mut_of, h->ctl->mcnt, h->region_cap, nullptr, nullptr};
+    return SearchOut{h->net_rec, h->net_path, h->mut_of, h->ctl->mcnt, h->region_cap, nullptr, nullptr, 0u};
   return search_out(h);
 }
 
@@ -467,8 +468,8 @@ extern "C" gfsl_t gfsl_create_ex(uint64_t key_range, uint64_t capacity, const gf
     while (dcap < (1u << 22) && (uint64_t)dcap < key_range + 1) dcap <<= 1;
     h->d.dir_cap = dcap;
     if ((e = cudaMalloc(&h->d.dir, (size_t)dcap * 4)) != cudaSuccess) return fail("cudaMalloc(dir)", e);
-    if ((e = cudaMalloc(&h->d.dir_hdr, 4 * 4)) != cudaSuccess) return fail("cudaMalloc(dir)", e);
-    cudaMemset(h->d.dir_hdr, 0, 4 * 4);
+    if ((e = cudaMalloc(&h->d.dir_hdr, 64 * 4)) != cudaSuccess) return fail("cudaMalloc(dir)", e);
+    cudaMemset(h->d.dir_hdr, 0, 64 * 4);
 #ifdef GFSL_DEBUG_TIMING
     if ((e = cudaMalloc(&h->d.debug_times, ((size_t)148 * 64 * 48 + 64) * 8)) != cudaSuccess) return fail("cudaMalloc", e);
     cudaMemset(h->d.debug_times, 0, ((size_t)148 * 64 * 48 + 64) * 8);
@@ -880,7 +881,7 @@ extern "C" gfsl_status gfsl_load(gfsl_t h, const gfsl_meta *meta, const uint64_t
   CK(cudaMemcpy(h->d.counter, meta->counters, 32 * 4, cudaMemcpyHostToDevice));
   uint32_t bump[2] = {meta->used_bottom, meta->used_upper};
   CK(cudaMemcpy(h->d.bump, bump, 8, cudaMemcpyHostToDevice));
-  CK(cudaMemset(h->d.dir_hdr, 0, 4 * 4));  // the directory describes the old structure
+  CK(cudaMemset(h->d.dir_hdr, 0, 64 * 4));  // the directory describes the old structure
   return GFSL_OK;
 }
 

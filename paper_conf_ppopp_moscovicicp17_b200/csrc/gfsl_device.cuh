@@ -60,9 +60,12 @@ struct DevState {
   uint32_t *fl;          // [0] free chunks in the current list, [1] taken, [2] buffer,
                          // [3..5] reclaim scratch
   unsigned long long *debug_times;  // GFSL_DEBUG_TIMING builds: per-team (start, end, ops)
-  // Level-1 directory (R27): dir[b] = the level-1 chunk holding the largest level-1 key
-  // <= (b << shift), written by each upper-level rebuild.  dir_hdr = {shift, valid,
-  // buckets}; valid = 0 until the first rebuild (and after gfsl_load).
+  // Directory (R27): dir[b] = how many level-1 keys of the last rebuild are <= (b << shift)
+  // (the rank r of the bucket's low key).  The rebuilt level l holds every F^(l-1)-th
+  // level-1 key F per chunk, so the chunk of level l that holds the largest key <= b << shift
+  // is chunk r / F^l of that level: chunk l-1 (the head) if 0, else dir_hdr[32 + l] + r / F^l - 1.
+  // dir_hdr = {shift, valid, buckets, F, ..., [32 + l] = base of level l}; valid = 0 until the
+  // first rebuild (and after gfsl_load).
   uint32_t *dir;
   uint32_t *dir_hdr;
   uint32_t dir_cap;      // entries allocated (a power of two)

@@ -190,10 +190,11 @@ __global__ void __launch_bounds__(256) rebuild_rank_kernel(const __grid_constant
   pdl_wait();
   if (!rb_active(b)) return;
   {
-    // R27: bucket q = keys [q << shift, (q+1) << shift); its entry is the level-1 chunk
-    // that holds the largest level-1 key <= q << shift.  Level-1 entry i >= 1 is the i-th
-    // marked min key, so that entry is number rank(q << shift), in chunk rank / F of the
-    // packed level 1 (rebuild_pack_kernel).  About one bucket per level-1 key.
+    // R27: bucket q = keys [q << shift, (q+1) << shift); its entry is r = rank(q << shift),
+    // the number of marked min keys (= level-1 entries >= 1) <= q << shift.  Level-1 entry
+    // r is then the largest level-1 key <= q << shift, in chunk r / F of the packed level 1,
+    // and level l's largest key <= q << shift is in its chunk r / F^l (rebuild_pack_kernel).
+    // About one bucket per level-1 key.
     const uint32_t n1 = b.n1[0];
     uint32_t target = 1024;
     while (target < 2u * n1 && target < d.dir_cap) target <<= 1;
@@ -202,15 +203,17 @@ __global__ void __launch_bounds__(256) rebuild_rank_kernel(const __grid_constant
     while (((uint64_t)d.key_max >> shift) + 1 > target) ++shift;
     const uint32_t buckets = (uint32_t)((uint64_t)d.key_max >> shift) + 1;
     const RbLevels *L = (const RbLevels *)b.levels;
-    const uint32_t base1 = L->base[1];
-    for (uint32_t q = blockIdx.x * blockDim.x + threadIdx.x; q < buckets; q += gridDim.x * blockDim.x) {
-      const uint32_t j = rb_rank_le(b, q << shift) / b.fill;
-      d.dir[q] = j == 0 ? 0u : base1 + j - 1;  // rb_chunk(L, 1, j)
-    }
-    if (blockIdx.x == 0 && threadIdx.x == 0) {
-      d.dir_hdr[0] = (uint32_t)shift;
-      d.dir_hdr[1] = 1u;
-      d.dir_hdr[2] = buckets;
+    for (uint32_t q = blockIdx.x * blockDim.x + threadIdx.x; q < buckets; q += gridDim.x * blockDim.x)
+      d.dir[q] = rb_rank_le(b, q << shift);
+    if (blockIdx.x == 0 && threadIdx.x < 32) {
+      const int l = threadIdx.x;
+      d.dir_hdr[32 + l] = (l >= 1 && l < N) ? L->base[l] : 0u;
+      if (l == 0) {
+        d.dir_hdr[0] = (uint32_t)shift;
+        d.dir_hdr[1] = 1u;
+        d.dir_hdr[2] = buckets;
+        d.dir_hdr[3] = b.fill;
+      }
     }
   }
   const uint32_t used = min(d.bump[0], d.cap_bottom);

@@ -74,6 +74,7 @@ struct SearchOut {
   uint32_t *comb_key;   // [n] or NULL (combining mode, R26): op i's sort key = internal key
                         // for a valid Insert/Delete, else all ones
   uint32_t *comb_w;     // [n]: op i | CW_* flags (the sort's payload)
+  uint32_t full_path;   // 1 = every Insert/Delete traverses from the top (serial mode)
 };
 
 // A record slot in the writing block's region (BatchCtl::mcnt).
@@ -104,6 +105,7 @@ search_kernel(DevState d, const BatchIn in, BatchCtl *__restrict__ ctl, SearchOu
   constexpr uint32_t FULL = 0xFFFFFFFFu;
 
   __shared__ uint32_t s_start, s_height, s_dir_shift;
+  __shared__ uint32_t s_dir_base[PLAN_LEVELS];  // base of each rebuilt level (R27)
   // the path of the team's current op (written by its lane 0 only), copied out compactly
   // at the end if the op mutates (about 1 op in 10)
   __shared__ __align__(16) uint32_t s_path[(256 / 32) * TPW][PLAN_LEVELS];
@@ -122,17 +124,26 @@ search_kernel(DevState d, const BatchIn in, BatchCtl *__restrict__ ctl, SearchOu
       s_dir_shift = (h >= 2 && d.dir_hdr[1]) ? d.dir_hdr[0] : 32u;
       if (blockIdx.x == 0) ctl->snap_height = h;
     }
+    if (lane < PLAN_LEVELS) s_dir_base[lane] = d.dir_hdr[32 + lane];
   }
   __syncthreads();
   const uint32_t start = s_start;
   const int height = (int)s_height;
   const uint32_t dir_shift = s_dir_shift;
   const bool use_dir = dir_shift < 32u;
-  // where a traversal starts: searchDown from the top (Alg 4.2 l.2-4), or -- for a
-  // Contains when the directory is valid -- at level 1, in the chunk the directory names
-  // for k's bucket (R27).  Insert/Delete always start at the top: searchSlow records the
-  // whole path (Alg 4.6).
-  auto dir_op = [&](uint32_t opw) { return use_dir && !(opw & (UPDATE_FLAG | INVALID_FLAG)); };
+  // where a traversal starts: searchDown from the top (Alg 4.2 l.2-4), or -- when the
+  // directory is valid -- at level 1, in the chunk of rank r / F that the directory names
+  // for k's bucket (R27).  An Insert/Delete entered there records its path at levels 1
+  // and 0 as it goes (searchSlow, Alg 4.6) and takes the levels above from the same rank
+  // (chunk r / F^l of level l: a valid start for findAndLockEnclosing); a Delete
+  // that finds k at level 1 starts over from the top, since its exact top level is needed.
+  // Serial mode (full_path) traverses every Insert/Delete from the top.
+  constexpr uint32_t F = N - 4;  // keys per rebuilt upper chunk (RebuildBufs::fill)
+  const bool dir_upd = use_dir && !so.full_path;
+  auto dir_op = [&](uint32_t opw) {
+    return use_dir && !(opw & INVALID_FLAG) && (dir_upd || !(opw & UPDATE_FLAG));
+  };
+  auto l1_chunk = [&](uint32_t r) { const uint32_t q = r / F; return q ? s_dir_base[1] + q - 1u : 0u; };
   const uint32_t n = in.n;
   uint8_t *__restrict__ res = in.res;
 
@@ -177,11 +188,13 @@ search_kernel(DevState d, const BatchIn in, BatchCtl *__restrict__ ctl, SearchOu
   RawOp nxt = load_raw(slot + total_teams);
   bool active = lane_live && slot < n;
   uint32_t k = cur_op.y;
-  uint32_t cur = dir_op(cur_op.x) ? __ldg(d.dir + (k >> dir_shift)) : start;
-  int level = dir_op(cur_op.x) ? 1 : height;
+  bool via_dir = dir_op(cur_op.x);
+  uint32_t cur_r = via_dir ? __ldg(d.dir + (k >> dir_shift)) : 0u;  // the op's directory rank
+  uint32_t cur = via_dir ? l1_chunk(cur_r) : start;
+  int level = via_dir ? 1 : height;
   // the next op's directory word is loaded one loop iteration after its raw op (so that
   // its key has arrived), and is ready when the op becomes current
-  uint32_t nxt_dir = start;
+  uint32_t nxt_dir = 0;
   bool pf_dir = use_dir;
   uint32_t bt = NULL_CHUNK, bt_c = NULL_CHUNK;       // prevKv, reduced
   int seen_top = 0;                                  // highest level where k was seen
@@ -192,7 +205,8 @@ search_kernel(DevState d, const BatchIn in, BatchCtl *__restrict__ ctl, SearchOu
     ChunkSlice<EPL> s;
     ld_slice_nc<EPL>(d.pool + (size_t)cur * N + t * EPL, s);  // idle teams re-read `cur`
     if (pf_dir) {
-      if (nxt.op == 0 && (uint64_t)nxt.key < in.key_range) nxt_dir = __ldg(d.dir + ((nxt.key + 1u) >> dir_shift));
+      if ((nxt.op == 0 || (dir_upd && nxt.op <= 2)) && (uint64_t)nxt.key < in.key_range)
+        nxt_dir = __ldg(d.dir + ((nxt.key + 1u) >> dir_shift));
       pf_dir = false;
     }
     if (COUNT && active) {
@@ -237,10 +251,12 @@ search_kernel(DevState d, const BatchIn in, BatchCtl *__restrict__ ctl, SearchOu
       const bool lat = (np & (F_ZOMBIE | F_LATERAL)) != 0;  // zombie (l.9-11) / lateral (l.15-18)
       const bool done = !lat && level == 0;                 // bottom enclosing chunk (Alg 4.4)
       const bool down = !lat && level > 0;                  // down step (l.19-23) / backtrack
-      // (l.25): only from a directory entry made stale by the batches since the last
-      // rebuild (R27: level-1 keys <= k deleted from that chunk); never from the top
-      const bool restart = down && !tb && bt == NULL_CHUNK;
       const bool upd = (cur_op.x & UPDATE_FLAG) != 0;
+      // restart (l.25): only from a directory entry made stale by the batches since the
+      // last rebuild (R27: level-1 keys <= k deleted from that chunk), never from the top;
+      // and on purpose when a Delete entered at level 1 finds k there (its exact top)
+      const bool redo = via_dir && down && level == 1 && tb && (dptr & F_EQUAL) && (cur_op.x & DELETE_FLAG);
+      const bool restart = (down && !tb && bt == NULL_CHUNK) || redo;
       const uint32_t here = cur;
       if (down && upd && t == 0 && level < PLAN_LEVELS)     // searchSlow's path (Alg 4.6 l.28-37)
         my_path[level] = tb ? cur : bt_c;
@@ -252,8 +268,10 @@ search_kernel(DevState d, const BatchIn in, BatchCtl *__restrict__ ctl, SearchOu
       cur = restart ? start : next_cur;
       level = restart ? height : level - (down ? 1 : 0);
       if (restart) {
-        ++restarts;
+        restarts += redo ? 0 : 1;
         seen_top = 0;
+        via_dir = false;
+        bt = bt_c = NULL_CHUNK;
       }
       if (done) {
         const bool te = tb != 0;
@@ -272,6 +290,14 @@ search_kernel(DevState d, const BatchIn in, BatchCtl *__restrict__ ctl, SearchOu
               const uint32_t w = opi | (cur_op.x & DELETE_FLAG);
               so.mut_rec[m] = make_uint4(w, k, here, (cur_op.x & DELETE_FLAG) ? seen_top : cur_val);
               my_path[0] = here;  // path[0] = the enclosing bottom chunk
+              if (via_dir) {      // levels >= 2 from the directory rank (R27)
+                uint32_t q = cur_r / F;
+#pragma unroll
+                for (int l = 2; l < PLAN_LEVELS; ++l) {
+                  q /= F;
+                  my_path[l] = q ? s_dir_base[l] + q - 1u : (uint32_t)(l - 1);
+                }
+              }
               const uint4 *src = reinterpret_cast<const uint4 *>(my_path);
               uint4 *dst = reinterpret_cast<uint4 *>(so.plan_path + (size_t)m * PLAN_LEVELS);
 #pragma unroll
@@ -293,8 +319,10 @@ search_kernel(DevState d, const BatchIn in, BatchCtl *__restrict__ ctl, SearchOu
         cur_val = load_val(slot, nxt);
         k = cur_op.y;
         nxt = load_raw(slot + total_teams);
-        cur = dir_op(cur_op.x) ? nxt_dir : start;
-        level = dir_op(cur_op.x) ? 1 : height;
+        via_dir = dir_op(cur_op.x);
+        cur_r = nxt_dir;
+        cur = via_dir ? l1_chunk(cur_r) : start;
+        level = via_dir ? 1 : height;
         pf_dir = use_dir;
         bt = bt_c = NULL_CHUNK;
         seen_top = 0;
