@@ -275,7 +275,14 @@ def run_gpu(args, world, rank, local):
 
     # weak scaling: each rank owns a shard of R1 keys and issues B1 ops per step
     R = R1 * world
-    if world > 1:
+    if world > 1 and args.exchange == "peer":
+        # fused exchange (NEXT-3): route kernels store/load straight through peer windows
+        from paper_conf_ppopp_moscovicicp17_b200.router import PeerShardedGFSL
+        g = PeerShardedGFSL(R, rank, world, max_slice=B1, capacity=R1, chunk_entries=N,
+                            contains_team=args.team)
+        lo = g.key_lo
+        prefill_gpu(g.local, R1, pre1, dev, key_lo=lo, seed=SEED_BASE + 1000 * rank)
+    elif world > 1:
         from paper_conf_ppopp_moscovicicp17_b200.router import ShardedGFSL
         g = ShardedGFSL(R, rank, world, capacity=R1, chunk_entries=N,
                         contains_team=args.team)
@@ -332,8 +339,10 @@ def run_gpu(args, world, rank, local):
     st_t = local_g.stats()
     n_mut = (st_t["mutations"] - mut0) / max(steps, 1)
     # our kernels launched inside the timed region (counted by libgfsl at enqueue), plus the
-    # route kernels of the multi-GPU path (3 plan + pack + unpack per step)
-    launches = int(st_t["kernel_launches"] - st0["kernel_launches"]) + (5 * steps if world > 1 else 0)
+    # route kernels of the multi-GPU path: NCCL exchange 3 plan + pack + unpack per step;
+    # peer exchange 3 plan + counts + push + 2 barriers + pull per step
+    route_k = (8 if args.exchange == "peer" else 5) if world > 1 else 0
+    launches = int(st_t["kernel_launches"] - st0["kernel_launches"]) + route_k * steps
     lib_launches = int(st_t["library_launches"] - st0["library_launches"])
     # per-kernel breakdown: CUDA events between the kernels of PROF extra batches (events
     # between kernels would defeat the programmatic dependent launch of the timed steps)
@@ -484,7 +493,9 @@ def run_gpu(args, world, rank, local):
                        else "S1 snapshot, <=1 mutation per key (R1/R2)",
                        "chunk_entries": N, "p_chunk": args.p_chunk, "contains_team": contains_team,
                        "l2": "flushed (256 MiB write) between timed steps",
-                       "parallelism": f"range-shard x{world}" if world > 1 else "1 GPU"},
+                       "parallelism": f"range-shard x{world}" if world > 1 else "1 GPU",
+                       "exchange": (("peer windows (CUDA IPC, fused route kernels)" if args.exchange == "peer"
+                                     else "NCCL all-to-all") if world > 1 else None)},
             "roofline": roofline,
             "roofline_kernels": {"search": roof_c, "update": roof_u},
             "search_gathers": gather,
@@ -529,6 +540,9 @@ def main():
                          "0 = library default (4), -1 = never (the paper's dynamics only)")
     ap.add_argument("--dist-backend", default="nccl", choices=["nccl", "gloo"],
                     help="gloo: exercise the multi-rank path with ranks sharing a GPU (no timing value)")
+    ap.add_argument("--exchange", default="peer", choices=["peer", "nccl"],
+                    help="N>1 exchange: peer = fused route kernels over CUDA-IPC windows "
+                         "(NEXT-3); nccl = torch.distributed all-to-all (baseline)")
     ap.add_argument("--l2-window", action="store_true",
                     help="pin the upper-level pool in L2 (access-policy window; ablation)")
     args = ap.parse_args()

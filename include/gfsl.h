@@ -45,7 +45,8 @@ typedef enum gfsl_status {
   GFSL_ENOMEM = 2,   /* device or host allocation failed */
   GFSL_EPOOL = 3,    /* chunk pool exhausted: sticky; the structure is undefined */
   GFSL_ECUDA = 4,    /* a CUDA runtime call failed: sticky */
-  GFSL_ECORRUPT = 5  /* gfsl_validate found an invariant violation */
+  GFSL_ECORRUPT = 5, /* gfsl_validate found an invariant violation */
+  GFSL_ETIMEOUT = 6  /* gfsl_xr_*: a peer did not reach an exchange barrier in time: sticky */
 } gfsl_status;
 
 #define GFSL_REBUILD_DEFAULT_PERIOD 4u
@@ -258,6 +259,68 @@ gfsl_status gfsl_route_pack(const uint32_t *perm, const uint8_t *op_types,
                             void *stream);
 gfsl_status gfsl_route_unpack(const uint32_t *perm, const uint8_t *recv_res, uint64_t n,
                               uint8_t *results, void *stream);
+
+/* ---- fused multi-GPU exchange over peer memory ----
+ * The same range partition as above, without NCCL on the data path: every rank owns one
+ * device WINDOW (receive arrays for world * max_slice ops, a double-buffered count matrix,
+ * barrier flags) that the peers map through CUDA IPC (one node, NVLink/NVSwitch).  The
+ * push kernel stores each routed op once, straight from the caller's arrays into its
+ * destination's window; the local shard runs gfsl_batch on its window; the pull kernel
+ * loads every result straight from the destination's window into the caller's order.
+ * Ranks synchronise with device-side barriers (release/acquire flags at system scope),
+ * each spin bounded by `timeout_ms`; an expired barrier makes the handle sticky-failed
+ * (GFSL_ETIMEOUT) and the batch's results GFSL_RESULT_INVALID.  The semantics are those of
+ * gfsl_batch on one map holding every shard (S1 per shard = S1 globally: a key lives on one
+ * shard and every op touches one key).
+ *
+ * gfsl_xr_create: this rank's window on the current device.  rank < world <= 64;
+ *   key_range as gfsl_create; max_slice = the largest n any rank will pass (the receive
+ *   arrays hold world * max_slice <= 2^32 - 1 ops); timeout_ms 0 = 60 s.  NULL on failure.
+ * gfsl_xr_export: writes the window's CUDA IPC handle (GFSL_XR_HANDLE_BYTES bytes, host).
+ * gfsl_xr_attach: maps peer `peer`'s window from its exported handle (another process).
+ * gfsl_xr_attach_local: uses the window of another handle of THIS process (one process
+ *   driving several shards, e.g. on one GPU; a handle on another device gets peer access).
+ *   Every rank must attach every peer before its first batch.
+ * A batch is collective over all ranks.  Each rank makes these calls in this order; one
+ * process driving several shards makes each call for every shard before the next call
+ * (the barriers are split into arrive and wait launches, so this order never waits on a
+ * launch that is not yet enqueued):
+ *   gfsl_xr_send(ops of this rank's slice, n <= max_slice, stream): route plan, count row
+ *     into every peer, arrive.  Enqueue only; the caller's arrays must stay valid until the
+ *     stream passes the batch.
+ *   gfsl_xr_push(stream): wait for all counts, push the ops into the peers' windows, arrive.
+ *   gfsl_xr_recv(..., stream): blocks the host until this rank's count exchange has
+ *     completed, enqueues the wait for everyone's pushes, and returns the received count and
+ *     the window's receive arrays (device pointers, owned by the handle, valid until
+ *     gfsl_xr_finish): op/key/val to feed the local shard, `results` for its answers.
+ *   (the caller enqueues gfsl_batch(local, op, key, val, results, n_recv, stream))
+ *   gfsl_xr_done(stream): arrive (this shard's results are written).
+ *   gfsl_xr_finish(results[n] of the slice, device, stream): wait, then the pull.
+ * gfsl_xr_batch: all of the above plus the local gfsl_batch, for one shard per process.
+ * gfsl_xr_status: GFSL_ETIMEOUT once any barrier of this handle has expired (synchronous).
+ * gfsl_xr_window: the window's base pointer and size (tests). */
+typedef struct gfsl_xr gfsl_xr;
+typedef gfsl_xr *gfsl_xr_t;
+#define GFSL_XR_HANDLE_BYTES 64
+gfsl_xr_t gfsl_xr_create(uint32_t rank, uint32_t world, uint64_t key_range, uint64_t max_slice,
+                         uint64_t timeout_ms);
+void gfsl_xr_destroy(gfsl_xr_t x);
+gfsl_status gfsl_xr_export(gfsl_xr_t x, void *handle);
+gfsl_status gfsl_xr_attach(gfsl_xr_t x, uint32_t peer, const void *handle);
+gfsl_status gfsl_xr_attach_local(gfsl_xr_t x, uint32_t peer, gfsl_xr_t other);
+gfsl_status gfsl_xr_send(gfsl_xr_t x, const uint8_t *op_types, const uint32_t *keys,
+                         const uint32_t *values, uint64_t n, void *stream);
+gfsl_status gfsl_xr_push(gfsl_xr_t x, void *stream);
+gfsl_status gfsl_xr_recv(gfsl_xr_t x, const uint8_t **op_types, const uint32_t **keys,
+                         const uint32_t **values, uint8_t **results, uint64_t *n_recv,
+                         void *stream);
+gfsl_status gfsl_xr_done(gfsl_xr_t x, void *stream);
+gfsl_status gfsl_xr_finish(gfsl_xr_t x, uint8_t *results, void *stream);
+gfsl_status gfsl_xr_batch(gfsl_xr_t x, gfsl_t local, const uint8_t *op_types,
+                          const uint32_t *keys, const uint32_t *values, uint8_t *results,
+                          uint64_t n, void *stream);
+gfsl_status gfsl_xr_status(gfsl_xr_t x);
+gfsl_status gfsl_xr_window(gfsl_xr_t x, void **base, uint64_t *bytes);
 
 /* ---- measurement: the roofline denominators of SURVEY 8(d) (B6) ----
  * gfsl_ubench: random aligned `block_bytes` (256 or 128) gathers over a fresh device buffer

@@ -14,7 +14,7 @@ HERE = os.path.dirname(os.path.abspath(__file__))
 ROOT = os.path.dirname(HERE)
 CSRC = os.path.join(HERE, "csrc")
 LIB = os.path.join(HERE, "libgfsl.so")
-SOURCES = ["gfsl.cu"]
+SOURCES = ["gfsl.cu", "gfsl_xroute.cu"]
 HEADERS = ["gfsl_device.cuh", "gfsl_search.cuh", "gfsl_update.cuh", "gfsl_ubench.cuh", "gfsl_rebuild.cuh", "gfsl_combine.cuh"]
 
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")

@@ -34,6 +34,7 @@ using namespace gfsl_dev;
 static thread_local std::string g_last_error = "no error";
 static void set_last_error(const std::string &s) { g_last_error = s; }
 extern "C" const char *gfsl_last_error(void) { return g_last_error.c_str(); }
+void gfsl_internal_set_error(const std::string &s) { set_last_error(s); }  // gfsl_xroute.cu
 
 #define CK(call)                                                                      \
   do {                                                                                \
@@ -1185,6 +1186,29 @@ __global__ void route_unpack_kernel(const uint32_t *perm, const uint8_t *rr, uin
     res[perm[j]] = rr[j];
 }
 
+// Route plan with a caller-provided workspace of gfsl_internal_route_ws_bytes() (used by
+// gfsl_xroute.cu, whose batches must not allocate: a stream-ordered allocation may wait on
+// another shard's stream, which can be spinning in an exchange barrier).
+size_t gfsl_internal_route_ws_bytes(uint64_t n, uint32_t world) {
+  return (size_t)((n + ROUTE_TILE - 1) / ROUTE_TILE) * world * 4;
+}
+gfsl_status gfsl_internal_route_plan(const uint8_t *op_types, const uint32_t *keys, uint64_t n,
+                                     uint64_t key_range, uint32_t world, uint64_t *counts,
+                                     uint32_t *perm, uint32_t *tile_counts, cudaStream_t s) {
+  if (n == 0) {
+    CK(cudaMemsetAsync(counts, 0, world * 8, s));
+    return GFSL_OK;
+  }
+  const uint64_t span = (key_range + world - 1) / world;
+  const uint32_t tiles = (uint32_t)((n + ROUTE_TILE - 1) / ROUTE_TILE);
+  route_hist_kernel<<<tiles, 256, 0, s>>>(op_types, keys, (uint32_t)n, key_range, span, world, tile_counts);
+  route_scan_kernel<<<1, 32, 0, s>>>(tile_counts, tiles, world, (unsigned long long *)counts);
+  route_scatter_kernel<<<tiles, 256, 0, s>>>(op_types, keys, (uint32_t)n, key_range, span, world,
+                                             tile_counts, perm);
+  CK(cudaGetLastError());
+  return GFSL_OK;
+}
+
 extern "C" gfsl_status gfsl_route_plan(const uint8_t *op_types, const uint32_t *keys, uint64_t n,
                                        uint64_t key_range, uint32_t world, uint64_t *counts,
                                        uint32_t *perm, void *stream) {
@@ -1197,17 +1221,12 @@ extern "C" gfsl_status gfsl_route_plan(const uint8_t *op_types, const uint32_t *
     CK(cudaMemsetAsync(counts, 0, world * 8, s));
     return GFSL_OK;
   }
-  const uint64_t span = (key_range + world - 1) / world;
   const uint32_t tiles = (uint32_t)((n + ROUTE_TILE - 1) / ROUTE_TILE);
   uint32_t *tile_counts = nullptr;
   CK(cudaMallocAsync(&tile_counts, (size_t)tiles * world * 4, s));
-  route_hist_kernel<<<tiles, 256, 0, s>>>(op_types, keys, (uint32_t)n, key_range, span, world, tile_counts);
-  route_scan_kernel<<<1, 32, 0, s>>>(tile_counts, tiles, world, (unsigned long long *)counts);
-  route_scatter_kernel<<<tiles, 256, 0, s>>>(op_types, keys, (uint32_t)n, key_range, span, world,
-                                             tile_counts, perm);
+  gfsl_status st = gfsl_internal_route_plan(op_types, keys, n, key_range, world, counts, perm, tile_counts, s);
   CK(cudaFreeAsync(tile_counts, s));
-  CK(cudaGetLastError());
-  return GFSL_OK;
+  return st;
 }
 
 extern "C" gfsl_status gfsl_route_pack(const uint32_t *perm, const uint8_t *op_types,

@@ -20,11 +20,12 @@ _HERE = os.path.dirname(os.path.abspath(__file__))
 # GFSL_LIB: an alternative build of the same library (tools/ experiments only)
 LIB_PATH = os.environ.get("GFSL_LIB") or os.path.join(_HERE, "libgfsl.so")
 
-GFSL_OK, GFSL_EINVAL, GFSL_ENOMEM, GFSL_EPOOL, GFSL_ECUDA, GFSL_ECORRUPT = range(6)
+GFSL_OK, GFSL_EINVAL, GFSL_ENOMEM, GFSL_EPOOL, GFSL_ECUDA, GFSL_ECORRUPT, GFSL_ETIMEOUT = range(7)
 CONTAINS, INSERT, DELETE = 0, 1, 2
 RES_FALSE, RES_TRUE, RES_INVALID = 0, 1, 0xFF
 REBUILD_DEFAULT, REBUILD_NEVER = 0, 0xFFFFFFFF  # rebuild_every: library default period / never
-STATUS_NAMES = ["OK", "EINVAL", "ENOMEM", "EPOOL", "ECUDA", "ECORRUPT"]
+STATUS_NAMES = ["OK", "EINVAL", "ENOMEM", "EPOOL", "ECUDA", "ECORRUPT", "ETIMEOUT"]
+XR_HANDLE_BYTES = 64
 
 
 class gfsl_config(ctypes.Structure):
@@ -72,6 +73,10 @@ EXPORTS = [
     "gfsl_validate", "gfsl_last_error", "gfsl_get_stats", "gfsl_dump", "gfsl_load",
     "gfsl_route_plan", "gfsl_route_pack", "gfsl_route_unpack", "gfsl_phase_times",
     "gfsl_configure", "gfsl_ubench",
+    "gfsl_xr_create", "gfsl_xr_destroy", "gfsl_xr_export", "gfsl_xr_attach",
+    "gfsl_xr_attach_local", "gfsl_xr_send", "gfsl_xr_push", "gfsl_xr_recv", "gfsl_xr_done",
+    "gfsl_xr_finish", "gfsl_xr_batch",
+    "gfsl_xr_status", "gfsl_xr_window",
 ]
 
 _lib = None
@@ -123,6 +128,33 @@ def load_library(path: str = LIB_PATH):
     lib.gfsl_route_pack.argtypes = [vp, vp, vp, vp, u64, vp, vp, vp, vp]
     lib.gfsl_route_unpack.restype = i32
     lib.gfsl_route_unpack.argtypes = [vp, vp, u64, vp, vp]
+    lib.gfsl_xr_create.restype = vp
+    lib.gfsl_xr_create.argtypes = [u32, u32, u64, u64, u64]
+    lib.gfsl_xr_destroy.restype = None
+    lib.gfsl_xr_destroy.argtypes = [vp]
+    lib.gfsl_xr_export.restype = i32
+    lib.gfsl_xr_export.argtypes = [vp, vp]
+    lib.gfsl_xr_attach.restype = i32
+    lib.gfsl_xr_attach.argtypes = [vp, u32, vp]
+    lib.gfsl_xr_attach_local.restype = i32
+    lib.gfsl_xr_attach_local.argtypes = [vp, u32, vp]
+    lib.gfsl_xr_send.restype = i32
+    lib.gfsl_xr_send.argtypes = [vp, vp, vp, vp, u64, vp]
+    lib.gfsl_xr_push.restype = i32
+    lib.gfsl_xr_push.argtypes = [vp, vp]
+    lib.gfsl_xr_recv.restype = i32
+    lib.gfsl_xr_recv.argtypes = [vp, ctypes.POINTER(vp), ctypes.POINTER(vp), ctypes.POINTER(vp),
+                                 ctypes.POINTER(vp), ctypes.POINTER(u64), vp]
+    lib.gfsl_xr_done.restype = i32
+    lib.gfsl_xr_done.argtypes = [vp, vp]
+    lib.gfsl_xr_finish.restype = i32
+    lib.gfsl_xr_finish.argtypes = [vp, vp, vp]
+    lib.gfsl_xr_batch.restype = i32
+    lib.gfsl_xr_batch.argtypes = [vp, vp, vp, vp, vp, vp, u64, vp]
+    lib.gfsl_xr_status.restype = i32
+    lib.gfsl_xr_status.argtypes = [vp]
+    lib.gfsl_xr_window.restype = i32
+    lib.gfsl_xr_window.argtypes = [vp, ctypes.POINTER(vp), ctypes.POINTER(u64)]
     _lib = lib
     return lib
 
@@ -215,6 +247,12 @@ class GFSL:
         _check(self.lib.gfsl_batch(self.h, _ptr(op), _ptr(key), _ptr(val), _ptr(out), n,
                                    _stream(stream)), "gfsl_batch")
         return out
+
+    def batch_ptr(self, op_ptr: int, key_ptr: int, val_ptr: int | None, res_ptr: int, n: int,
+                  stream=None):
+        """Asynchronous batch on raw device pointers (e.g. an exchange window's arrays)."""
+        _check(self.lib.gfsl_batch(self.h, op_ptr, key_ptr, val_ptr, res_ptr, n, _stream(stream)),
+               "gfsl_batch")
 
     def batch_host(self, op, key, val=None, out=None, stream=None):
         """Synchronous batch on HOST tensors (the end-to-end entry point)."""
@@ -343,3 +381,74 @@ def ubench(block_bytes: int = 256, buffer_bytes: int = 16 << 30):
     g, c = ctypes.c_double(), ctypes.c_double()
     _check(lib.gfsl_ubench(block_bytes, buffer_bytes, ctypes.byref(g), ctypes.byref(c)), "gfsl_ubench")
     return g.value, c.value
+
+
+# ---- fused exchange over peer memory (gfsl_xr_*) ----------------
+class XRoute:
+    """One rank's exchange window (C handle ``gfsl_xr_t``) on the current CUDA device."""
+
+    def __init__(self, rank: int, world: int, key_range: int, max_slice: int,
+                 timeout_ms: int = 0):
+        self.lib = load_library()
+        self.rank, self.world, self.max_slice = int(rank), int(world), int(max_slice)
+        self.h = self.lib.gfsl_xr_create(self.rank, self.world, int(key_range),
+                                         self.max_slice, int(timeout_ms))
+        if not self.h:
+            raise RuntimeError("gfsl_xr_create failed: " + self.lib.gfsl_last_error().decode())
+
+    def close(self):
+        if getattr(self, "h", None):
+            self.lib.gfsl_xr_destroy(self.h)
+            self.h = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+    def export(self) -> bytes:
+        buf = (ctypes.c_char * XR_HANDLE_BYTES)()
+        _check(self.lib.gfsl_xr_export(self.h, buf), "gfsl_xr_export")
+        return bytes(buf)
+
+    def attach(self, peer: int, handle: bytes):
+        buf = (ctypes.c_char * XR_HANDLE_BYTES).from_buffer_copy(handle)
+        _check(self.lib.gfsl_xr_attach(self.h, peer, buf), "gfsl_xr_attach")
+
+    def attach_local(self, peer: int, other: "XRoute"):
+        _check(self.lib.gfsl_xr_attach_local(self.h, peer, other.h), "gfsl_xr_attach_local")
+
+    def send(self, op, key, val=None, stream=None):
+        _check(self.lib.gfsl_xr_send(self.h, _ptr(op), _ptr(key), _ptr(val), op.numel(),
+                                     _stream(stream)), "gfsl_xr_send")
+
+    def push(self, stream=None):
+        _check(self.lib.gfsl_xr_push(self.h, _stream(stream)), "gfsl_xr_push")
+
+    def recv(self, stream=None):
+        """(n_recv, op_ptr, key_ptr, val_ptr, res_ptr): the window's receive arrays."""
+        o, k, v, r = ctypes.c_void_p(), ctypes.c_void_p(), ctypes.c_void_p(), ctypes.c_void_p()
+        m = ctypes.c_uint64()
+        _check(self.lib.gfsl_xr_recv(self.h, ctypes.byref(o), ctypes.byref(k), ctypes.byref(v),
+                                     ctypes.byref(r), ctypes.byref(m), _stream(stream)),
+               "gfsl_xr_recv")
+        return m.value, o.value, k.value, v.value, r.value
+
+    def done(self, stream=None):
+        _check(self.lib.gfsl_xr_done(self.h, _stream(stream)), "gfsl_xr_done")
+
+    def finish(self, out, stream=None):
+        _check(self.lib.gfsl_xr_finish(self.h, _ptr(out), _stream(stream)), "gfsl_xr_finish")
+        return out
+
+    def batch(self, local: "GFSL", op, key, val=None, out=None, stream=None):
+        import torch
+        if out is None:
+            out = torch.empty(op.numel(), dtype=torch.uint8, device=op.device)
+        _check(self.lib.gfsl_xr_batch(self.h, local.h, _ptr(op), _ptr(key), _ptr(val), _ptr(out),
+                                      op.numel(), _stream(stream)), "gfsl_xr_batch")
+        return out
+
+    def status(self) -> int:
+        return self.lib.gfsl_xr_status(self.h)

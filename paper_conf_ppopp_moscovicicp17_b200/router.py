@@ -100,3 +100,93 @@ class ShardedGFSL:
         self._a2a(back, rr, send_split, recv_split)
         self.last_counts = (send_split, recv_split)
         return self.k.unpack(perm, back, n)
+
+
+class PeerShardedGFSL:
+    """Range-partitioned GFSL with the fused peer-memory exchange (gfsl_xr_*; SURVEY 8(f)
+    NEXT-3): one rank per process and GPU.  Same partition and the same collective
+    ``batch`` contract as ShardedGFSL, but no NCCL on the data path: the route kernels
+    store every op straight into its destination's window and load every result straight
+    back (CUDA IPC mappings over NVLink).  torch.distributed only exchanges the windows'
+    IPC handles once, at construction."""
+
+    def __init__(self, key_range: int, rank: int, world: int, max_slice: int, capacity: int = 0,
+                 group=None, timeout_ms: int = 0, **gfsl_kw):
+        self.key_range = int(key_range)
+        self.rank, self.world, self.group = rank, world, group
+        self.key_lo, self.key_hi, self.span = shard_bounds(self.key_range, world, rank)
+        cap = capacity if capacity else max(1, self.key_hi - self.key_lo)
+        self.local = G.GFSL(self.key_range, capacity=cap, **gfsl_kw)
+        self.xr = G.XRoute(rank, world, self.key_range, max_slice, timeout_ms)
+        handles = [None] * world
+        dist.all_gather_object(handles, self.xr.export(), group=group)
+        for p in range(world):
+            if p != rank:
+                self.xr.attach(p, handles[p])
+        dist.barrier(group=group)
+
+    def batch(self, op, key, val=None, out=None, stream=None):
+        """Collective.  op uint8[n], key 32-bit[n], val 32-bit[n] (this rank's slice);
+        returns uint8[n] results in the slice's order."""
+        return self.xr.batch(self.local, op, key, val, out=out, stream=stream)
+
+
+class LoopbackShards:
+    """`world` shards driven by ONE process on the current device, exchanging through the
+    same windows and kernels as PeerShardedGFSL (attach_local instead of IPC); each shard
+    runs on its own stream and every phase is enqueued for all shards before the next
+    (split-phase barriers), so the device barriers between the shards are real and never
+    wait on a launch that is not yet enqueued.  Used to
+    test the exchange on one GPU; ``batch`` takes a GLOBAL batch and splits it into
+    `world` contiguous slices, like `world` ranks would hold it."""
+
+    def __init__(self, key_range: int, world: int, max_slice: int, capacity: int = 0,
+                 timeout_ms: int = 20000, **gfsl_kw):
+        self.key_range, self.world = int(key_range), int(world)
+        self.bounds = [shard_bounds(self.key_range, world, r) for r in range(world)]
+        self.local = []
+        for lo, hi, _ in self.bounds:
+            cap = capacity if capacity else max(1, hi - lo)
+            self.local.append(G.GFSL(self.key_range, capacity=cap, **gfsl_kw))
+        self.xr = [G.XRoute(r, world, self.key_range, max_slice, timeout_ms) for r in range(world)]
+        for r in range(world):
+            for p in range(world):
+                if p != r:
+                    self.xr[r].attach_local(p, self.xr[p])
+        self.streams = [torch.cuda.Stream() for _ in range(world)]
+
+    def slices(self, n: int):
+        q, rem = divmod(n, self.world)
+        out, a = [], 0
+        for r in range(self.world):
+            b = a + q + (1 if r < rem else 0)
+            out.append((a, b))
+            a = b
+        return out
+
+    def batch(self, op, key, val=None):
+        n = op.numel()
+        if val is None:
+            val = torch.zeros_like(key)
+        cur = torch.cuda.current_stream()
+        sl = self.slices(n)
+        out = torch.empty(n, dtype=torch.uint8, device=op.device)
+        for s in self.streams:
+            s.wait_stream(cur)
+        for r, (a, b) in enumerate(sl):
+            self.xr[r].send(op[a:b], key[a:b], val[a:b], stream=self.streams[r])
+        for r in range(self.world):
+            self.xr[r].push(stream=self.streams[r])
+        recv = []
+        for r in range(self.world):
+            recv.append(self.xr[r].recv(stream=self.streams[r]))
+            m, o, k, v, res = recv[-1]
+            if m:
+                self.local[r].batch_ptr(o, k, v, res, m, stream=self.streams[r])
+            self.xr[r].done(stream=self.streams[r])
+        for r, (a, b) in enumerate(sl):
+            self.xr[r].finish(out[a:b], stream=self.streams[r])
+        for s in self.streams:
+            cur.wait_stream(s)
+        self.last_recv = [x[0] for x in recv]
+        return out

@@ -1,5 +1,5 @@
 """bench.py end to end on the GPU: the 1-GPU JSON line carries the contract's keys, and
-the N>1 path (router + all-to-all exchange) runs as 2 ranks sharing one GPU over gloo."""
+the N>1 path (router + NCCL-style all-to-all exchange, or the fused peer-window exchange) runs as 2 ranks sharing one GPU over gloo."""
 import json
 import os
 import subprocess
@@ -27,8 +27,10 @@ def test_bench_single_gpu_line():
     assert d["value"] > 0 and d["roofline"]["peak"] > 0 and d["cpu_baseline"]["kind"] == "oracle"
 
 
-def test_bench_two_ranks_gloo():
+@pytest.mark.parametrize("exchange,port", [("nccl", 29533), ("peer", 29534)])
+def test_bench_two_ranks_gloo(exchange, port):
     d = run([sys.executable, "-m", "torch.distributed.run", "--nnodes=1", "--nproc-per-node", "2",
-             "--master-addr", "127.0.0.1", "--master-port", "29533", "bench.py", "--gpus", "2",
-             "--config", "C1", "--steps", "3", "--dist-backend", "gloo", "--validate", "--no-ubench"])
+             "--master-addr", "127.0.0.1", "--master-port", str(port), "bench.py", "--gpus", "2",
+             "--config", "C1", "--steps", "3", "--dist-backend", "gloo", "--validate", "--no-ubench",
+             "--exchange", exchange])
     assert d["n_gpus"] == 2 and d["value"] > 0 and d["validate"]["violations"] == 0
