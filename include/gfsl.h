@@ -49,7 +49,13 @@ typedef enum gfsl_status {
   GFSL_ETIMEOUT = 6  /* gfsl_xr_*: a peer did not reach an exchange barrier in time: sticky */
 } gfsl_status;
 
-#define GFSL_REBUILD_DEFAULT_PERIOD 4u
+/* Default upper-level rebuild policy (rebuild_every = 0; R29): rebuild after the
+ * batch at which the ops submitted since the last rebuild reach GFSL_REBUILD_DEFAULT_WEAR x
+ * L, L = min(capacity, ops submitted up to the last rebuild) -- an upper bound on the live
+ * keys, so a structure growing from empty is rebuilt at geometrically spaced sizes.  In
+ * steady state with the paper's [10,10,80] mix at half fill this is about one mutation per
+ * live key (every 4 batches at C1-C3, every 20 at C5). */
+#define GFSL_REBUILD_DEFAULT_WEAR 2.5
 #define GFSL_REBUILD_NEVER 0xFFFFFFFFu
 
 /* Largest batch (ops per gfsl_batch call): the op index shares a 32-bit word with three
@@ -82,8 +88,9 @@ typedef struct gfsl_config {
                                dependent launch (ablation) */
   uint32_t rebuild_every;   /* after every k-th batch, rebuild the levels >= 1 from level 0
                                (R24: "compact the structure between kernel
-                               launches").  0 = GFSL_REBUILD_DEFAULT_PERIOD;
-                               GFSL_REBUILD_NEVER = the paper's structure dynamics only */
+                               launches").  0 = the default wear policy
+                               (GFSL_REBUILD_DEFAULT_WEAR, R29); GFSL_REBUILD_NEVER = the
+                               paper's structure dynamics only */
   uint32_t combine;         /* 1 = combining mode (R26): exact
                                for ANY batch, with no <=1-mutation-per-key contract.  The
                                Contains of a batch still see the map before the batch (S1);
@@ -189,6 +196,15 @@ typedef struct gfsl_report {
  * order and sets *count to the number of live keys.  rep and count may be NULL.
  * Returns GFSL_OK, GFSL_ECORRUPT (rep->violations says which), or an error.
  */
+/*
+ * Rebuild the upper levels now (R24: "compact the structure between kernel
+ * launches"; with the zombie reclamation of R25 and the level-1 directory of R27), e.g.
+ * after a bulk load.  A no-op if no batch mutated the structure since the last rebuild.
+ * Asynchronous on `stream`, ordered after the handle's previous batch; restarts the default
+ * policy's count.  Returns a sticky error of an earlier batch, if any.
+ */
+gfsl_status gfsl_rebuild(gfsl_t h, void *stream);
+
 gfsl_status gfsl_validate(gfsl_t h, gfsl_report *rep, uint32_t *keys_out,
                           uint32_t *vals_out, uint64_t cap, uint64_t *count);
 

@@ -58,11 +58,16 @@ def raise_draw(rkey: int, level: int) -> int:
 
 class GFSLModel:
     def __init__(self, N: int, key_range: int, cap_bottom: int, cap_upper: int,
-                 rebuild_every: int = 0, p_chunk_q32: int = 0):
+                 rebuild_every: int = 0, p_chunk_q32: int = 0, rebuild_capacity: int = 0):
         assert N >= 6
         # p_chunk as a 32-bit fraction; 0 = p_chunk = 1 (R16)
         self.p_chunk_q32 = p_chunk_q32
         self.rebuild_every = rebuild_every
+        # R29, used if rebuild_every = 0 and rebuild_capacity > 0: rebuild after
+        # the batch at which the ops since the last rebuild reach 2.5 x min(capacity, ops
+        # submitted up to the last rebuild)
+        self.rebuild_capacity = rebuild_capacity
+        self.ops_total = self.ops_since = self.ops_at_rebuild = 0
         self.batches = 0
         self.dirty = False
         self.free, self.free_taken = [], 0  # R25 free list of reclaimed level-0 chunks
@@ -488,7 +493,16 @@ class GFSLModel:
             self.upkeep()
         if plans:
             self.dirty = True  # a mutating batch since the last rebuild
-        if n and self.rebuild_every and (self.batches + 1) % self.rebuild_every == 0 and self.dirty:
+        due = False
+        if n and self.rebuild_every:
+            due = (self.batches + 1) % self.rebuild_every == 0
+        elif n and self.rebuild_capacity:
+            self.ops_since += n
+            due = 2 * self.ops_since >= 5 * min(self.rebuild_capacity, self.ops_at_rebuild)
+            if due:
+                self.ops_since, self.ops_at_rebuild = 0, self.ops_total + n
+        self.ops_total += n
+        if due and self.dirty:
             self.rebuild()
             self.reclaim()
             self.dirty = False
@@ -504,6 +518,15 @@ class GFSLModel:
             self.pool[c] = [EMPTY] * (self.N - 1) + [HELD]
         self.free = self.free[self.free_taken:] + zombies
         self.free_taken = 0
+
+    def rebuild_now(self):
+        """gfsl_rebuild (R29): rebuild now if a batch mutated the structure since the last
+        rebuild; the default policy counts again from here."""
+        if self.dirty:
+            self.rebuild()
+            self.reclaim()
+            self.dirty = False
+        self.ops_since, self.ops_at_rebuild = 0, self.ops_total
 
     def rebuild(self):
         """R24: re-derive levels >= 1 from level 0 between batches ("compact the

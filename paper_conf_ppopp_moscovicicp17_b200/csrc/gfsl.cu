@@ -2,7 +2,7 @@
 //
 // A batch is enqueued as (DESIGN.md §Batch pipeline):
 //   memset(ctl) -> search_kernel (intake + B1, a2/a3) -> update_kernel (B2, a4/a5)
-//   -> upkeep (-> rebuild every `rebuild_every` batches)
+//   -> upkeep (-> upper-level rebuild, R24 / R29)
 // with no host synchronization.  The library owns the chunk pool, the head
 // array and per-level counters, the bump counters and the sticky error word; the
 // caller owns the op / key / value / result arrays.
@@ -70,6 +70,9 @@ struct gfsl {
   cudaStream_t copy_stream = nullptr;
   cudaEvent_t ev_in[2] = {nullptr, nullptr}, ev_used[2] = {nullptr, nullptr};
   uint64_t batches = 0, ops = 0;
+  uint64_t capacity = 0;           // max live keys (gfsl_create)
+  uint64_t ops_since_rebuild = 0;  // default rebuild policy (R29)
+  uint64_t ops_at_rebuild = 0;     // h->ops after the batch of the last rebuild
   uint64_t launches = 0, lib_launches = 0;  // our kernels / CUB's (combining sort) enqueued by batches
   std::vector<std::array<cudaEvent_t, 5>> phase_ev;  // profile_phases
   // L2 persistence for the upper pool (the search kernel's access-policy window)
@@ -205,6 +208,45 @@ static bool dispatch_contains(gfsl *h, const BatchIn &in, cudaStream_t s) {
   return false;
 }
 
+// R24 (+ R25 reclamation, R27 directory): the upper-level rebuild sequence.  Its first
+// kernel makes it a no-op unless a batch mutated the structure since the last one.
+template <int N>
+static void launch_rebuild(gfsl *h, cudaStream_t s) {
+  cudaLaunchConfig_t lc{};
+  cudaLaunchAttribute attr[1];
+  set_pdl(h, attr[0]);
+  lc.attrs = attr;
+  lc.numAttrs = 1;
+  lc.stream = s;
+  const RebuildBufs &b = h->rb;
+  h->launches += 9;
+  lc.gridDim = dim3(1);
+  lc.blockDim = dim3(32);
+  cudaLaunchKernelEx(&lc, rebuild_begin_kernel, b);
+  lc.blockDim = dim3(256);
+  lc.gridDim = dim3(h->sms * 4);
+  cudaLaunchKernelEx(&lc, rebuild_mark_kernel<N>, h->d, b);
+  lc.gridDim = dim3(b.blocks);
+  lc.blockDim = dim3(1024);
+  cudaLaunchKernelEx(&lc, rebuild_scan_kernel, b);
+  lc.gridDim = dim3(1);
+  cudaLaunchKernelEx(&lc, rebuild_scan_top_kernel<N>, b);
+  lc.blockDim = dim3(256);
+  lc.gridDim = dim3(h->sms * 4);
+  cudaLaunchKernelEx(&lc, rebuild_rank_kernel<N>, h->d, b);
+  lc.gridDim = dim3(h->sms * 8);
+  cudaLaunchKernelEx(&lc, rebuild_pack_kernel<N>, h->d, b);
+  // R25: reclaim the (now unreachable) zombie level-0 chunks (+ the bitmap clear)
+  lc.gridDim = dim3(h->sms * 4);
+  cudaLaunchKernelEx(&lc, reclaim_count_kernel<N>, h->d, b, h->rc_tiles);
+  lc.gridDim = dim3(1);
+  lc.blockDim = dim3(1024);
+  cudaLaunchKernelEx(&lc, reclaim_scan_kernel, h->d, b, h->rc_tiles);
+  lc.gridDim = dim3(h->sms * 4);
+  lc.blockDim = dim3(256);
+  cudaLaunchKernelEx(&lc, reclaim_write_kernel<N>, h->d, b, (const uint32_t *)h->rc_tiles);
+}
+
 template <int N>
 static void launch_update(gfsl *h, const BatchIn &in, cudaStream_t s, cudaEvent_t after_update) {
   cudaLaunchConfig_t lc{};
@@ -227,36 +269,23 @@ static void launch_update(gfsl *h, const BatchIn &in, cudaStream_t s, cudaEvent_
   if (after_update) cudaEventRecord(after_update, s);
   lc.gridDim = dim3(h->sms * 4);
   cudaLaunchKernelEx(&lc, upkeep_kernel<N>, h->d);
-  // R24: rebuild the upper levels from level 0 after every `rebuild_every`-th batch
-  const uint32_t every = h->cfg.rebuild_every == 0 ? GFSL_REBUILD_DEFAULT_PERIOD : h->cfg.rebuild_every;
-  if (every != GFSL_REBUILD_NEVER && (h->batches + 1) % every == 0) {
-    const RebuildBufs &b = h->rb;
-    h->launches += 9;
-    lc.gridDim = dim3(1);
-    lc.blockDim = dim3(32);
-    cudaLaunchKernelEx(&lc, rebuild_begin_kernel, b);
-    lc.blockDim = dim3(256);
-    lc.gridDim = dim3(h->sms * 4);
-    cudaLaunchKernelEx(&lc, rebuild_mark_kernel<N>, h->d, b);
-    lc.gridDim = dim3(b.blocks);
-    lc.blockDim = dim3(1024);
-    cudaLaunchKernelEx(&lc, rebuild_scan_kernel, b);
-    lc.gridDim = dim3(1);
-    cudaLaunchKernelEx(&lc, rebuild_scan_top_kernel<N>, b);
-    lc.blockDim = dim3(256);
-    lc.gridDim = dim3(h->sms * 4);
-    cudaLaunchKernelEx(&lc, rebuild_rank_kernel<N>, h->d, b);
-    lc.gridDim = dim3(h->sms * 8);
-    cudaLaunchKernelEx(&lc, rebuild_pack_kernel<N>, h->d, b);
-    // R25: reclaim the (now unreachable) zombie level-0 chunks (+ the bitmap clear)
-    lc.gridDim = dim3(h->sms * 4);
-    cudaLaunchKernelEx(&lc, reclaim_count_kernel<N>, h->d, b, h->rc_tiles);
-    lc.gridDim = dim3(1);
-    lc.blockDim = dim3(1024);
-    cudaLaunchKernelEx(&lc, reclaim_scan_kernel, h->d, b, h->rc_tiles);
-    lc.gridDim = dim3(h->sms * 4);
-    lc.blockDim = dim3(256);
-    cudaLaunchKernelEx(&lc, reclaim_write_kernel<N>, h->d, b, (const uint32_t *)h->rc_tiles);
+  // R24 / R29: rebuild the upper levels from level 0 -- by default after the batch at
+  // which the ops since the last rebuild reach GFSL_REBUILD_DEFAULT_WEAR x L, where L =
+  // min(capacity, ops ever submitted up to the last rebuild) bounds the live keys from
+  // above (so a structure growing from empty is rebuilt at geometrically spaced sizes);
+  // else after every `rebuild_every`-th batch
+  bool rebuild;
+  if (h->cfg.rebuild_every == 0) {
+    h->ops_since_rebuild += in.n;
+    const uint64_t L = std::min(h->capacity, h->ops_at_rebuild);
+    rebuild = 2 * h->ops_since_rebuild >= (uint64_t)(2 * GFSL_REBUILD_DEFAULT_WEAR) * L;
+  } else {
+    rebuild = h->cfg.rebuild_every != GFSL_REBUILD_NEVER && (h->batches + 1) % h->cfg.rebuild_every == 0;
+  }
+  if (rebuild) {
+    h->ops_since_rebuild = 0;
+    h->ops_at_rebuild = h->ops + in.n;
+    launch_rebuild<N>(h, s);
   }
 }
 
@@ -370,6 +399,7 @@ static void free_all(gfsl *h) {
   cudaFree(h->vw);
   cudaFree(h->cub_tmp);
   cudaFree(h->d.freelist);
+  cudaFree(h->d.zbits);
   cudaFree(h->d.fl);
   cudaFree(h->d.dir);
   cudaFree(h->d.dir_hdr);
@@ -405,6 +435,7 @@ extern "C" gfsl_t gfsl_create_ex(uint64_t key_range, uint64_t capacity, const gf
   h->team = cfg.contains_team;
   h->cfg = cfg;
   h->key_range = key_range;
+  h->capacity = capacity;
   auto fail = [&](const char *what, cudaError_t e) -> gfsl_t {
     set_last_error(std::string(what) + ": " + cudaGetErrorString(e));
     free_all(h);
@@ -471,6 +502,10 @@ extern "C" gfsl_t gfsl_create_ex(uint64_t key_range, uint64_t capacity, const gf
     if ((e = cudaMalloc(&h->d.dir, (size_t)dcap * 4)) != cudaSuccess) return fail("cudaMalloc(dir)", e);
     if ((e = cudaMalloc(&h->d.dir_hdr, 64 * 4)) != cudaSuccess) return fail("cudaMalloc(dir)", e);
     cudaMemset(h->d.dir_hdr, 0, 64 * 4);
+    // R30: zombie marks, two bitmaps over every chunk index
+    h->d.zwords = (uint32_t)(((uint64_t)h->d.cap_upper + h->d.cap_bottom + 31) / 32);
+    if ((e = cudaMalloc(&h->d.zbits, (size_t)h->d.zwords * 8)) != cudaSuccess) return fail("cudaMalloc(zbits)", e);
+    cudaMemset(h->d.zbits, 0, (size_t)h->d.zwords * 8);
 #ifdef GFSL_DEBUG_TIMING
     if ((e = cudaMalloc(&h->d.debug_times, ((size_t)148 * 64 * 48 + 64) * 8)) != cudaSuccess) return fail("cudaMalloc", e);
     cudaMemset(h->d.debug_times, 0, ((size_t)148 * 64 * 48 + 64) * 8);
@@ -635,6 +670,7 @@ static gfsl_status enqueue_combine(gfsl *h, const BatchIn &in, cudaStream_t s) {
 static gfsl_status enqueue_batch(gfsl *h, const uint8_t *ops, const uint32_t *keys,
                                  const uint32_t *vals, uint8_t *res, uint64_t n, cudaStream_t s) {
   CK(cudaStreamWaitEvent(s, h->last, 0));
+  h->d.zparity = (uint32_t)(h->batches & 1);  // R30: this batch's zombie-mark bitmap
   std::array<cudaEvent_t, 5> ev{};
   const bool prof = h->cfg.profile_phases != 0;
   if (prof) {
@@ -674,6 +710,28 @@ static gfsl_status enqueue_batch(gfsl *h, const uint8_t *ops, const uint32_t *ke
   CK(cudaEventRecord(h->last, s));
   h->batches++;
   h->ops += n;
+  return GFSL_OK;
+}
+
+extern "C" gfsl_status gfsl_rebuild(gfsl_t h, void *stream) {
+  if (!h) {
+    set_last_error("NULL handle");
+    return GFSL_EINVAL;
+  }
+  gfsl_status st = sticky(h);
+  if (st != GFSL_OK) return st;
+  cudaStream_t s = (cudaStream_t)stream;
+  CK(cudaStreamWaitEvent(s, h->last, 0));
+  switch (h->N) {
+    case 32: launch_rebuild<32>(h, s); break;
+    case 16: launch_rebuild<16>(h, s); break;
+    case 12: launch_rebuild<12>(h, s); break;
+    case 6: launch_rebuild<6>(h, s); break;
+  }
+  CK(cudaGetLastError());
+  CK(cudaEventRecord(h->last, s));
+  h->ops_since_rebuild = 0;
+  h->ops_at_rebuild = h->ops;
   return GFSL_OK;
 }
 
@@ -883,6 +941,7 @@ extern "C" gfsl_status gfsl_load(gfsl_t h, const gfsl_meta *meta, const uint64_t
   uint32_t bump[2] = {meta->used_bottom, meta->used_upper};
   CK(cudaMemcpy(h->d.bump, bump, 8, cudaMemcpyHostToDevice));
   CK(cudaMemset(h->d.dir_hdr, 0, 64 * 4));  // the directory describes the old structure
+  CK(cudaMemset(h->d.zbits, 0, (size_t)h->d.zwords * 8));
   return GFSL_OK;
 }
 

@@ -69,6 +69,14 @@ struct DevState {
   uint32_t *dir;
   uint32_t *dir_hdr;
   uint32_t dir_cap;      // entries allocated (a power of two)
+  // Zombie marks (R30): the update kernel sets bit c of zbits[zparity] when it makes chunk c
+  // a zombie; the upkeep sweep after the batch only has to follow NEXT pointers whose target
+  // bit is set, instead of reading every successor's lock word.  Two bitmaps of zwords words
+  // alternate by batch parity; a bit is cleared when upkeep passes the zombie two batches
+  // later, or when reclamation (R25) resets the chunk.
+  uint32_t *zbits;
+  uint32_t zwords;
+  uint32_t zparity;
   uint32_t p_chunk_q32;  // isKeyRaised probability as a 32-bit fraction; 0 = 1 (R16)
 };
 

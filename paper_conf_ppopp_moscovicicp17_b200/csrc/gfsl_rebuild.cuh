@@ -419,6 +419,8 @@ __global__ void __launch_bounds__(256) reclaim_write_kernel(const __grid_constan
       if (!z[q]) continue;
       const uint32_t c = d.cap_upper + tile * RC_TILE + threadIdx.x * 4 + q;
       newl[pos++] = c;
+      for (uint32_t par = 0; par < 2; ++par)  // R30: the chunk is no zombie any more
+        atomicAnd(d.zbits + (size_t)par * d.zwords + (c >> 5), ~(1u << (c & 31)));
       uint64_t *ch = d.pool + (size_t)c * N;
       for (int e = 0; e < N - 1; ++e) ch[e] = EMPTY_ENTRY;
       ch[N - 1] = (uint64_t)LOCK_HELD;

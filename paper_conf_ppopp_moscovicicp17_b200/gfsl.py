@@ -72,7 +72,7 @@ EXPORTS = [
     "gfsl_batch_host_async",
     "gfsl_validate", "gfsl_last_error", "gfsl_get_stats", "gfsl_dump", "gfsl_load",
     "gfsl_route_plan", "gfsl_route_pack", "gfsl_route_unpack", "gfsl_phase_times",
-    "gfsl_configure", "gfsl_ubench",
+    "gfsl_configure", "gfsl_ubench", "gfsl_rebuild",
     "gfsl_xr_create", "gfsl_xr_destroy", "gfsl_xr_export", "gfsl_xr_attach",
     "gfsl_xr_attach_local", "gfsl_xr_send", "gfsl_xr_push", "gfsl_xr_recv", "gfsl_xr_done",
     "gfsl_xr_finish", "gfsl_xr_batch",
@@ -118,6 +118,8 @@ def load_library(path: str = LIB_PATH):
     lib.gfsl_load.argtypes = [vp, ctypes.POINTER(gfsl_meta), vp, u64]
     lib.gfsl_ubench.restype = i32
     lib.gfsl_ubench.argtypes = [u32, u64, ctypes.POINTER(ctypes.c_double), ctypes.POINTER(ctypes.c_double)]
+    lib.gfsl_rebuild.restype = i32
+    lib.gfsl_rebuild.argtypes = [vp, vp]
     lib.gfsl_configure.restype = i32
     lib.gfsl_configure.argtypes = [vp, ctypes.POINTER(gfsl_config)]
     lib.gfsl_phase_times.restype = i32
@@ -247,6 +249,10 @@ class GFSL:
         _check(self.lib.gfsl_batch(self.h, _ptr(op), _ptr(key), _ptr(val), _ptr(out), n,
                                    _stream(stream)), "gfsl_batch")
         return out
+
+    def rebuild(self, stream=None):
+        """Rebuild the upper levels now (gfsl_rebuild; R24/R29), e.g. after a bulk load."""
+        _check(self.lib.gfsl_rebuild(self.h, _stream(stream)), "gfsl_rebuild")
 
     def batch_ptr(self, op_ptr: int, key_ptr: int, val_ptr: int | None, res_ptr: int, n: int,
                   stream=None):

@@ -195,3 +195,24 @@ def test_raise_draw_is_uniform():
     d = np.array([raise_draw(k, lv) for k in range(1, 20001) for lv in range(3)], np.uint64)
     for p in (0.25, 0.5, 0.75):
         assert abs(float((d < int(p * 2**32)).mean()) - p) < 0.01
+
+
+def test_default_rebuild_policy_counts_ops():
+    """R29: with rebuild_every = 0 the model rebuilds after the batch at which the ops
+    since the last rebuild reach 2.5 x min(capacity, ops submitted up to the last rebuild),
+    then counts again from zero; results and invariants are unchanged."""
+    R, N = 2000, 16
+    m = GFSLModel(N, R, cap_bottom=4000, cap_upper=1000, rebuild_every=0, rebuild_capacity=400)
+    o = OracleMap(R)
+    done = []
+    real = m.rebuild
+    m.rebuild = lambda: (done.append(m.batches), real())[1]
+    w = Workload(R, 150, mix=(35, 35, 30), seed=SEED_BASE + 41)
+    for b in range(12):
+        op, key, val, _ = w.make_batch(b)
+        opn, kn, vn = op.numpy(), key.numpy().astype(np.uint32), val.numpy().astype(np.uint32)
+        assert m.batch(opn.tolist(), kn.tolist(), vn.tolist()) == o.batch(opn, kn, vn).tolist()
+        assert m.check_invariants() == []
+    # 150-op batches: batch 0 (threshold 2.5 x 0), batch 3 (450 >= 2.5 x 150), then the
+    # threshold is 2.5 x min(400, 600) = 1000: batch 10 (1050)
+    assert done == [0, 3, 10]
