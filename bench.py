@@ -297,8 +297,7 @@ def run_gpu(args, world, rank, local):
         h.configure(combine=1 if combine_mode(args) else 0,
                     p_chunk_q32=int(args.p_chunk * 2**32) if args.p_chunk < 1.0 else 0,
                     l2_window=1 if args.l2_window else 0, no_pdl=1 if args.no_pdl else 0,
-                    rebuild_every=0xFFFFFFFF if args.rebuild_every < 0 else args.rebuild_every,
-                    key_order=1 if args.key_order == "on" else 0)
+                    rebuild_every=0xFFFFFFFF if args.rebuild_every < 0 else args.rebuild_every)
 
     apply_options(g.local if world > 1 else g)
     PROF = 3  # extra batches after the timed region, for the per-kernel breakdown
@@ -494,7 +493,6 @@ def run_gpu(args, world, rank, local):
                        "semantics": "combining (R26): mutations in input order, any batch" if combine_mode(args)
                        else "S1 snapshot, <=1 mutation per key (R1/R2)",
                        "chunk_entries": N, "p_chunk": args.p_chunk, "contains_team": contains_team,
-                       "key_order": args.key_order,
                        "l2": "flushed (256 MiB write) between timed steps",
                        "parallelism": f"range-shard x{world}" if world > 1 else "1 GPU",
                        "exchange": (("peer windows (CUDA IPC, fused route kernels)" if args.exchange == "peer"
@@ -543,9 +541,6 @@ def main():
                          "0 = library default (4), -1 = never (the paper's dynamics only)")
     ap.add_argument("--dist-backend", default="nccl", choices=["nccl", "gloo"],
                     help="gloo: exercise the multi-rank path with ranks sharing a GPU (no timing value)")
-    ap.add_argument("--key-order", default="off", choices=["on", "off"],
-                    help="key-ordered intake (R31, measured, off by default): radix-sort each "
-                         "batch by its keys' top 16 bits before the search phase")
     ap.add_argument("--exchange", default="peer", choices=["peer", "nccl"],
                     help="N>1 exchange: peer = fused route kernels over CUDA-IPC windows "
                          "(NEXT-3); nccl = torch.distributed all-to-all (baseline)")

@@ -108,13 +108,6 @@ typedef struct gfsl_config {
                                (raised key, level), so runs are reproducible.  The periodic
                                upper-level rebuild (rebuild_every) replaces what the raises
                                built; combine with GFSL_REBUILD_NEVER to study p_chunk. */
-  uint32_t key_order;       /* 1 = key-ordered intake (R31, measured and not the
-                               default): the batch's ops are radix-sorted by the high 16
-                               bits of their keys before the search phase, so that the ops
-                               in flight at one time share chunks, and the update records
-                               are taken in a spread order; results are unchanged (S1
-                               answers every op on the snapshot, in any order).  0 = off.
-                               Ignored in serial mode. */
 } gfsl_config;
 
 /*

@@ -88,12 +88,6 @@ struct gfsl {
   uint2 *vw = nullptr;
   void *cub_tmp = nullptr;
   size_t cub_bytes = 0;
-  // key-ordered intake (R31)
-  uint32_t *ko_key = nullptr, *ko_w[2] = {nullptr, nullptr};
-  void *ko_tmp = nullptr;
-  size_t ko_bytes = 0;
-  uint64_t ko_cap = 0;
-  bool spread_now = false;  // this batch's update records are taken in spread order
   uint64_t comb_cap = 0;
   int sort_bits = 32;
   uint32_t region_cap = 1;  // record slots per region for the current batch
@@ -147,9 +141,9 @@ static SearchOut search_out(gfsl *h) {
   const uint32_t full = h->cfg.serial_updates ? 1u : 0u;  // serial mode: traversals from the top
   if (h->cfg.combine)
     return SearchOut{h->mut_rec, h->plan_path, h->mut_of, h->ctl->ccnt, h->region_cap, h->ck[0], h->cw[0], full,
-                     h->spread_now ? 1u : 0u, nullptr};
+                     0u, nullptr};
   return SearchOut{h->mut_rec, h->plan_path, h->cfg.serial_updates ? h->mut_of : nullptr,
-                   h->ctl->mcnt, h->region_cap, nullptr, nullptr, full, h->spread_now ? 1u : 0u,
+                   h->ctl->mcnt, h->region_cap, nullptr, nullptr, full, 0u,
                    h->cfg.serial_updates ? nullptr : h->mut_ver};
 }
 // What the update kernel reads: the same records, or the net mutations of combining mode.
@@ -409,10 +403,6 @@ static void free_all(gfsl *h) {
   cudaFree(h->net_path);
   cudaFree(h->vw);
   cudaFree(h->cub_tmp);
-  cudaFree(h->ko_key);
-  cudaFree(h->ko_w[0]);
-  cudaFree(h->ko_w[1]);
-  cudaFree(h->ko_tmp);
   cudaFree(h->d.freelist);
   cudaFree(h->d.zbits);
   cudaFree(h->d.fl);
@@ -666,66 +656,6 @@ static gfsl_status ensure_combine(gfsl *h, uint64_t n) {
 
 // R26: sort the batch's (key, op) pairs so that each key's Insert/Delete chain is
 // contiguous and in input order (LSD radix sort is stable), then reduce the chains.
-// ---- key-ordered intake (R31) ----
-static bool use_key_order(const gfsl *h, uint64_t n) {
-  return n > 0 && h->cfg.key_order == 1 && !h->cfg.serial_updates;
-}
-// bits [lo, hi) of the user key that the intake sort orders by: the top 16 of the key range
-static void key_order_bits(const gfsl *h, int &lo, int &hi) {
-  hi = 1;
-  while (hi < 32 && (1ull << hi) < h->key_range) ++hi;
-  lo = std::max(0, hi - 16);
-}
-static gfsl_status ensure_key_order(gfsl *h, uint64_t n) {
-  if (!use_key_order(h, n)) return GFSL_OK;
-  int lo, hi;
-  key_order_bits(h, lo, hi);
-  size_t need = 0;
-  CK(cub::DeviceRadixSort::SortPairs(nullptr, need, (const uint32_t *)nullptr, (uint32_t *)nullptr,
-                                     (const uint32_t *)nullptr, (uint32_t *)nullptr,
-                                     (int)std::max<uint64_t>(n, h->ko_cap), lo, hi));
-  if (n <= h->ko_cap && need <= h->ko_bytes) return GFSL_OK;
-  cudaDeviceSynchronize();
-  if (n > h->ko_cap) {
-    cudaFree(h->ko_key);
-    cudaFree(h->ko_w[0]);
-    cudaFree(h->ko_w[1]);
-    h->ko_key = h->ko_w[0] = h->ko_w[1] = nullptr;
-    h->ko_cap = 0;
-    CK(cudaMalloc(&h->ko_key, n * 4));
-    CK(cudaMalloc(&h->ko_w[0], n * 4));
-    CK(cudaMalloc(&h->ko_w[1], n * 4));
-    h->ko_cap = n;
-  }
-  if (need > h->ko_bytes) {
-    cudaFree(h->ko_tmp);
-    h->ko_tmp = nullptr;
-    h->ko_bytes = 0;
-    CK(cudaMalloc(&h->ko_tmp, need));
-    h->ko_bytes = need;
-  }
-  return GFSL_OK;
-}
-// the sort's payload: op index | op code (capped at 3 = invalid) << 29
-__global__ void key_order_pack_kernel(const uint8_t *ops, uint32_t n, uint32_t *w) {
-  for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < n; i += gridDim.x * blockDim.x)
-    w[i] = i | ((uint32_t)min(ops[i], (uint8_t)3) << 29);
-}
-static gfsl_status enqueue_key_order(gfsl *h, BatchIn &in, cudaStream_t s) {
-  int lo, hi;
-  key_order_bits(h, lo, hi);
-  const int grid = (int)std::min<uint64_t>((in.n + 255) / 256, (uint64_t)h->sms * 8);
-  key_order_pack_kernel<<<grid, 256, 0, s>>>(in.ops, in.n, h->ko_w[0]);
-  h->launches += 1;
-  size_t bytes = h->ko_bytes;
-  CK(cub::DeviceRadixSort::SortPairs(h->ko_tmp, bytes, in.keys, h->ko_key, h->ko_w[0], h->ko_w[1],
-                                     (int)in.n, lo, hi, s));
-  h->lib_launches += 1 + (uint64_t)(hi - lo + 7) / 8;  // onesweep: histogram + one pass per digit
-  in.skey = h->ko_key;
-  in.sw = h->ko_w[1];
-  return GFSL_OK;
-}
-
 static gfsl_status enqueue_combine(gfsl *h, const BatchIn &in, cudaStream_t s) {
   cub::DoubleBuffer<uint32_t> kb(h->ck[0], h->ck[1]), vb(h->cw[0], h->cw[1]);
   size_t bytes = h->cub_bytes;
@@ -756,13 +686,8 @@ static gfsl_status enqueue_batch(gfsl *h, const uint8_t *ops, const uint32_t *ke
     CK(cudaEventRecord(ev[0], s));
   }
   CK(cudaMemsetAsync(h->ctl, 0, offsetof(BatchCtl, uq) + (size_t)std::min(h->update_grid, BatchCtl::UQ_MAX) * 32, s));
-  BatchIn in{ops, keys, vals, res, (uint32_t)n, h->key_range, nullptr, nullptr};
-  h->spread_now = use_key_order(h, n);
-  if (h->spread_now) {
-    gfsl_status ks = enqueue_key_order(h, in, s);
-    if (ks != GFSL_OK) return ks;
-  }
   if (prof) CK(cudaEventRecord(ev[1], s));
+  const BatchIn in{ops, keys, vals, res, (uint32_t)n, h->key_range};
   bool ok = dispatch_contains(h, in, s);
   if (!ok) {
     set_last_error("no contains kernel for this (N, team)");
@@ -834,7 +759,6 @@ extern "C" gfsl_status gfsl_batch(gfsl_t h, const uint8_t *op_types, const uint3
   }
   if ((st = ensure_lists(h, n)) != GFSL_OK) return st;
   if (h->cfg.combine && (st = ensure_combine(h, n)) != GFSL_OK) return st;
-  if ((st = ensure_key_order(h, n)) != GFSL_OK) return st;
   return enqueue_batch(h, op_types, keys, values, results, n, (cudaStream_t)stream);
 }
 
@@ -884,7 +808,6 @@ static gfsl_status batch_host_async(gfsl *h, const uint8_t *op_types, const uint
   if ((st = ensure_staging(h, n)) != GFSL_OK) return st;
   if ((st = ensure_lists(h, n)) != GFSL_OK) return st;
   if (h->cfg.combine && (st = ensure_combine(h, n)) != GFSL_OK) return st;
-  if ((st = ensure_key_order(h, n)) != GFSL_OK) return st;
   const int b = h->st_slot;
   h->st_slot ^= 1;
   cudaStream_t c = h->copy_stream;

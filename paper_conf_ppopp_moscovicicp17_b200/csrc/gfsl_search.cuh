@@ -59,10 +59,6 @@ struct BatchIn {
   uint8_t *res;
   uint32_t n;
   uint64_t key_range;
-  // Key-ordered intake (R31), or NULL: slot j holds op sw[j] & OPI_MASK, whose op code
-  // (capped at 3 = invalid) is in bits 29-30 of sw[j] and whose key is skey[j]
-  const uint32_t *skey;
-  const uint32_t *sw;
 };
 
 // The mutations a batch's search phase hands to the update phase, compact: mutation m
@@ -79,7 +75,8 @@ struct SearchOut {
                         // for a valid Insert/Delete, else all ones
   uint32_t *comb_w;     // [n]: op i | CW_* flags (the sort's payload)
   uint32_t full_path;   // 1 = every Insert/Delete traverses from the top (serial mode)
-  uint32_t spread;      // 1 = the update kernel takes the records in a spread order (R31)
+  uint32_t spread;      // 1 = the update kernel takes the records in a spread order (R31:
+                        // combining mode, whose net records come out of a key sort)
   uint32_t *mut_ver;    // [n] or NULL: mutation m's path[0] lock version in the snapshot
                         // (R32: the update kernel's one-round-trip lock)
 };
@@ -169,33 +166,24 @@ search_kernel(DevState d, const BatchIn in, BatchCtl *__restrict__ ctl, SearchOu
   // The prefetched op stays raw (loaded, not yet looked at) until it becomes current, so
   // its loads overlap the current traversal.
   // An Insert's value is loaded when the op becomes current (it is needed only at its end).
-  // Key-ordered intake (R31): slot j is the j-th op in key order, carrying its input index.
   struct RawOp {
-    uint32_t op, key, idx;
+    uint32_t op, key;
   };
   auto load_raw = [&](uint32_t i) -> RawOp {
-    RawOp r{3u, 0u, i};
+    RawOp r{3u, 0u};
     if (lane_live && i < n) {
-      if (in.sw) {
-        const uint32_t w = __ldg(in.sw + i);
-        r.op = (w >> 29) & 3u;
-        r.idx = w & OPI_MASK;
-        r.key = __ldg(in.skey + i);
-      } else {
-        r.op = __ldg(in.ops + i);
-        r.key = __ldg(in.keys + i);
-      }
+      r.op = __ldg(in.ops + i);
+      r.key = __ldg(in.keys + i);
     }
     return r;
   };
   auto load_val = [&](uint32_t i, const RawOp &r) -> uint32_t {
-    return (t == 0 && in.vals && r.op == 1 && lane_live && i < n) ? __ldg(in.vals + r.idx) : 0u;
+    return (t == 0 && in.vals && r.op == 1 && lane_live && i < n) ? __ldg(in.vals + i) : 0u;
   };
   auto decode = [&](uint32_t i, const RawOp &r) -> uint2 {
-    (void)i;
     const bool valid = r.op <= 2 && (uint64_t)r.key < in.key_range;
     const uint32_t fl = !valid ? INVALID_FLAG : (r.op == 2 ? (DELETE_FLAG | UPDATE_FLAG) : (r.op == 1 ? UPDATE_FLAG : 0u));
-    return make_uint2(r.idx | fl, valid ? r.key + 1u : 1u);
+    return make_uint2(i | fl, valid ? r.key + 1u : 1u);
   };
   uint32_t slot = warp_global * TPW + team_in_warp;  // this team's current op slot
   RawOp raw = load_raw(slot);
@@ -366,8 +354,8 @@ struct MutMap {
   uint32_t cap;
   uint32_t spread;       // R31: take slot s as (s * 2654435761) mod total (a bijection: the
                          // multiplier is a prime > 2^29 >= total), so that the records the
-                         // update teams hold at one time -- which a key-ordered search
-                         // phase wrote in about key order -- are far apart in key space
+                         // update teams hold at one time -- which the combining sort wrote
+                         // in key order -- are far apart in key space
   __device__ __forceinline__ uint32_t total() const { return excl[BatchCtl::MUT_REGIONS]; }
   __device__ __forceinline__ uint32_t rec(uint32_t s) const {
     if (spread) s = (uint32_t)(((uint64_t)s * 2654435761ull) % total());

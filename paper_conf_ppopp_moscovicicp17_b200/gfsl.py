@@ -36,7 +36,7 @@ class gfsl_config(ctypes.Structure):
                 ("profile_phases", ctypes.c_uint32), ("l2_window", ctypes.c_uint32),
                 ("no_pdl", ctypes.c_uint32),
                 ("rebuild_every", ctypes.c_uint32), ("combine", ctypes.c_uint32),
-                ("p_chunk_q32", ctypes.c_uint32), ("key_order", ctypes.c_uint32)]
+                ("p_chunk_q32", ctypes.c_uint32)]
 
 
 class gfsl_report(ctypes.Structure):
@@ -207,8 +207,7 @@ class GFSL:
                  contains_team: int = 0, serial_updates: bool = False,
                  contains_blocks_per_sm: int = 0, update_blocks_per_sm: int = 0,
                  count_reads: bool = False, profile_phases: bool = False,
-                 rebuild_every: int = 0, combine: bool = False, p_chunk: float = 1.0,
-                 key_order: int = 0):
+                 rebuild_every: int = 0, combine: bool = False, p_chunk: float = 1.0):
         import torch
         if not torch.cuda.is_available():
             raise RuntimeError("GFSL needs a CUDA device (there is no CPU fallback)")
@@ -217,7 +216,7 @@ class GFSL:
                           update_blocks_per_sm, 1 if serial_updates else 0,
                           1 if count_reads else 0, 1 if profile_phases else 0, 0, 0,
                           rebuild_every, 1 if combine else 0,
-                          0 if p_chunk >= 1.0 else int(p_chunk * 2**32), key_order)
+                          0 if p_chunk >= 1.0 else int(p_chunk * 2**32))
         self.key_range = int(key_range)
         self.chunk_entries = int(chunk_entries)
         self.cfg = cfg
