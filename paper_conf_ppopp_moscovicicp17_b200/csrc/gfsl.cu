@@ -56,7 +56,6 @@ struct gfsl {
   BatchCtl *ctl = nullptr;
   uint32_t *plan_path = nullptr, *mut_of = nullptr;
   uint4 *mut_rec = nullptr;
-  uint32_t *mut_ver = nullptr;  // R32
   uint64_t list_cap = 0;
   uint32_t *h_error = nullptr;  // mapped host memory, device alias in d.error
   cudaEvent_t last = nullptr;
@@ -141,16 +140,15 @@ static SearchOut search_out(gfsl *h) {
   const uint32_t full = h->cfg.serial_updates ? 1u : 0u;  // serial mode: traversals from the top
   if (h->cfg.combine)
     return SearchOut{h->mut_rec, h->plan_path, h->mut_of, h->ctl->ccnt, h->region_cap, h->ck[0], h->cw[0], full,
-                     0u, nullptr};
+                     0u};
   return SearchOut{h->mut_rec, h->plan_path, h->cfg.serial_updates ? h->mut_of : nullptr,
-                   h->ctl->mcnt, h->region_cap, nullptr, nullptr, full, 0u,
-                   h->cfg.serial_updates ? nullptr : h->mut_ver};
+                   h->ctl->mcnt, h->region_cap, nullptr, nullptr, full, 0u};
 }
 // What the update kernel reads: the same records, or the net mutations of combining mode.
 static SearchOut update_in(gfsl *h) {
   if (h->cfg.combine)
     return SearchOut{h->net_rec, h->net_path, h->mut_of, h->ctl->mcnt, h->region_cap, nullptr, nullptr, 0u,
-                     1u, nullptr};  // net records come out of the combining sort in key order (R31)
+                     1u};  // net records come out of the combining sort in key order (R31)
   return search_out(h);
 }
 
@@ -377,7 +375,6 @@ static void free_all(gfsl *h) {
   cudaFree(h->plan_path);
   cudaFree(h->mut_of);
   cudaFree(h->mut_rec);
-  cudaFree(h->mut_ver);
   for (int b = 0; b < 2; ++b) {
     cudaFree(h->st_op[b]);
     cudaFree(h->st_res[b]);
@@ -594,17 +591,14 @@ static gfsl_status ensure_lists(gfsl *h, uint64_t n) {
   cudaFree(h->plan_path);
   cudaFree(h->mut_of);
   cudaFree(h->mut_rec);
-  cudaFree(h->mut_ver);
   h->plan_path = nullptr;
   h->mut_of = nullptr;
   h->mut_rec = nullptr;
-  h->mut_ver = nullptr;
   h->list_cap = 0;
   const uint64_t cap = std::max<uint64_t>(n, 1024);
   CK(cudaMalloc(&h->plan_path, cap * 4 * PLAN_LEVELS));
   CK(cudaMalloc(&h->mut_of, cap * 4));
   CK(cudaMalloc(&h->mut_rec, cap * 16));
-  CK(cudaMalloc(&h->mut_ver, cap * 4));
   h->list_cap = cap;
   return GFSL_OK;
 }
@@ -679,6 +673,11 @@ static gfsl_status enqueue_batch(gfsl *h, const uint8_t *ops, const uint32_t *ke
                                  const uint32_t *vals, uint8_t *res, uint64_t n, cudaStream_t s) {
   CK(cudaStreamWaitEvent(s, h->last, 0));
   h->d.zparity = (uint32_t)(h->batches & 1);  // R30: this batch's zombie-mark bitmap
+#ifdef GFSL_NO_LAZY_UPPER  // ablation
+  h->d.lazy_upper = 0;
+#else
+  h->d.lazy_upper = (!h->cfg.serial_updates && h->cfg.rebuild_every != GFSL_REBUILD_NEVER) ? 1u : 0u;  // R33
+#endif
   std::array<cudaEvent_t, 5> ev{};
   const bool prof = h->cfg.profile_phases != 0;
   if (prof) {

@@ -77,6 +77,9 @@ struct DevState {
   uint32_t *zbits;
   uint32_t zwords;
   uint32_t zparity;
+  // R33: concurrent batches with the upper-level rebuild on leave the levels >= 1 to the
+  // next rebuild: no raise after a split (isKeyRaised false) and no updateDownPtrs
+  uint32_t lazy_upper;
   uint32_t p_chunk_q32;  // isKeyRaised probability as a 32-bit fraction; 0 = 1 (R16)
 };
 

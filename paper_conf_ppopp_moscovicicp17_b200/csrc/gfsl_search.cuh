@@ -77,8 +77,6 @@ struct SearchOut {
   uint32_t full_path;   // 1 = every Insert/Delete traverses from the top (serial mode)
   uint32_t spread;      // 1 = the update kernel takes the records in a spread order (R31:
                         // combining mode, whose net records come out of a key sort)
-  uint32_t *mut_ver;    // [n] or NULL: mutation m's path[0] lock version in the snapshot
-                        // (R32: the update kernel's one-round-trip lock)
 };
 
 // A record slot in the writing block's region (BatchCtl::mcnt).
@@ -250,11 +248,6 @@ search_kernel(DevState d, const BatchIn in, BatchCtl *__restrict__ ctl, SearchOu
     const int src = tb ? team_base + 31 - __clz(tb) : lane;
     const uint32_t dptr = __shfl_sync(FULL, dv, src);
     const uint32_t np = __shfl_sync(FULL, nx, next_src);
-    // R32: an Insert/Delete on the bottom level keeps its chunk's lock version (hi32 of
-    // the LOCK entry, unlocked in the snapshot) for the update kernel's validated lock
-    uint32_t lver = 0;
-    if (so.mut_ver && __any_sync(FULL, active && level == 0 && (cur_op.x & UPDATE_FLAG)))
-      lver = __shfl_sync(FULL, s.v[LOCK_J], lane_live ? team_base + LOCK_LANE : lane);
 
     if (active) {
       const bool lat = (np & (F_ZOMBIE | F_LATERAL)) != 0;  // zombie (l.9-11) / lateral (l.15-18)
@@ -298,7 +291,6 @@ search_kernel(DevState d, const BatchIn in, BatchCtl *__restrict__ ctl, SearchOu
               // {op index | DELETE_FLAG, key, path[0], top (Delete) | value (Insert)}
               const uint32_t w = opi | (cur_op.x & DELETE_FLAG);
               so.mut_rec[m] = make_uint4(w, k, here, (cur_op.x & DELETE_FLAG) ? seen_top : cur_val);
-              if (so.mut_ver) so.mut_ver[m] = lver;
               my_path[0] = here;  // path[0] = the enclosing bottom chunk
               if (via_dir) {      // levels >= 2 from the directory rank (R27)
                 uint32_t q = cur_r / F;
