@@ -73,6 +73,7 @@ struct gfsl {
   uint64_t capacity = 0;           // max live keys (gfsl_create)
   uint64_t ops_since_rebuild = 0;  // default rebuild policy (R29)
   uint64_t ops_at_rebuild = 0;     // h->ops after the batch of the last rebuild
+  bool upper_stale = false;        // R33: a lazy batch ran since the last rebuild
   uint64_t launches = 0, lib_launches = 0;  // our kernels / CUB's (combining sort) enqueued by batches
   std::vector<std::array<cudaEvent_t, 5>> phase_ev;  // profile_phases
   // L2 persistence for the upper pool (the search kernel's access-policy window)
@@ -214,6 +215,7 @@ static bool dispatch_contains(gfsl *h, const BatchIn &in, cudaStream_t s) {
 // kernel makes it a no-op unless a batch mutated the structure since the last one.
 template <int N>
 static void launch_rebuild(gfsl *h, cudaStream_t s) {
+  h->upper_stale = false;  // R33: levels >= 1 re-derived from level 0
   cudaLaunchConfig_t lc{};
   cudaLaunchAttribute attr[1];
   set_pdl(h, attr[0]);
@@ -678,6 +680,7 @@ static gfsl_status enqueue_batch(gfsl *h, const uint8_t *ops, const uint32_t *ke
 #else
   h->d.lazy_upper = (!h->cfg.serial_updates && h->cfg.rebuild_every != GFSL_REBUILD_NEVER) ? 1u : 0u;  // R33
 #endif
+  if (h->d.lazy_upper) h->upper_stale = true;
   std::array<cudaEvent_t, 5> ev{};
   const bool prof = h->cfg.profile_phases != 0;
   if (prof) {
@@ -1109,11 +1112,20 @@ extern "C" gfsl_status gfsl_validate(gfsl_t h, gfsl_report *rep_out, uint32_t *k
       const uint32_t k = up[i].first;
       auto it = std::lower_bound(lo.begin(), lo.end(), std::make_pair(k, 0u),
                                  [](auto a, auto b) { return a.first < b.first; });
+      uint32_t target;
       if (it == lo.end() || it->first != k) {
-        V(4);
-        continue;
+        // R33: after lazy batches a level-1 key may be a stale separator (deleted from
+        // level 0 since the last rebuild); its down pointer must still reach, laterally,
+        // the level-0 chunk that encloses k (the chunk of the next larger key, or the last)
+        if (!(h->upper_stale && l == 0) || chunks[0].empty()) {
+          V(4);
+          continue;
+        }
+        // k above every key (or level 0 empty): the last chunk of the level
+        target = it == lo.end() ? chunks[0].back() : keychunk[l][it - lo.begin()];
+      } else {
+        target = keychunk[l][it - lo.begin()];
       }
-      const uint32_t target = keychunk[l][it - lo.begin()];
       // walk laterally from the down pointer to the chunk holding k
       uint32_t c = up[i].second;
       uint64_t steps = 0;

@@ -78,7 +78,8 @@ struct DevState {
   uint32_t zwords;
   uint32_t zparity;
   // R33: concurrent batches with the upper-level rebuild on leave the levels >= 1 to the
-  // next rebuild: no raise after a split (isKeyRaised false) and no updateDownPtrs
+  // next rebuild: no raise after a split (isKeyRaised false), no updateDownPtrs, and a
+  // Delete removes k from level 0 only (its upper copies stay as stale separators)
   uint32_t lazy_upper;
   uint32_t p_chunk_q32;  // isKeyRaised probability as a 32-bit fraction; 0 = 1 (R16)
 };

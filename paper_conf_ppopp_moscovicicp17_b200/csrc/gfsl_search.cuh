@@ -257,7 +257,8 @@ search_kernel(DevState d, const BatchIn in, BatchCtl *__restrict__ ctl, SearchOu
       // restart (l.25): only from a directory entry made stale by the batches since the
       // last rebuild (R27: level-1 keys <= k deleted from that chunk), never from the top;
       // and on purpose when a Delete entered at level 1 finds k there (its exact top)
-      const bool redo = via_dir && down && level == 1 && tb && (dptr & F_EQUAL) && (cur_op.x & DELETE_FLAG);
+      const bool redo = via_dir && down && level == 1 && tb && (dptr & F_EQUAL) && (cur_op.x & DELETE_FLAG) &&
+                        !d.lazy_upper;  // R33: a lazy Delete removes k from level 0 only
       const bool restart = (down && !tb && bt == NULL_CHUNK) || redo;
       const uint32_t here = cur;
       if (down && upd && t == 0 && level < PLAN_LEVELS)     // searchSlow's path (Alg 4.6 l.28-37)
@@ -290,7 +291,9 @@ search_kernel(DevState d, const BatchIn in, BatchCtl *__restrict__ ctl, SearchOu
               m = mut_slot(so);
               // {op index | DELETE_FLAG, key, path[0], top (Delete) | value (Insert)}
               const uint32_t w = opi | (cur_op.x & DELETE_FLAG);
-              so.mut_rec[m] = make_uint4(w, k, here, (cur_op.x & DELETE_FLAG) ? seen_top : cur_val);
+              // R33: in lazy mode a Delete's top is 0 (level-1 copies of k stay until the
+              // next rebuild, as stale separators)
+              so.mut_rec[m] = make_uint4(w, k, here, (cur_op.x & DELETE_FLAG) ? (d.lazy_upper ? 0u : (uint32_t)seen_top) : cur_val);
               my_path[0] = here;  // path[0] = the enclosing bottom chunk
               if (via_dir) {      // levels >= 2 from the directory rank (R27)
                 uint32_t q = cur_r / F;
