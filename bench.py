@@ -488,7 +488,7 @@ def run_gpu(args, world, rank, local):
             "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
             "dtype": "u32", "data": "synthetic",
             "config": {"workload": args.config, "key_range": R,
-                       "rebuild_every": "never" if args.rebuild_every < 0 else (args.rebuild_every or "default: ops since the last rebuild >= 2.5 x capacity (R29)"), "prefill": pre1 * world,
+                       "rebuild_every": "never" if args.rebuild_every < 0 else (args.rebuild_every or "default: ops since the last rebuild >= 5 x min(capacity, ops up to it) (R29)"), "prefill": pre1 * world,
                        "batch_ops": B1 * world, "mix_ins_del_con": list(mix), "keys": dist,
                        "semantics": "combining (R26): mutations in input order, any batch" if combine_mode(args)
                        else "S1 snapshot, <=1 mutation per key (R1/R2)",

@@ -53,9 +53,9 @@ typedef enum gfsl_status {
  * batch at which the ops submitted since the last rebuild reach GFSL_REBUILD_DEFAULT_WEAR x
  * L, L = min(capacity, ops submitted up to the last rebuild) -- an upper bound on the live
  * keys, so a structure growing from empty is rebuilt at geometrically spaced sizes.  In
- * steady state with the paper's [10,10,80] mix at half fill this is about one mutation per
- * live key (every 4 batches at C1-C3, every 20 at C5). */
-#define GFSL_REBUILD_DEFAULT_WEAR 2.5
+ * steady state with the paper's [10,10,80] mix at half fill this is about two mutations
+ * per live key (every 8 batches at C1-C3, every 40 at C5). */
+#define GFSL_REBUILD_DEFAULT_WEAR 5
 #define GFSL_REBUILD_NEVER 0xFFFFFFFFu
 
 /* Largest batch (ops per gfsl_batch call): the op index shares a 32-bit word with three

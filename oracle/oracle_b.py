@@ -64,8 +64,8 @@ class GFSLModel:
         self.p_chunk_q32 = p_chunk_q32
         self.rebuild_every = rebuild_every
         # R29, used if rebuild_every = 0 and rebuild_capacity > 0: rebuild after
-        # the batch at which the ops since the last rebuild reach 2.5 x min(capacity, ops
-        # submitted up to the last rebuild)
+        # the batch at which the ops since the last rebuild reach 5 x min(capacity, ops
+        # submitted up to the last rebuild) (GFSL_REBUILD_DEFAULT_WEAR)
         self.rebuild_capacity = rebuild_capacity
         self.ops_total = self.ops_since = self.ops_at_rebuild = 0
         self.batches = 0
@@ -498,7 +498,7 @@ class GFSLModel:
             due = (self.batches + 1) % self.rebuild_every == 0
         elif n and self.rebuild_capacity:
             self.ops_since += n
-            due = 2 * self.ops_since >= 5 * min(self.rebuild_capacity, self.ops_at_rebuild)
+            due = self.ops_since >= 5 * min(self.rebuild_capacity, self.ops_at_rebuild)
             if due:
                 self.ops_since, self.ops_at_rebuild = 0, self.ops_total + n
         self.ops_total += n

@@ -74,6 +74,7 @@ struct gfsl {
   uint64_t ops_since_rebuild = 0;  // default rebuild policy (R29)
   uint64_t ops_at_rebuild = 0;     // h->ops after the batch of the last rebuild
   bool upper_stale = false;        // R33: a lazy batch ran since the last rebuild
+  bool upkeep_pending = false;     // R33: lazy batches skipped the upkeep sweep
   uint64_t launches = 0, lib_launches = 0;  // our kernels / CUB's (combining sort) enqueued by batches
   std::vector<std::array<cudaEvent_t, 5>> phase_ev;  // profile_phases
   // L2 persistence for the upper pool (the search kernel's access-policy window)
@@ -222,6 +223,15 @@ static void launch_rebuild(gfsl *h, cudaStream_t s) {
   lc.attrs = attr;
   lc.numAttrs = 1;
   lc.stream = s;
+  if (h->upkeep_pending) {  // R33: the zombie unlinking the lazy batches deferred
+    DevState d = h->d;
+    d.upkeep_force = 1;
+    lc.gridDim = dim3(h->sms * 4);
+    lc.blockDim = dim3(256);
+    cudaLaunchKernelEx(&lc, upkeep_kernel<N>, d);
+    h->launches += 1;
+    h->upkeep_pending = false;
+  }
   const RebuildBufs &b = h->rb;
   h->launches += 9;
   lc.gridDim = dim3(1);
@@ -263,7 +273,7 @@ static void launch_update(gfsl *h, const BatchIn &in, cudaStream_t s, cudaEvent_
   lc.gridDim = dim3(h->cfg.serial_updates ? 1 : h->update_grid);
   const int serial = h->cfg.serial_updates ? 1 : 0;
   cudaLaunchKernelEx(&lc, update_kernel<N>, h->d, in, h->ctl, update_in(h), serial);
-  h->launches += 2;  // update + upkeep
+  h->launches += 1;  // update
   lc.blockDim = dim3(256);
   if (h->cfg.combine) {  // R26: keys deleted and re-inserted in this batch get their new value
     lc.gridDim = dim3(h->sms * 2);
@@ -271,8 +281,23 @@ static void launch_update(gfsl *h, const BatchIn &in, cudaStream_t s, cudaEvent_
     h->launches += 1;
   }
   if (after_update) cudaEventRecord(after_update, s);
-  lc.gridDim = dim3(h->sms * 4);
-  cudaLaunchKernelEx(&lc, upkeep_kernel<N>, h->d);
+  // upkeep (R23): after every batch, or -- lazy batches (R33) -- deferred to just before
+  // the next rebuild (zombie chains at level 0 are passed laterally meanwhile); the
+  // zombie marks (R30) then accumulate in one bitmap, cleared by the reclamation
+#ifdef GFSL_NO_DEFER_UPKEEP  // ablation
+  if (true) {
+#else
+  if (!h->d.lazy_upper) {
+#endif
+    DevState d = h->d;
+    d.upkeep_force = h->upkeep_pending ? 1u : 0u;
+    lc.gridDim = dim3(h->sms * 4);
+    cudaLaunchKernelEx(&lc, upkeep_kernel<N>, d);
+    h->launches += 1;
+    h->upkeep_pending = false;
+  } else {
+    h->upkeep_pending = true;
+  }
   // R24 / R29: rebuild the upper levels from level 0 -- by default after the batch at
   // which the ops since the last rebuild reach GFSL_REBUILD_DEFAULT_WEAR x L, where L =
   // min(capacity, ops ever submitted up to the last rebuild) bounds the live keys from
@@ -680,7 +705,10 @@ static gfsl_status enqueue_batch(gfsl *h, const uint8_t *ops, const uint32_t *ke
 #else
   h->d.lazy_upper = (!h->cfg.serial_updates && h->cfg.rebuild_every != GFSL_REBUILD_NEVER) ? 1u : 0u;  // R33
 #endif
-  if (h->d.lazy_upper) h->upper_stale = true;
+  if (h->d.lazy_upper) {
+    h->upper_stale = true;
+    h->d.zparity = 0;  // R33: the marks of all lazy batches since the last rebuild
+  }
   std::array<cudaEvent_t, 5> ev{};
   const bool prof = h->cfg.profile_phases != 0;
   if (prof) {

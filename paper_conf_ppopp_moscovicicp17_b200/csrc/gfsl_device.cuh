@@ -81,6 +81,8 @@ struct DevState {
   // next rebuild: no raise after a split (isKeyRaised false), no updateDownPtrs, and a
   // Delete removes k from level 0 only (its upper copies stay as stale separators)
   uint32_t lazy_upper;
+  uint32_t upkeep_force;  // R33: the deferred upkeep before a rebuild runs even if this
+                          // batch merged nothing (earlier lazy batches did)
   uint32_t p_chunk_q32;  // isKeyRaised probability as a 32-bit fraction; 0 = 1 (R16)
 };
 

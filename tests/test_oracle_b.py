@@ -199,7 +199,7 @@ def test_raise_draw_is_uniform():
 
 def test_default_rebuild_policy_counts_ops():
     """R29: with rebuild_every = 0 the model rebuilds after the batch at which the ops
-    since the last rebuild reach 2.5 x min(capacity, ops submitted up to the last rebuild),
+    since the last rebuild reach 5 x min(capacity, ops submitted up to the last rebuild),
     then counts again from zero; results and invariants are unchanged."""
     R, N = 2000, 16
     m = GFSLModel(N, R, cap_bottom=4000, cap_upper=1000, rebuild_every=0, rebuild_capacity=400)
@@ -213,6 +213,6 @@ def test_default_rebuild_policy_counts_ops():
         opn, kn, vn = op.numpy(), key.numpy().astype(np.uint32), val.numpy().astype(np.uint32)
         assert m.batch(opn.tolist(), kn.tolist(), vn.tolist()) == o.batch(opn, kn, vn).tolist()
         assert m.check_invariants() == []
-    # 150-op batches: batch 0 (threshold 2.5 x 0), batch 3 (450 >= 2.5 x 150), then the
-    # threshold is 2.5 x min(400, 600) = 1000: batch 10 (1050)
-    assert done == [0, 3, 10]
+    # 150-op batches: batch 0 (threshold 5 x 0), batch 5 (750 >= 5 x 150), then the
+    # threshold is 5 x min(400, 900) = 2000: not reached by batch 11 (900)
+    assert done == [0, 5]
