@@ -290,7 +290,8 @@ def run_gpu(args, world, rank, local):
         lo = g.key_lo
         prefill_gpu(g.local, R1, pre1, dev, key_lo=lo, seed=SEED_BASE + 1000 * rank)
     else:
-        g = GFSL(R, capacity=R, chunk_entries=N, contains_team=args.team)
+        g = GFSL(R, capacity=R, chunk_entries=N, contains_team=args.team,
+                 contains_blocks_per_sm=args.contains_blocks, update_blocks_per_sm=args.update_blocks)
         prefill_gpu(g, R, pre1, dev)
     def apply_options(h):
         """The run's library options (identical for the timed and the e2e handles)."""
@@ -428,7 +429,8 @@ def run_gpu(args, world, rank, local):
     e2e = None
     if not args.no_e2e and world == 1:
         g.close()  # the timed handle is done: free its pool for the e2e handles
-        g2 = GFSL(R, capacity=R, chunk_entries=N, contains_team=args.team)
+        g2 = GFSL(R, capacity=R, chunk_entries=N, contains_team=args.team,
+                 contains_blocks_per_sm=args.contains_blocks, update_blocks_per_sm=args.update_blocks)
         prefill_gpu(g2, R, pre1, dev)
         apply_options(g2)
         host = [(x[0].cpu().pin_memory(), x[1].cpu().pin_memory(), x[2].cpu().pin_memory())
@@ -450,7 +452,8 @@ def run_gpu(args, world, rank, local):
         # (b) the headline: the K steps back to back through gfsl_batch_host_async, as a
         # user streams batches (copy-in of step j+1 overlaps the kernels of step j), from
         # the first call until every step's results are in host memory; wall clock
-        g3 = GFSL(R, capacity=R, chunk_entries=N, contains_team=args.team)
+        g3 = GFSL(R, capacity=R, chunk_entries=N, contains_team=args.team,
+                 contains_blocks_per_sm=args.contains_blocks, update_blocks_per_sm=args.update_blocks)
         prefill_gpu(g3, R, pre1, dev)
         apply_options(g3)
         out_w = torch.empty(B1, dtype=torch.uint8).pin_memory()
@@ -527,6 +530,10 @@ def main():
     ap.add_argument("--config", default="C2", choices=sorted(CONFIGS))
     ap.add_argument("--team", type=int, default=0)
     ap.add_argument("--chunk", type=int, default=0)
+    ap.add_argument("--contains-blocks", type=int, default=0,
+                    help="cap on Contains-kernel blocks per SM (0 = occupancy default; sweeps)")
+    ap.add_argument("--update-blocks", type=int, default=0,
+                    help="cap on update-kernel blocks per SM (0 = occupancy default; sweeps)")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--validate", action="store_true")
