@@ -160,10 +160,14 @@ gfsl_status gfsl_batch_host(gfsl_t h, const uint8_t *op_types, const uint32_t *k
 
 /*
  * The same, asynchronous: returns once the copies and kernels are enqueued.  The inputs
- * are copied on a library-owned copy stream into one of two device staging slots, so
- * the copy-in of the next batch overlaps the kernels of this one; the batch and the
- * copy-out of the results run on `stream`.  `results` holds the answers once `stream`
- * has reached this point (e.g. after cudaStreamSynchronize).  The host buffers must stay
+ * are copied on a library-owned copy stream into one of two device staging slots, the
+ * kernels run on a library-owned exec stream and the results come back on a
+ * library-owned copy-out stream, so the copy-in of the next batch and the copy-out of
+ * the previous one overlap the kernels of this one.  `stream` is made to wait for the
+ * copy-out: `results` holds the answers once `stream` has reached this point (e.g.
+ * after cudaStreamSynchronize).  The batch itself does not wait for earlier work on
+ * `stream` (its inputs are host memory); it is ordered after the handle's earlier
+ * batches, as every batch is.  The host buffers must stay
  * valid and unmodified until then, and must be pinned (page-locked) for the copies to
  * be asynchronous (pageable buffers still work, with synchronous copies).
  */

@@ -67,8 +67,9 @@ struct gfsl {
   uint32_t *st_key[2] = {nullptr, nullptr}, *st_val[2] = {nullptr, nullptr};
   uint64_t st_cap = 0;
   int st_slot = 0;
-  cudaStream_t copy_stream = nullptr;
+  cudaStream_t copy_stream = nullptr, exec_stream = nullptr, d2h_stream = nullptr;
   cudaEvent_t ev_in[2] = {nullptr, nullptr}, ev_used[2] = {nullptr, nullptr};
+  cudaEvent_t ev_out[2] = {nullptr, nullptr};
   uint64_t batches = 0, ops = 0;
   uint64_t capacity = 0;           // max live keys (gfsl_create)
   uint64_t ops_since_rebuild = 0;  // default rebuild policy (R29)
@@ -409,8 +410,11 @@ static void free_all(gfsl *h) {
     cudaFree(h->st_val[b]);
     if (h->ev_in[b]) cudaEventDestroy(h->ev_in[b]);
     if (h->ev_used[b]) cudaEventDestroy(h->ev_used[b]);
+    if (h->ev_out[b]) cudaEventDestroy(h->ev_out[b]);
   }
   if (h->copy_stream) cudaStreamDestroy(h->copy_stream);
+  if (h->exec_stream) cudaStreamDestroy(h->exec_stream);
+  if (h->d2h_stream) cudaStreamDestroy(h->d2h_stream);
   cudaFree(h->rb.bitmap);
   cudaFree(h->rb.word_prefix);
   cudaFree(h->rb.block_sum);
@@ -795,9 +799,12 @@ extern "C" gfsl_status gfsl_batch(gfsl_t h, const uint8_t *op_types, const uint3
 static gfsl_status ensure_staging(gfsl *h, uint64_t n) {
   if (!h->copy_stream) {
     CK(cudaStreamCreateWithFlags(&h->copy_stream, cudaStreamNonBlocking));
+    CK(cudaStreamCreateWithFlags(&h->exec_stream, cudaStreamNonBlocking));
+    CK(cudaStreamCreateWithFlags(&h->d2h_stream, cudaStreamNonBlocking));
     for (int b = 0; b < 2; ++b) {
       CK(cudaEventCreateWithFlags(&h->ev_in[b], cudaEventDisableTiming));
       CK(cudaEventCreateWithFlags(&h->ev_used[b], cudaEventDisableTiming));
+      CK(cudaEventCreateWithFlags(&h->ev_out[b], cudaEventDisableTiming));
     }
   }
   if (n <= h->st_cap) return GFSL_OK;
@@ -821,10 +828,14 @@ static gfsl_status ensure_staging(gfsl *h, uint64_t n) {
   return GFSL_OK;
 }
 
-// The host-buffer batch, asynchronous: the inputs go to staging slot b on the copy stream
-// (after the kernels of the batch that last used the slot have read it), the batch runs
-// on `stream` once they have arrived, and the results come back on `stream`.  So with
-// pinned host memory the copy-in of the next batch overlaps this batch's kernels.
+// The host-buffer batch, asynchronous, on three library streams: the inputs go to staging
+// slot b on the copy stream (after the kernels of the batch that last used the slot have
+// read it), the kernels run on the exec stream once they have arrived (and once the
+// slot's previous results have left), the results come back on the d2h stream, and
+// `stream` waits for them.  With pinned host memory the copy-in of the next batch and
+// the copy-out of the previous one both overlap this batch's kernels (the kernels of
+// batch i+1 do not queue behind the copy-out of batch i, as they would on `stream`).
+// Batches of one handle stay ordered by the handle's own event (enqueue_batch).
 static gfsl_status batch_host_async(gfsl *h, const uint8_t *op_types, const uint32_t *keys,
                                     const uint32_t *values, uint8_t *results, uint64_t n,
                                     cudaStream_t s) {
@@ -846,11 +857,16 @@ static gfsl_status batch_host_async(gfsl *h, const uint8_t *op_types, const uint
   CK(cudaMemcpyAsync(h->st_key[b], keys, n * 4, cudaMemcpyHostToDevice, c));
   if (values) CK(cudaMemcpyAsync(h->st_val[b], values, n * 4, cudaMemcpyHostToDevice, c));
   CK(cudaEventRecord(h->ev_in[b], c));
-  CK(cudaStreamWaitEvent(s, h->ev_in[b], 0));
-  st = enqueue_batch(h, h->st_op[b], h->st_key[b], values ? h->st_val[b] : nullptr, h->st_res[b], n, s);
+  cudaStream_t k = h->exec_stream, o = h->d2h_stream;
+  CK(cudaStreamWaitEvent(k, h->ev_in[b], 0));
+  CK(cudaStreamWaitEvent(k, h->ev_out[b], 0));  // the slot's previous results have left
+  st = enqueue_batch(h, h->st_op[b], h->st_key[b], values ? h->st_val[b] : nullptr, h->st_res[b], n, k);
   if (st != GFSL_OK) return st;
-  CK(cudaEventRecord(h->ev_used[b], s));
-  CK(cudaMemcpyAsync(results, h->st_res[b], n, cudaMemcpyDeviceToHost, s));
+  CK(cudaEventRecord(h->ev_used[b], k));
+  CK(cudaStreamWaitEvent(o, h->ev_used[b], 0));
+  CK(cudaMemcpyAsync(results, h->st_res[b], n, cudaMemcpyDeviceToHost, o));
+  CK(cudaEventRecord(h->ev_out[b], o));
+  CK(cudaStreamWaitEvent(s, h->ev_out[b], 0));
   return GFSL_OK;
 }
 
