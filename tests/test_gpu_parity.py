@@ -196,6 +196,36 @@ def test_batch_host_async_pipelined():
     check_same_set(g, o)
 
 
+def test_batch_host_async_interleaved_on_caller_stream():
+    """Async host batches (kernels on the library's exec stream, copy-out on its d2h
+    stream) interleaved with device batches, all issued on a caller stream: batches apply
+    in issue order, and synchronising only the caller stream makes every async result
+    visible in host memory (the contract of gfsl_batch_host_async in include/gfsl.h)."""
+    R = 20_000
+    g = GFSL(R)
+    o = OracleMap(R)
+    batches = list(workload_batches(R, 5_003, 8, (20, 20, 60)))
+    side = torch.cuda.Stream()
+    outs, keep = [], []  # inputs stay referenced until the stream is synchronised
+    with torch.cuda.stream(side):
+        for i, (op, key, val) in enumerate(batches):
+            if i % 3 == 1:  # device entry point on the same handle and stream
+                d = [torch.from_numpy(np.ascontiguousarray(a).view(np.int32) if a.dtype == np.uint32 else a).cuda()
+                     for a in (op, key, val)]
+                keep.append(d)
+                outs.append(g.batch(*d, stream=side))
+            else:
+                h = [torch.from_numpy(np.ascontiguousarray(a).view(np.int32) if a.dtype == np.uint32 else a).pin_memory()
+                     for a in (op, key, val)]
+                keep.append(h)
+                outs.append(g.batch_host_async(*h, out=torch.empty(len(op), dtype=torch.uint8).pin_memory(),
+                                               stream=side))
+    side.synchronize()
+    for (op, key, val), out in zip(batches, outs):
+        assert np.array_equal(out.cpu().numpy(), o.batch(op, key, val))
+    check_same_set(g, o)
+
+
 @pytest.mark.parametrize("p", [0.25, 0.5])
 def test_p_chunk_concurrent(p):
     """p_chunk < 1 with the concurrent update kernel and the paper's structure dynamics."""
