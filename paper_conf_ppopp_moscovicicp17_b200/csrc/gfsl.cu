@@ -271,7 +271,11 @@ static void launch_update(gfsl *h, const BatchIn &in, cudaStream_t s, cudaEvent_
   lc.numAttrs = 1;
   lc.stream = s;
   lc.blockDim = dim3(h->cfg.serial_updates ? 32 : 256);
-  lc.gridDim = dim3(h->cfg.serial_updates ? 1 : h->update_grid);
+  // a small batch needs no more warps than it has ops (2 per warp at N = 16, else 1;
+  // 8 warps per block), and never fewer blocks than SMs
+  const uint64_t per_block = N == 16 ? 16 : 8;
+  const uint64_t need = std::max<uint64_t>((uint64_t)h->sms, (in.n + per_block - 1) / per_block);
+  lc.gridDim = dim3(h->cfg.serial_updates ? 1 : (unsigned)std::min<uint64_t>((uint64_t)h->update_grid, need));
   const int serial = h->cfg.serial_updates ? 1 : 0;
   cudaLaunchKernelEx(&lc, update_kernel<N>, h->d, in, h->ctl, update_in(h), serial);
   h->launches += 1;  // update
