@@ -6,10 +6,20 @@ because the exact *structure* (not only the results) is defined for a single tea
 GPU's serial mode (one team applies the batch's updates in op order) must produce the
 same pool, entry for entry, except the lock versions (test_gpu_structure.py).
 
-Pinned by (tests/test_oracle_b.py): the worked examples of Fig 4.1-4.6 (P:287-289,
-P:429) on the fixtures of SURVEY
-Appendix B; Oracle-A's results and final sets on random sequences; its own invariant
-checker; the special case "one chunk holds everything" (a sorted array).
+Pinned by (tests/test_oracle_b.py, tests/test_oracle_b_pins.py): the worked examples of
+Fig 4.1-4.6 on the
+fixtures of SURVEY Appendix B, including the restart of Contains(70) under two injected
+Deletes and the printed intermediate state of the merge write order
+(F = [24, 26, EMPTY, 26]); a hand-worked splitRemove; Oracle-A's results
+and final sets on random sequences; the invariants V1-V12 after every op; the special
+case "one chunk holds everything" (a sorted array).  The B200 design's between-batch
+steps (upkeep R23, rebuild R24, reclamation R25) are pinned by properties checked
+against plain re-derivations written in the tests (not by this model's own code).
+
+What this model does NOT contain: any scheduling policy of the GPU library (the wear
+rule R29 is a GPU-side policy; the model rebuilds only on a fixed period or on demand),
+and any kernel shortcut (a Delete checks every level from the current height, Alg 4.11
+l.12-16, instead of the kernel's start at the level where its snapshot saw k).
 
 Layout (Fig 3.1): chunk = N entries of 64 bits; DATA i = key | value << 32,
 NEXT = max | next << 32, LOCK = state | version << 32.  Internal key = user key + 1;
@@ -58,17 +68,15 @@ def raise_draw(rkey: int, level: int) -> int:
 
 class GFSLModel:
     def __init__(self, N: int, key_range: int, cap_bottom: int, cap_upper: int,
-                 rebuild_every: int = 0, p_chunk_q32: int = 0, rebuild_capacity: int = 0):
+                 rebuild_every: int = 0, p_chunk_q32: int = 0):
         assert N >= 6
         # p_chunk as a 32-bit fraction; 0 = p_chunk = 1 (R16)
         self.p_chunk_q32 = p_chunk_q32
+        # R24: rebuild the upper levels after every k-th batch (0 = never); the GPU's
+        # default wear rule (R29) is a library policy and is not modelled here
         self.rebuild_every = rebuild_every
-        # R29, used if rebuild_every = 0 and rebuild_capacity > 0: rebuild after
-        # the batch at which the ops since the last rebuild reach 5 x min(capacity, ops
-        # submitted up to the last rebuild) (GFSL_REBUILD_DEFAULT_WEAR)
-        self.rebuild_capacity = rebuild_capacity
-        self.ops_total = self.ops_since = self.ops_at_rebuild = 0
         self.batches = 0
+        self.rebuilds = 0       # upper-level rebuilds so far (R24)
         self.dirty = False
         self.free, self.free_taken = [], 0  # R25 free list of reclaimed level-0 chunks
         self.N, self.DSIZE, self.NEXT, self.LOCK, self.MAXL = N, N - 2, N - 2, N - 1, N
@@ -89,9 +97,19 @@ class GFSLModel:
             self.head[l] = c
         self.bump = [1, N - 1]  # [bottom pool, upper pool]
         self.trace = None       # chunks read by the last search (for the worked examples)
+        self.wtrace = None      # list -> every entry write is appended as (chunk, index, entry)
         self.merges = 0         # merges of the current batch (-> upkeep)
+        self.restarts = 0       # searchDown restarts (Alg 4.2 l.25; only under injection)
+        self.check_each_op = False  # run check_invariants() after every op of a batch
+        self.reset_log = set()  # chunks reset to the allocated state since the last snapshot
 
     # ---- chunk accessors ----------------------------------------------------------------
+    def w(self, c, i, e):
+        """One atomic 64-bit entry write (AtomicWrite of Alg 4.7 / 4.9 / 4.12)."""
+        self.pool[c][i] = e
+        if self.wtrace is not None:
+            self.wtrace.append((c, i, e))
+
     def keys(self, c):
         return [K(e) for e in self.pool[c][: self.DSIZE]]
 
@@ -136,10 +154,14 @@ class GFSLModel:
         assert self.state(c) == FREE
         ch = self.pool[c]
         ch[self.LOCK] = E(HELD, V(ch[self.LOCK]))
+        if self.wtrace is not None:
+            self.wtrace.append((c, self.LOCK, ch[self.LOCK]))
 
     def unlock(self, c, state=FREE):
         ch = self.pool[c]
         ch[self.LOCK] = E(state, V(ch[self.LOCK]) + 1)
+        if self.wtrace is not None:
+            self.wtrace.append((c, self.LOCK, ch[self.LOCK]))
 
     def alloc(self, level):  # bump a counter, the chunk is already +inf and locked
         if level == 0 and self.free_taken < len(self.free):  # R25: reclaimed chunks first
@@ -155,16 +177,31 @@ class GFSLModel:
         return i if p else self.cap_upper + i
 
     # ---- search phase (Alg 4.1-4.4 and searchSlow's path, on the snapshot; R1, R21) ------
-    def search(self, k):
-        """Returns (found, path{level: chunk}, top level that held k)."""
-        height = self.height()
+    def search(self, k, hook=None):
+        """searchDown + searchLateral (Alg 4.2-4.4) with searchSlow's path (Alg 4.6).
+        Returns (found, path{level: chunk}, top level that held k).  `hook(chunk)` (tests
+        only) runs before every chunk read, so a test can interleave other operations as a
+        concurrent team would; a backtrack with no prevKv then restarts the traversal from
+        the top (Alg 4.2 l.25), counted in self.restarts.  Within a batch the
+        search runs on the quiescent snapshot (R1) and never restarts."""
+        while True:
+            r = self._search_once(k, hook)
+            if r is not None:
+                return r
+            self.restarts += 1
+
+    def _search_once(self, k, hook):
+        height = self.height()                        # getHeight (P:293)
         cur, level = self.head[height], height
         bt = bt_c = None
         top = 0
         path = {}
-        self.trace = []
+        trace = self.trace = []                       # chunks read by this pass
         while True:
-            self.trace.append(cur)
+            if hook is not None:
+                hook(cur)
+                self.trace = trace
+            trace.append(cur)
             if self.zombie(cur):                      # Alg 4.2 l.9-11
                 cur = self.nxt(cur)
                 continue
@@ -186,8 +223,8 @@ class GFSLModel:
             elif bt is not None:                      # backtrack (l.24-28, 33-38)
                 path[level] = bt_c
                 cur = bt
-            else:                                     # restart (l.25): not on a snapshot
-                raise AssertionError("restart on a quiescent structure")
+            else:                                     # restart (l.25): prevKv is null
+                return None
             level -= 1
             bt = bt_c = None
 
@@ -226,7 +263,7 @@ class GFSLModel:
             return
         self.lock(prev)
         if self.nxt(prev) == z:
-            self.pool[prev][self.NEXT] = E(self.mx(prev), fnz)
+            self.w(prev, self.NEXT, E(self.mx(prev), fnz))
         self.unlock(prev)
 
     def find_and_lock_enclosing(self, c, k, level):
@@ -261,7 +298,7 @@ class GFSLModel:
                 skipped = True
                 continue
             if skipped:  # unlink the zombies from c's NEXT (we hold c)
-                self.pool[c][self.NEXT] = E(self.mx(c), n)
+                self.w(c, self.NEXT, E(self.mx(c), n))
             self.lock(n)
             return n
         return None
@@ -270,11 +307,12 @@ class GFSLModel:
     def execute_insert(self, c, k, v):  # Alg 4.7, Fig 4.3: shift right from insertIdx
         ch = self.pool[c]
         ks = self.keys(c)
-        idx = sum(1 for x in ks if x < k)
-        cnt = self.count(c)
+        idx = sum(1 for x in ks if x < k)             # insertion index (l.3)
         old = ch[:]
-        for t in range(idx, min(cnt, self.DSIZE - 1) + 1):
-            ch[t] = E(k, v) if t == idx else old[t - 1]
+        for t in range(self.DSIZE - 1, idx - 1, -1):  # l.7-10: from DSIZE-1 down to idx
+            ins = E(k, v) if t == idx else old[t - 1]  # l.2: each lane takes its left neighbour
+            if K(ins) != INF:
+                self.w(c, t, ins)
 
     def execute_remove_no_merge(self, c, k):  # P:900-902, Fig 4.6, R13
         ch = self.pool[c]
@@ -282,26 +320,26 @@ class GFSLModel:
         cnt = self.count(c)
         last = self.nxt(c) == NULL
         old = ch[:]
-        for t in range(idx, cnt - 1):
-            ch[t] = old[t + 1]
-        ch[cnt - 1] = EMPTY
-        if idx == cnt - 1 and not last:  # the max follows the largest key
-            ch[self.NEXT] = E(K(old[idx - 1]), V(old[self.NEXT]))
+        if idx == cnt - 1 and not last:  # k was the max: the max field goes first
+            self.w(c, self.NEXT, E(K(old[idx - 1]), V(old[self.NEXT])))
+        for t in range(idx, cnt - 1):    # lanes idx+1 .. cnt-1 write leftwards, ascending
+            self.w(c, t, old[t + 1])
+        self.w(c, cnt - 1, EMPTY)        # the vacated last slot (Q20)
 
     def split(self, level, c):  # Alg 4.9 preSplit + splitCopy (also splitRemove)
         HALF = self.DSIZE // 2
-        pnext = self.lock_next_chunk(c)
+        pnext = self.lock_next_chunk(c)               # preSplit (l.16-21)
         pnew = self.alloc(level)
-        ch, nw = self.pool[c], self.pool[pnew]
+        ch = self.pool[c]
         cnt = self.count(c)
         thresh = K(ch[HALF - 1])
         oldmax = self.mx(c)
-        for t in range(cnt - HALF):
-            nw[t] = ch[t + HALF]
-        nw[self.NEXT] = E(oldmax, NULL if pnext is None else pnext)
-        ch[self.NEXT] = E(thresh, pnew)               # one 64-bit write links the new chunk
+        self.w(pnew, self.NEXT, E(oldmax, NULL if pnext is None else pnext))  # new -> next
+        for t in range(cnt - HALF):                   # splitCopy l.27-28: lanes >= DSIZE/2
+            self.w(pnew, t, ch[t + HALF])
+        self.w(c, self.NEXT, E(thresh, pnew))         # l.30: one 64-bit write links it
         for t in range(HALF, cnt):
-            ch[t] = EMPTY                             # setMovedValsEmpty
+            self.w(c, t, EMPTY)                       # l.32 setMovedValsEmpty
         if pnext is not None:
             self.unlock(pnext)
         self.counter[level] += 1                      # Alg 4.5 l.42 / 4.12 l.18 (R9)
@@ -333,7 +371,7 @@ class GFSLModel:
                 while self.zombie(lc) or self.mx(lc) < km:
                     lc = self.nxt(lc)
                 if self.eq_idx(lc, km) is not None and V(self.pool[upper][ui]) != lc:
-                    self.pool[upper][ui] = E(km, lc)
+                    self.w(upper, ui, E(km, lc))
             self.unlock(upper)
 
     # ---- Insert (Alg 4.5) ---------------------------------------------------------------
@@ -391,12 +429,16 @@ class GFSLModel:
         return True
 
     # ---- Delete (Alg 4.11-4.12) -----------------------------------------------------------
-    def execute_remove_merge(self, e, f, k):
+    def execute_remove_merge(self, e, f, k):  # P:947-951, Fig 4.5c
+        """Every value of e but k moves to f's low slots and f's own entries move right;
+        f is written serially in DESCENDING index order, so after the first write
+        of Fig 4.5c F reads [24, 26, EMPTY, 26]."""
         idx = self.eq_idx(e, k)
         eent = [x for i, x in enumerate(self.pool[e][: self.count(e)]) if i != idx]
         fent = self.pool[f][: self.count(f)]
-        for t, x in enumerate(eent + fent):
-            self.pool[f][t] = x
+        merged = eent + fent
+        for t in range(len(merged) - 1, -1, -1):
+            self.w(f, t, merged[t])
 
     def remove_from_chunk(self, level, pe, k):
         cnt = self.count(pe)
@@ -441,21 +483,19 @@ class GFSLModel:
             c = self.nxt(c)
         return self.eq_idx(c, k) is not None
 
-    def delete(self, k, path, top):
+    def delete(self, k, path, top=None):
+        """Alg 4.11.  `top` (the highest level where the snapshot search saw k) is not
+        used: the paper checks every level from the current height down (l.12-16)."""
         pb = self.find_and_lock_enclosing(path[0], k, 0)  # l.8
-        if self.eq_idx(pb, k) is None:                    # l.9-10 (R15)
+        if self.eq_idx(pb, k) is None:                    # l.9-10 (R15: unlock first)
             self.unlock(pb)
             return False
-        m = top                                           # l.12-16 (R12)
-        if pb != path[0]:  # k moved since the snapshot: it may have been raised as a minK
-            while m + 1 < self.MAXL and self.search_lateral(k, path[m + 1]):
-                m += 1
-        for i in range(m, 0, -1):                         # l.13-20
-            pe = self.find_and_lock_enclosing(path[i], k, i)
-            if self.eq_idx(pe, k) is None:
-                self.unlock(pe)
+        height = self.height()                            # l.12 rereadHeightAndUpdatePath
+        for i in range(height, 0, -1):                    # l.13-20
+            if not self.search_lateral(k, path[i]):       # l.15: containment before locking
                 continue
-            self.remove_from_chunk(i, pe, k)
+            pe = self.find_and_lock_enclosing(path[i], k, i)  # l.18
+            self.remove_from_chunk(i, pe, k)              # l.19
         self.remove_from_chunk(0, pb, k)                  # l.22
         return True
 
@@ -481,7 +521,7 @@ class GFSLModel:
         head_at_start = list(self.head)  # levels above the snapshot height start at head[l]
         self.merges = 0
         for i, op, k, path, top in plans:
-            full = [path[l] if (l <= snap_h and l < PLAN_LEVELS) else head_at_start[l]
+            full = [path[l] if l <= snap_h else head_at_start[l]
                     for l in range(self.N)]
             if op == 1:
                 r = self.insert(k, 0 if vals is None else int(vals[i]), full)
@@ -489,19 +529,14 @@ class GFSLModel:
                 r = self.delete(k, full, top)
             if not r:
                 res[i] = 0
+            if self.check_each_op:
+                bad = self.check_invariants()
+                assert not bad, f"after op {i} ({'insert' if op == 1 else 'delete'} {k - 1}): {bad[:5]}"
         if self.merges:
             self.upkeep()
         if plans:
             self.dirty = True  # a mutating batch since the last rebuild
-        due = False
-        if n and self.rebuild_every:
-            due = (self.batches + 1) % self.rebuild_every == 0
-        elif n and self.rebuild_capacity:
-            self.ops_since += n
-            due = self.ops_since >= 5 * min(self.rebuild_capacity, self.ops_at_rebuild)
-            if due:
-                self.ops_since, self.ops_at_rebuild = 0, self.ops_total + n
-        self.ops_total += n
+        due = bool(n and self.rebuild_every and (self.batches + 1) % self.rebuild_every == 0)
         if due and self.dirty:
             self.rebuild()
             self.reclaim()
@@ -516,17 +551,17 @@ class GFSLModel:
         zombies = [self.cap_upper + i for i in range(self.bump[0]) if self.zombie(self.cap_upper + i)]
         for c in zombies:
             self.pool[c] = [EMPTY] * (self.N - 1) + [HELD]
+            self.reset_log.add(c)
         self.free = self.free[self.free_taken:] + zombies
         self.free_taken = 0
 
     def rebuild_now(self):
-        """gfsl_rebuild (R29): rebuild now if a batch mutated the structure since the last
-        rebuild; the default policy counts again from here."""
+        """gfsl_rebuild: rebuild now if a batch mutated the structure since the last
+        rebuild."""
         if self.dirty:
             self.rebuild()
             self.reclaim()
             self.dirty = False
-        self.ops_since, self.ops_at_rebuild = 0, self.ops_total
 
     def rebuild(self):
         """R24: re-derive levels >= 1 from level 0 between batches ("compact the
@@ -558,6 +593,7 @@ class GFSLModel:
         def chunk(l, j):
             return l - 1 if j == 0 else base[l] + j - 1
 
+        self.rebuilds += 1
         head0, old_used = self.head[0], self.bump[1]
         for l in range(1, N):
             length = 1 if l > top else (n1 + 1 if l == 1 else m[l - 1])
@@ -630,8 +666,38 @@ class GFSLModel:
         kv = self.level_keys(0, with_values=True)
         return [k for k, _ in kv], [v for _, v in kv]
 
-    def check_invariants(self):
-        """The structural invariants (§4.3); returns a list of violations."""
+    def snapshot(self):
+        """State for the cross-batch invariants V6 / V11: every used
+        chunk's max field and the bytes of every zombie."""
+        self.reset_log = set()
+        used = list(range(self.bump[1])) + [self.cap_upper + i for i in range(self.bump[0])]
+        return {"max": {c: self.mx(c) for c in used},
+                "zombie": {c: list(self.pool[c][: self.LOCK]) for c in used if self.zombie(c)},
+                "upper_gen": self.rebuilds}
+
+    def reachable(self):
+        """Every chunk index reachable from the head array through NEXT and down pointers."""
+        seen, stack = set(), [(self.head[l], l) for l in range(self.N)]
+        while stack:
+            c, l = stack.pop()
+            if c == NULL or (c, l) in seen:
+                continue
+            seen.add((c, l))
+            stack.append((self.nxt(c), l))
+            if l > 0:
+                for e in self.pool[c][: self.DSIZE]:
+                    if K(e) != INF:
+                        stack.append((V(e), l - 1))
+        return {c for c, _ in seen}
+
+    def check_invariants(self, prev=None):
+        """The structural invariants of P:203 and §4.3, numbered as in
+        DESIGN.md: V1 sorted chunks, V2 max fields, V3 order between chunks, V4 level l+1
+        keys within level l, V5 down pointers reach their key laterally, V7 no
+        lock held, V8 the last chunk is not a zombie, V9 head chunks start with
+        -inf, V12 every reachable chunk index is allocated; with `prev` (a snapshot()):
+        V6 a max field never increases and V11 a zombie never changes.
+        Returns a list of violations."""
         bad = []
         for l in range(self.N):
             chain = self.level_chain(l)
@@ -661,4 +727,33 @@ class GFSLModel:
                 for k in self.level_keys(l + 1):
                     if k not in lower:
                         bad.append(f"V4 L{l + 1} k{k}")
+            if l > 0:                                     # V5
+                for c in nz:
+                    for e in self.pool[c][: self.DSIZE]:
+                        k = K(e)
+                        if k == INF:
+                            continue
+                        d, hops = V(e), 0
+                        while d != NULL and hops <= self.bump[0] + self.bump[1] and (
+                                self.zombie(d) or self.mx(d) < k):
+                            d, hops = self.nxt(d), hops + 1
+                        if d == NULL or self.eq_idx(d, k) is None:
+                            bad.append(f"V5 L{l} k{k}")
+        used_hi = {0: self.cap_upper + self.bump[0], 1: self.bump[1]}
+        for c in self.reachable():                        # V12
+            if c >= self.cap_upper + self.cap_bottom or (
+                    c >= self.cap_upper and c >= used_hi[0]) or (c < self.cap_upper and c >= used_hi[1]):
+                bad.append(f"V12 c{c}")
+        if prev is not None:
+            same_upper = prev["upper_gen"] == self.rebuilds
+            for c, m in prev["max"].items():              # V6
+                if c in self.reset_log or (c < self.cap_upper and not same_upper):
+                    continue
+                if self.mx(c) > m:
+                    bad.append(f"V6 c{c}")
+            for c, b in prev["zombie"].items():           # V11
+                if c in self.reset_log or (c < self.cap_upper and not same_upper):
+                    continue
+                if list(self.pool[c][: self.LOCK]) != b or not self.zombie(c):
+                    bad.append(f"V11 c{c}")
         return bad

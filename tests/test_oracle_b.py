@@ -107,8 +107,10 @@ def test_single_chunk_is_a_sorted_array():
 def test_model_matches_oracle_a(N):
     R = 400 if N <= 12 else 2000
     m = GFSLModel(N, R, cap_bottom=4000, cap_upper=1000)
+    m.check_each_op = True          # V1-V5, V7-V9, V12 after every Insert / Delete
     o = OracleMap(R)
     w = Workload(R, 150, mix=(35, 35, 30), seed=SEED_BASE + N)
+    snap = m.snapshot()
     for b in range(30):
         op, key, val, _ = w.make_batch(b)
         opn, kn, vn = op.numpy(), key.numpy().astype(np.uint32), val.numpy().astype(np.uint32)
@@ -118,7 +120,9 @@ def test_model_matches_oracle_a(N):
         ks, vs = m.export()
         ok, ov = o.export()
         assert ks == ok.tolist() and vs == ov.tolist()
-        assert m.check_invariants() == []
+        assert m.check_invariants(prev=snap) == []   # + V6 / V11 across the batch
+        snap = m.snapshot()
+    assert m.restarts == 0
 
 
 @pytest.mark.parametrize("N,every", [(6, 1), (12, 2), (16, 1), (32, 3)])
@@ -127,16 +131,18 @@ def test_model_with_rebuild_matches_oracle_a(N, every):
     every invariant; after a rebuild every level-0 chunk is the target of a level-1 key."""
     R = 400 if N <= 12 else 2000
     m = GFSLModel(N, R, cap_bottom=4000, cap_upper=1000, rebuild_every=every)
+    m.check_each_op = True
     o = OracleMap(R)
     w = Workload(R, 150, mix=(35, 35, 30), seed=SEED_BASE + 3 * N)
     for b in range(24):
+        snap = m.snapshot()
         op, key, val, _ = w.make_batch(b)
         opn, kn, vn = op.numpy(), key.numpy().astype(np.uint32), val.numpy().astype(np.uint32)
         assert m.batch(opn.tolist(), kn.tolist(), vn.tolist()) == o.batch(opn, kn, vn).tolist()
         ks, vs = m.export()
         ok, ov = o.export()
         assert ks == ok.tolist() and vs == ov.tolist()
-        assert m.check_invariants() == []
+        assert m.check_invariants(prev=snap) == []
         if (b + 1) % every == 0:
             l0 = [c for c in m.level_chain(0) if not m.zombie(c)][1:]
             targets = {V(e) for c in m.level_chain(1) for e in m.pool[c][: m.DSIZE] if K(e) != INF}
@@ -195,24 +201,3 @@ def test_raise_draw_is_uniform():
     d = np.array([raise_draw(k, lv) for k in range(1, 20001) for lv in range(3)], np.uint64)
     for p in (0.25, 0.5, 0.75):
         assert abs(float((d < int(p * 2**32)).mean()) - p) < 0.01
-
-
-def test_default_rebuild_policy_counts_ops():
-    """R29: with rebuild_every = 0 the model rebuilds after the batch at which the ops
-    since the last rebuild reach 5 x min(capacity, ops submitted up to the last rebuild),
-    then counts again from zero; results and invariants are unchanged."""
-    R, N = 2000, 16
-    m = GFSLModel(N, R, cap_bottom=4000, cap_upper=1000, rebuild_every=0, rebuild_capacity=400)
-    o = OracleMap(R)
-    done = []
-    real = m.rebuild
-    m.rebuild = lambda: (done.append(m.batches), real())[1]
-    w = Workload(R, 150, mix=(35, 35, 30), seed=SEED_BASE + 41)
-    for b in range(12):
-        op, key, val, _ = w.make_batch(b)
-        opn, kn, vn = op.numpy(), key.numpy().astype(np.uint32), val.numpy().astype(np.uint32)
-        assert m.batch(opn.tolist(), kn.tolist(), vn.tolist()) == o.batch(opn, kn, vn).tolist()
-        assert m.check_invariants() == []
-    # 150-op batches: batch 0 (threshold 5 x 0), batch 5 (750 >= 5 x 150), then the
-    # threshold is 5 x min(400, 900) = 2000: not reached by batch 11 (900)
-    assert done == [0, 5]
