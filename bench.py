@@ -1,23 +1,28 @@
 #!/usr/bin/env python3
 """GFSL batched Contains/Insert/Delete benchmark on B200 (BASELINE.json `metric`).
 
-One JSON line on rank 0.  A "step" is one `gfsl_batch` (classify -> Contains kernel ->
-update kernel) over one batch of synthetic ops; `value` is Mops/s over the K timed
-steps (all ops of all ranks / the slowest rank's summed step time).  Inputs are
-resident in HBM before each timed step; L2 is flushed (a 256 MiB write) between steps.
+One JSON line on rank 0.  A "step" is one collective `gfsl_batch` over one global batch of
+synthetic ops (search kernel -> update kernel -> upkeep; with N > 1 GPUs also the route
+kernels and the peer-window exchange); `value` is Mops/s = all ops of the K timed steps /
+the slowest rank's summed CUDA-event step time, averaged over `--runs` independent runs
+(the paper's 10 runs with a 95% CI), each on a freshly prefilled structure with
+the same seeds.  Inputs are resident in HBM before each timed step; L2 is flushed (a
+256 MiB write) before every timed step.
 
-    python bench.py [--config C2] [--gpus N --steps K --warmup W] [--impl reference]
+    python bench.py [--config C5] [--gpus N --steps K --warmup W] [--runs 10] [--impl reference]
 
-Configs: C1, C2 (default: R=1M, 10/10/80, the paper's
-Table 5.1 workload), C2-100, C2-2020, C2-5050, C3, C3-zipf, C4-32, C4-16, C5.
-N>1: weak scaling, each rank owns a key-range shard of the same size as the 1-GPU
-config, every rank draws ops over the whole key space and the batch is routed to the
-owners with NCCL all-to-all.
+Default workload: C5 (BASELINE.json configs[4]): a 1B-key range, 500M keys
+prefilled in random order, 125M-op global batches of [10,10,80] uniform ops.  N > 1 is
+STRONG scaling: the key range stays 1B, shard g owns [g*ceil(R/N), (g+1)*ceil(R/N)) as a
+GFSL over its local key space, each rank issues its 1/N slice of every global batch, and the
+fused route kernels move ops and results through the peers' windows.
+Other configs (C1 .. C4, NEXT-4 workloads): `--config`.
 """
 from __future__ import annotations
 
 import argparse
 import json
+import math
 import os
 import statistics
 import sys
@@ -34,6 +39,8 @@ from paper_conf_ppopp_moscovicicp17_b200.workload import (  # noqa: E402
     SEED_BASE, Workload, prefill_keys, prefill_values)
 
 METRIC = "Mops/s (mixed insert/delete/contains)"
+L2_BYTES = 126 << 20          # B200 L2 (B200_PROFILING.md)
+L2_FLUSH_BYTES = 256 << 20
 
 # name: (R, prefill, batch, n_batches, mix, dist, N)
 # N = chunk entries.  The paper's runs use N = 32; on B200 a chunk read costs L1
@@ -55,19 +62,22 @@ CONFIGS = {
     "M1-1-98": (1_000_000, 500_000, 625_000, 16, (1, 1, 98), "uniform", 16),
     "M5-5-90": (1_000_000, 500_000, 625_000, 16, (5, 5, 90), "uniform", 16),
     "M20-20-60-10M": (10_000_000, 5_000_000, 625_000, 16, (20, 20, 60), "uniform", 16),
-    "INS-1M": (1_000_000, 0, 125_000, 8, (100, 0, 0), "uniform", 16),     # R inserts, empty start
-    "DEL-1M": (1_000_000, 1_000_000, 125_000, 8, (0, 100, 0), "uniform", 16),  # R deletes, full start
+    # Fig 5.4b/c: R Inserts into an EMPTY structure / R Deletes from a FULL one,
+    # as one timed run from the first op (warm-up batches would change the start state)
+    "INS-1M": (1_000_000, 0, 125_000, 8, (100, 0, 0), "perm", 16),
+    "DEL-1M": (1_000_000, 1_000_000, 125_000, 8, (0, 100, 0), "perm", 16),
     # NEXT-1: raw Zipf(0.99) -- mutating keys i.i.d. too (no redraws), so hot keys carry
     # long Insert/Delete chains; run in combining mode (R26), exact for any batch
     "C2-zipf-raw": (1_000_000, 500_000, 625_000, 16, (10, 10, 80), "zipf", 16),
     "C3-zipf-raw": (10_000_000, 5_000_000, 6_250_000, 16, (10, 10, 80), "zipf", 16),
 }
 COMBINE_CONFIGS = {"C2-zipf-raw", "C3-zipf-raw"}
+# single-op configs: every key once, in permutation order, no warm-up batches
+PERM_CONFIGS = {"INS-1M", "DEL-1M"}
 
 
 def combine_mode(args) -> bool:
     return args.config in COMBINE_CONFIGS or getattr(args, "combine", False)
-L2_FLUSH_BYTES = 256 << 20
 
 
 def load_traffic(cfg):
@@ -89,9 +99,21 @@ def load_peaks():
     try:
         with open(p) as f:
             d = json.load(f)
-        return float(d["hbm_gbs"]), "measured"
+        return float(d["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs)"
     except Exception:
-        return 6650.0, "fallback"
+        return 6650.0, "fallback (B200_PROFILING.md)"
+
+
+def ci95(xs):
+    """Mean and the half-width of its 95% confidence interval (Student t)."""
+    n = len(xs)
+    m = statistics.fmean(xs)
+    if n < 2:
+        return m, None
+    t = {2: 12.706, 3: 4.303, 4: 3.182, 5: 2.776, 6: 2.571, 7: 2.447, 8: 2.365, 9: 2.306,
+         10: 2.262, 11: 2.228, 12: 2.201, 16: 2.131, 21: 2.086, 31: 2.042}
+    tv = t.get(n) or min((v for k, v in t.items() if k <= n), default=1.96)
+    return m, tv * statistics.stdev(xs) / math.sqrt(n)
 
 
 class ClockSampler:
@@ -116,6 +138,7 @@ class ClockSampler:
         except Exception:
             self.ok = False
         self._stop = threading.Event()
+        self.t = None
 
     def _run(self):
         while not self._stop.is_set():
@@ -130,14 +153,19 @@ class ClockSampler:
             time.sleep(0.002)
 
     def start(self):
-        if self.ok:
+        if self.ok and self.t is None:
+            self._stop.clear()
             self.t = threading.Thread(target=self._run, daemon=True)
             self.t.start()
 
-    def stop(self):
-        if self.ok:
+    def pause(self):
+        if self.ok and self.t is not None:
             self._stop.set()
             self.t.join()
+            self.t = None
+
+    def result(self):
+        self.pause()
         return {"sm_mhz": statistics.median(self.samples) if self.samples else None,
                 "sm_max_mhz": self.max_mhz, "reasons": sorted(self.reasons),
                 "samples": len(self.samples)}
@@ -149,15 +177,13 @@ def dist_setup(backend="nccl"):
     local = int(os.environ.get("LOCAL_RANK", "0"))
     if backend == "gloo":  # test path: several ranks may share one GPU
         local = local % max(1, torch.cuda.device_count())
+    torch.cuda.set_device(local)
     if world > 1:
         import torch.distributed as dist
-        torch.cuda.set_device(local)
         if backend == "nccl":
             dist.init_process_group("nccl", device_id=torch.device("cuda", local))
         else:
             dist.init_process_group(backend)
-    else:
-        torch.cuda.set_device(local)
     return world, rank, local
 
 
@@ -177,64 +203,189 @@ def max_over_ranks(x: float, world: int) -> float:
     return float(t.item())
 
 
+def slices(n: int, world: int):
+    q, rem = divmod(n, world)
+    out, a = [], 0
+    for r in range(world):
+        b = a + q + (1 if r < rem else 0)
+        out.append((a, b))
+        a = b
+    return out
+
+
+# --------------------------------------------------------------------------------------
+# inputs (seeded, synthetic)
+
+def make_batch(cfg_name, w: Workload, b: int, dev):
+    """Global batch b of the config: (op u8, key i32, val i32) on `dev`."""
+    R, pre, B, nb, mix, dist, N = CONFIGS[cfg_name]
+    if dist == "perm":  # Fig 5.4b/c: every key of [0, R) once, in random order (P:1007)
+        key = prefill_keys(SEED_BASE + 2, R, B, start=b * B, device=dev)
+        op = torch.full((B,), 1 if mix[0] else 2, dtype=torch.uint8, device=dev)
+        val = prefill_values(SEED_BASE + 2, key)
+        return op, key.to(torch.int32), val.to(torch.int32), 0
+    op, key, val, redraws = w.make_batch(b, device=dev)
+    return op.contiguous(), key.to(torch.int32).contiguous(), val.to(torch.int32).contiguous(), redraws
+
+
+def make_inputs(w: Workload, b: int, dev):  # (tools/ compatibility)
+    op, key, val, redraws = w.make_batch(b, device=dev)
+    return op.contiguous(), key.to(torch.int32).contiguous(), val.to(torch.int32).contiguous(), redraws
+
+
+def prefill_gpu(g, R, count, dev, key_lo=0, key_hi=None, seed=SEED_BASE, per_op=False):
+    """Random-order inserts of the first `count` elements of the keyed permutation of
+    [0, R).  Default: ONE insert batch, which the library applies through its bulk path
+    (R34: sorted and merged into level 0, upper levels rebuilt).  per_op=True:
+    the paper's per-op Insert path, in insert-only batches that grow with the structure (a
+    batch never exceeds ~1/4 of the keys present, so concurrent inserts spread over many
+    chunks), then a rebuild.  With [key_lo, key_hi) (a shard), only the keys in the shard
+    are inserted, in the same order, rebased to the shard's local key space (as the route
+    kernels rebase them)."""
+    key_hi = R if key_hi is None else key_hi
+    parts = []
+    for s in range(0, count, 1 << 25):
+        k = prefill_keys(seed, R, min(1 << 25, count - s), start=s, device=dev)
+        if key_lo or key_hi != R:
+            k = k[(k >= key_lo) & (k < key_hi)]
+        parts.append(k)
+    k = torch.cat(parts) if parts else torch.empty(0, dtype=torch.int64, device=dev)
+    del parts
+    v = prefill_values(seed, k).to(torch.int32)
+    k = (k - key_lo).to(torch.int32)
+    cap = (1 << 29) - 1  # GFSL_MAX_BATCH
+    ones = torch.ones(min(k.numel(), cap), dtype=torch.uint8, device=dev)
+    have = 0
+    while have < k.numel():
+        c = min(k.numel() - have, max(4096, have // 4), 1 << 26) if per_op else min(k.numel() - have, cap)
+        g.batch(ones[:c], k[have:have + c], v[have:have + c])
+        have += c
+    del k, v, ones
+    if per_op:
+        g.rebuild()  # bulk-load compaction of the upper levels (gfsl_rebuild, R29)
+    torch.cuda.synchronize()
+
+
 # --------------------------------------------------------------------------------------
 # reference arm / cpu baseline: the oracle as it stands, on this host's cores
 
-def oracle_sample(cfg_name, steps, warmup, budget_s=20.0, per_step_ops=1_000_000, combine=False):
-    """Times Oracle-A on a bounded sample of the config's own batches (1 host thread)."""
+def oracle_sample(cfg_name, steps, warmup, budget_s=20.0, threads=1, combine=False):
+    """Times Oracle-A (the sequential Pugh skiplist, S1 batches) on a bounded sample of the
+    config on `threads` host threads, range-sharded as SURVEY 8(d)(ii): thread t owns a
+    contiguous key range with its own skiplist, and each batch is pre-bucketed by key (the
+    bucketing time is reported separately).  The oracle calls release the GIL (ctypes), so
+    the shards run in parallel.  Sample: the config itself when small; else key-range
+    shards of 2M keys each (one per thread) at the config's prefill density and mix."""
+    from concurrent.futures import ThreadPoolExecutor
     from oracle.oracle_a import OracleMap
     R, pre, B, nb, mix, dist, N = CONFIGS[cfg_name]
-    if pre > 4_000_000:
-        # bounded sample of a big config: one key-range shard of 2M keys with the same
-        # prefill density and the ops that fall into it (DESIGN.md §CPU baseline)
-        shard = 2_000_000
-        Rs = shard
-        pre_s = int(round(pre * shard / R))
-        note = f"key-range shard [0,{shard}) of R={R} at the same fill, same mix"
+    T = max(1, int(threads))
+    if R > 4_000_000:
+        Rs = 2_000_000 * T
+        pre_s = int(round(pre * Rs / R))
+        note = f"key range [0,{Rs}) ({T} shards of 2M keys) of R={R} at the same fill, same mix"
     else:
         Rs, pre_s, note = R, pre, f"the config itself (R={R})"
-    o = OracleMap(Rs)
-    k = prefill_keys(SEED_BASE, Rs, pre_s)
-    o.batch(np.ones(pre_s, np.uint8), k.numpy().astype(np.uint32),
-            prefill_values(SEED_BASE, k).numpy().astype(np.uint32))
-    Bs = min(B, per_step_ops)
-    w = Workload(Rs, Bs, mix=mix, dist=dist, seed=SEED_BASE + 1, dedup=not combine)
+    Bs = min(B, 250_000 * T) if R > 4_000_000 else min(B, 1_000_000)
+    bounds = [(t * Rs // T, (t + 1) * Rs // T) for t in range(T)]
+    maps = [OracleMap(Rs) for _ in range(T)]
+    pool = ThreadPoolExecutor(T)
+    if pre_s:
+        k = prefill_keys(SEED_BASE, Rs, pre_s).numpy()
+        v = prefill_values(SEED_BASE, torch.from_numpy(k)).numpy().astype(np.uint32)
+        k = k.astype(np.uint32)
+        parts = [(k >= lo) & (k < hi) for lo, hi in bounds]
+        list(pool.map(lambda t: maps[t].batch(np.ones(int(parts[t].sum()), np.uint8), k[parts[t]], v[parts[t]]),
+                      range(T)))
+    w = Workload(Rs, Bs, mix=mix, dist="uniform" if dist == "perm" else dist, seed=SEED_BASE + 1,
+                 dedup=not combine)
     batches = []
     for b in range(warmup + steps):
         op, key, val, _ = w.make_batch(b)
         batches.append((op.numpy(), key.numpy().astype(np.uint32), val.numpy().astype(np.uint32)))
+
+    def bucket(batch):
+        op, key, val = batch
+        shard = np.minimum((key.astype(np.int64) * T) // Rs, T - 1)
+        order = np.argsort(shard, kind="stable")
+        cuts = np.searchsorted(shard[order], np.arange(T + 1))
+        return [(op[order[cuts[t]:cuts[t + 1]]], key[order[cuts[t]:cuts[t + 1]]],
+                 val[order[cuts[t]:cuts[t + 1]]]) for t in range(T)], order
+
+    def run(parts):
+        return list(pool.map(lambda t: maps[t].batch(*parts[t], combine=combine), range(T)))
+
     for b in range(warmup):
-        o.batch(*batches[b], combine=combine)
-    t_total, n_total, done = 0.0, 0, 0
+        run(bucket(batches[b])[0])
+    t_total = t_bucket = 0.0
+    n_total = done = 0
     for b in range(warmup, warmup + steps):
         t0 = time.perf_counter()
-        o.batch(*batches[b], combine=combine)
-        t_total += time.perf_counter() - t0
+        parts, _ = bucket(batches[b])
+        t1 = time.perf_counter()
+        run(parts)
+        t2 = time.perf_counter()
+        t_bucket += t1 - t0
+        t_total += t2 - t1
         n_total += Bs
         done += 1
-        if t_total > budget_s:
+        if t_total + t_bucket > budget_s:
             break
-    o.close()
+    pool.shutdown()
+    for m in maps:
+        m.close()
     mops = n_total / t_total / 1e6
-    return mops, t_total, done, Bs, note
+    return {"mops": mops, "mops_incl_bucketing": n_total / (t_total + t_bucket) / 1e6,
+            "seconds": t_total, "bucket_seconds": t_bucket, "batches": done, "batch_ops": Bs,
+            "threads": T, "note": note}
+
+
+def cpu_info():
+    model = None
+    try:
+        with open("/proc/cpuinfo") as f:
+            for line in f:
+                if line.startswith("model name"):
+                    model = line.split(":", 1)[1].strip()
+                    break
+    except Exception:
+        pass
+    return {"nproc": os.cpu_count(), "model": model}
+
+
+def cpu_baseline_obj(cfg, steps, combine, budget_each=12.0):
+    T = os.cpu_count() or 1
+    mt = oracle_sample(cfg, min(steps, 16), 1, budget_s=budget_each, threads=T, combine=combine)
+    st = oracle_sample(cfg, min(steps, 16), 1, budget_s=budget_each / 2, threads=1, combine=combine)
+    return {"value": round(mt["mops"], 4), "unit": "Mops/s", "cores": mt["threads"], "kind": "oracle",
+            "sample": (f"{mt['batches']} batches of {mt['batch_ops']} ops ({mt['seconds']:.1f} s) on "
+                       f"{mt['threads']} threads, range-sharded Oracle-A (sequential Pugh skiplist, S1 "
+                       f"batches) per thread; {mt['note']}; bucketing by key range excluded "
+                       f"({mt['bucket_seconds']:.2f} s; incl. it {mt['mops_incl_bucketing']:.2f} Mops/s)"),
+            "single_thread": {"value": round(st["mops"], 4), "cores": 1,
+                              "sample": f"{st['batches']} batches of {st['batch_ops']} ops; {st['note']}"},
+            "cpu": cpu_info()}
 
 
 def run_reference(args, world, rank):
-    cfg = args.config
     if rank != 0:
         return
-    mops, t, done, Bs, note = oracle_sample(cfg, args.steps, args.warmup, budget_s=60.0,
-                                            combine=combine_mode(args))
+    cfg = args.config
+    T = os.cpu_count() or 1
+    r = oracle_sample(cfg, args.steps, args.warmup, budget_s=60.0, threads=T, combine=combine_mode(args))
     line = {
-        "impl": "reference", "metric": METRIC, "value": round(mops, 4), "unit": "Mops/s",
-        "n_gpus": args.gpus, "steps": done, "warmup": args.warmup,
-        "ms_per_step": round(1000 * t / max(done, 1), 3), "higher_is_better": True,
-        "scaling": "weak", "vs_baseline": None, "dtype": "u32", "data": "synthetic",
-        "config": {"workload": cfg, "batch_ops_sampled": Bs},
-        "cpu_baseline": {"value": round(mops, 4), "unit": "Mops/s", "cores": 1,
+        "impl": "reference", "metric": METRIC, "value": round(r["mops"], 4), "unit": "Mops/s",
+        "n_gpus": args.gpus, "steps": r["batches"], "warmup": args.warmup,
+        "ms_per_step": round(1000 * r["seconds"] / max(r["batches"], 1), 3), "higher_is_better": True,
+        "scaling": "strong", "vs_baseline": None, "dtype": "u32", "data": "synthetic",
+        "config": {"workload": cfg, "batch_ops_sampled": r["batch_ops"]},
+        "cpu_baseline": {"value": round(r["mops"], 4), "unit": "Mops/s", "cores": r["threads"],
                          "kind": "oracle",
-                         "sample": f"{done} batches of {Bs} ops; {note}; Oracle-A (sequential Pugh skiplist, S1 batches)"},
-        "e2e": {"value": round(mops, 4), "unit": "Mops/s", "h2d_bytes_per_step": 0,
+                         "sample": (f"{r['batches']} batches of {r['batch_ops']} ops on {r['threads']} "
+                                    f"threads, range-sharded Oracle-A (sequential Pugh skiplist, S1 "
+                                    f"batches); {r['note']}"),
+                         "cpu": cpu_info()},
+        "e2e": {"value": round(r["mops"], 4), "unit": "Mops/s", "h2d_bytes_per_step": 0,
                 "d2h_bytes_per_step": 0},
     }
     print(json.dumps(line), flush=True)
@@ -243,293 +394,350 @@ def run_reference(args, world, rank):
 # --------------------------------------------------------------------------------------
 # GPU arm
 
-def make_inputs(w: Workload, b: int, dev):
-    op, key, val, redraws = w.make_batch(b, device=dev)
-    return op.contiguous(), key.to(torch.int32).contiguous(), val.to(torch.int32).contiguous(), redraws
+class Setup:
+    """The run's handle factory: one GFSL (N = 1) or this rank's shard of a range-sharded
+    GFSL with the fused peer-window exchange (default) or the NCCL all-to-all router."""
+
+    def __init__(self, args, world, rank, dev):
+        self.args, self.world, self.rank, self.dev = args, world, rank, dev
+        R, pre, B, nb, mix, dist, N = CONFIGS[args.config]
+        self.N = args.chunk or N
+        self.R, self.pre, self.B = R, pre, B
+        from paper_conf_ppopp_moscovicicp17_b200.router import shard_bounds
+        self.lo, self.hi, _ = shard_bounds(R, world, rank) if world > 1 else (0, R, R)
+        self.sl = slices(B, world)[rank]
+        self.max_slice = max(b - a for a, b in slices(B, world))
+
+    def create(self):
+        a, kw = self.args, dict(chunk_entries=self.N, contains_team=self.args.team,
+                                 contains_blocks_per_sm=self.args.contains_blocks,
+                                 update_blocks_per_sm=self.args.update_blocks)
+        if self.world > 1 and a.exchange == "peer":
+            from paper_conf_ppopp_moscovicicp17_b200.router import PeerShardedGFSL
+            g = PeerShardedGFSL(self.R, self.rank, self.world, max_slice=self.max_slice, **kw)
+            local = g.local
+        elif self.world > 1:
+            from paper_conf_ppopp_moscovicicp17_b200.router import ShardedGFSL
+            g = ShardedGFSL(self.R, self.rank, self.world, **kw)
+            local = g.local
+        else:
+            from paper_conf_ppopp_moscovicicp17_b200.gfsl import GFSL
+            g = GFSL(self.R, capacity=self.R, **kw)
+            local = g
+        if self.pre:
+            prefill_gpu(local, self.R, self.pre, self.dev, key_lo=self.lo, key_hi=self.hi,
+                        per_op=self.args.prefill == "per-op")
+        local.configure(bulk={"auto": 0, "off": 1, "always": 2}[a.bulk],
+                        combine=1 if combine_mode(a) else 0,
+                        p_chunk_q32=max(1, int(a.p_chunk * 2**32)) if a.p_chunk < 1.0 else 0,
+                        l2_window=a.l2_window, no_pdl=1 if a.no_pdl else 0,
+                        rebuild_every=0xFFFFFFFF if a.rebuild_every < 0 else a.rebuild_every)
+        barrier(self.world)
+        return g, local
+
+    @staticmethod
+    def close(g):
+        if hasattr(g, "xr"):
+            g.xr.close()
+        (g.local if hasattr(g, "local") else g).close()
+        torch.cuda.synchronize()
 
 
-def prefill_gpu(g, R, count, dev, chunk=1 << 24, key_lo=0, seed=SEED_BASE):
-    """Random-order inserts in insert-only batches that grow with the structure
-    (a batch never exceeds ~1/4 of the keys already present, so concurrent inserts spread
-    over many chunks instead of queueing on the few chunks of a small structure)."""
-    s = 0
-    while s < count:
-        c = min(chunk, count - s, max(4096, s // 4))
-        k = prefill_keys(seed, R, c, start=s, device=dev) + key_lo
-        v = prefill_values(seed, k)
-        g.batch(torch.ones(c, dtype=torch.uint8, device=dev), k.to(torch.int32),
-                v.to(torch.int32))
-        s += c
-    g.rebuild()  # bulk-load compaction (gfsl_rebuild, R29), as a user would after a load
-    torch.cuda.synchronize()
-
-
-def run_gpu(args, world, rank, local):
-    from paper_conf_ppopp_moscovicicp17_b200.gfsl import GFSL
-    dev = torch.device("cuda", local)
-    R1, pre1, B1, nb, mix, dist, N = CONFIGS[args.config]
-    if args.chunk:
-        N = args.chunk
+def run_gpu(args, world, rank, local_rank):
+    dev = torch.device("cuda", local_rank)
+    S = Setup(args, world, rank, dev)
+    R, pre, B, nb, mix, dist, N0 = CONFIGS[args.config]
+    N = S.N
+    perm_cfg = args.config in PERM_CONFIGS
     steps = args.steps if args.steps else nb
-    W = args.warmup
+    W = 0 if perm_cfg else args.warmup
     hbm_peak, peak_kind = load_peaks()
+    PROF = 0 if perm_cfg else 3  # extra batches after the timed region, for the per-kernel breakdown
+    a, b_ = S.sl
 
-    # weak scaling: each rank owns a shard of R1 keys and issues B1 ops per step
-    R = R1 * world
-    if world > 1 and args.exchange == "peer":
-        # fused exchange (NEXT-3): route kernels store/load straight through peer windows
-        from paper_conf_ppopp_moscovicicp17_b200.router import PeerShardedGFSL
-        g = PeerShardedGFSL(R, rank, world, max_slice=B1, capacity=R1, chunk_entries=N,
-                            contains_team=args.team)
-        lo = g.key_lo
-        prefill_gpu(g.local, R1, pre1, dev, key_lo=lo, seed=SEED_BASE + 1000 * rank)
-    elif world > 1:
-        from paper_conf_ppopp_moscovicicp17_b200.router import ShardedGFSL
-        g = ShardedGFSL(R, rank, world, capacity=R1, chunk_entries=N,
-                        contains_team=args.team)
-        lo = g.key_lo
-        prefill_gpu(g.local, R1, pre1, dev, key_lo=lo, seed=SEED_BASE + 1000 * rank)
-    else:
-        g = GFSL(R, capacity=R, chunk_entries=N, contains_team=args.team,
-                 contains_blocks_per_sm=args.contains_blocks, update_blocks_per_sm=args.update_blocks)
-        prefill_gpu(g, R, pre1, dev)
-    def apply_options(h):
-        """The run's library options (identical for the timed and the e2e handles)."""
-        h.configure(combine=1 if combine_mode(args) else 0,
-                    p_chunk_q32=int(args.p_chunk * 2**32) if args.p_chunk < 1.0 else 0,
-                    l2_window=1 if args.l2_window else 0, no_pdl=1 if args.no_pdl else 0,
-                    rebuild_every=0xFFFFFFFF if args.rebuild_every < 0 else args.rebuild_every)
-
-    apply_options(g.local if world > 1 else g)
-    PROF = 3  # extra batches after the timed region, for the per-kernel breakdown
-    w = Workload(R, B1, mix=mix, dist=dist, seed=SEED_BASE + 1 + 7919 * rank,
+    # the global batches (same seeds on every rank); this rank keeps its slice
+    w = Workload(R, B, mix=mix, dist="uniform" if dist == "perm" else dist, seed=SEED_BASE + 1,
                  dedup=not combine_mode(args))
-    inputs = [make_inputs(w, b, dev) for b in range(W + steps + PROF)]
-    redraws = sum(x[3] for x in inputs)
+    inputs, redraws = [], 0
+    for b in range(W + steps + PROF):
+        op, key, val, rd = make_batch(args.config, w, b, dev)
+        inputs.append((op[a:b_].contiguous(), key[a:b_].contiguous(), val[a:b_].contiguous()))
+        redraws += rd
+        del op, key, val
+    n_local = b_ - a
     flush = torch.empty(L2_FLUSH_BYTES, dtype=torch.uint8, device=dev)
     stream = torch.cuda.current_stream()
+    clocks = ClockSampler(local_rank)
 
-    for b in range(W):
-        g.batch(*inputs[b][:3])
-    torch.cuda.synchronize()
-    barrier(world)
-    local_g = g.local if world > 1 else g
-    st0 = local_g.stats()
-    mut0 = st0["mutations"]
+    runs_mops, runs_ms, launches, lib_launches, wall_total = [], [], 0, 0, 0.0
+    extras = {}
+    # single-op configs start from a fixed state, so their warm-up is one whole untimed run
+    # of the sequence on a throwaway handle (run -1)
+    for run in range(-1 if perm_cfg else 0, args.runs):
+        g, local_g = S.create()
+        for b in range(W):
+            g.batch(*inputs[b])
+        torch.cuda.synchronize()
+        st0 = local_g.stats()
+        starts = [torch.cuda.Event(enable_timing=True) for _ in range(steps)]
+        ends = [torch.cuda.Event(enable_timing=True) for _ in range(steps)]
+        barrier(world)
+        torch.cuda.synchronize()
+        clocks.start()
+        wall0 = time.perf_counter()
+        for j in range(steps):
+            flush.zero_()  # L2 flush between timed steps (outside the step's events)
+            starts[j].record(stream)
+            g.batch(*inputs[W + j])
+            ends[j].record(stream)
+        torch.cuda.synchronize()
+        barrier(world)
+        clocks.pause()
+        if run < 0:
+            S.close(g)
+            continue
+        wall_total += time.perf_counter() - wall0
+        local_ms = sum(s.elapsed_time(e) for s, e in zip(starts, ends))
+        total_ms = max_over_ranks(local_ms, world)
+        runs_ms.append(total_ms)
+        runs_mops.append(B * steps / (total_ms / 1e3) / 1e6)
+        st_t = local_g.stats()
+        if run == 0:
+            extras = run_extras(args, S, g, local_g, inputs, W, steps, PROF, st0, st_t, flush, dev)
+            # our kernels launched inside the timed region (counted by libgfsl at enqueue),
+            # plus the route/exchange kernels: peer exchange 3 plan + counts + wait + push +
+            # arrive + wait + arrive + wait + pull per step; NCCL router 3 plan + pack + unpack
+            route_k = (11 if args.exchange == "peer" else 5) if world > 1 else 0
+            launches = int(st_t["kernel_launches"] - st0["kernel_launches"]) + route_k * steps
+            lib_launches = int(st_t["library_launches"] - st0["library_launches"])
+        S.close(g)
 
-    starts = [torch.cuda.Event(enable_timing=True) for _ in range(steps)]
-    ends = [torch.cuda.Event(enable_timing=True) for _ in range(steps)]
-    clocks = ClockSampler(local)
-    barrier(world)
-    torch.cuda.synchronize()
-    clocks.start()
-    wall0 = time.perf_counter()
-    for j in range(steps):
-        flush.zero_()  # L2 flush between timed steps (outside the step's events)
-        starts[j].record(stream)
-        g.batch(*inputs[W + j][:3])
-        ends[j].record(stream)
-    torch.cuda.synchronize()
-    wall = time.perf_counter() - wall0
-    barrier(world)
-    clk = clocks.stop()
-    step_ms = [s.elapsed_time(e) for s, e in zip(starts, ends)]
-    local_ms = sum(step_ms)
-    total_ms = max_over_ranks(local_ms, world)
-    ops_total = B1 * steps * world
-    mops = ops_total / (total_ms / 1e3) / 1e6
-    st_t = local_g.stats()
-    n_mut = (st_t["mutations"] - mut0) / max(steps, 1)
-    # our kernels launched inside the timed region (counted by libgfsl at enqueue), plus the
-    # route kernels of the multi-GPU path: NCCL exchange 3 plan + pack + unpack per step;
-    # peer exchange 3 plan + counts + push + 2 barriers + pull per step
-    route_k = (8 if args.exchange == "peer" else 5) if world > 1 else 0
-    launches = int(st_t["kernel_launches"] - st0["kernel_launches"]) + route_k * steps
-    lib_launches = int(st_t["library_launches"] - st0["library_launches"])
-    # per-kernel breakdown: CUDA events between the kernels of PROF extra batches (events
-    # between kernels would defeat the programmatic dependent launch of the timed steps)
-    local_g.configure(profile_phases=1)
-    local_g.phase_times()
-    for j in range(PROF):
-        flush.zero_()
-        g.batch(*inputs[W + steps + j][:3])
-    torch.cuda.synchronize()
-    phases, nbat = local_g.phase_times()
-    local_g.configure(profile_phases=0)
+    mean_mops, half = ci95(runs_mops)
+    mean_ms = statistics.fmean(runs_ms)
+    clk = clocks.result()
 
-    # algorithmic bytes: chunk reads per Contains op, counted on a Contains-only replay
-    # of the last timed batch's keys (untimed, non-mutating)
+    e2e = None
+    if not args.no_e2e:
+        e2e = run_e2e(args, S, inputs, W, steps, world, dev)
+
+    cpu = None
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+        cpu = cpu_baseline_obj(args.config, steps, combine_mode(args))
+
+    if rank == 0:
+        ex = extras
+        line = {
+            "metric": METRIC, "value": round(mean_mops, 3), "unit": "Mops/s", "n_gpus": world,
+            "steps": steps, "warmup": W if not perm_cfg else "one untimed run of the whole sequence",
+            "ms_per_step": round(mean_ms / steps, 4),
+            "higher_is_better": True, "scaling": "strong", "vs_baseline": None,
+            "dtype": "u32", "data": "synthetic",
+            "runs": {"n": len(runs_mops), "mean": round(mean_mops, 3),
+                     "ci95_half_width": None if half is None else round(half, 3),
+                     "values": [round(x, 2) for x in runs_mops],
+                     "how": "each run: a fresh handle, the same seeded prefill, W warm-up and K timed steps "
+                            "(the paper's 10 runs with a 95% CI, P:1009)"},
+            "config": {"workload": args.config, "key_range": R,
+                       "rebuild_every": "never" if args.rebuild_every < 0 else (args.rebuild_every or "default: ops since the last rebuild >= 5 x min(capacity, ops up to it) (R29)"),
+                       "prefill": pre, "batch_ops": B, "mix_ins_del_con": list(mix), "keys": dist,
+                       "semantics": "combining (R26): mutations in input order, any batch" if combine_mode(args)
+                       else "S1 snapshot, <=1 mutation per key (R1/R2)",
+                       "chunk_entries": N, "p_chunk": args.p_chunk, "contains_team": ex.get("contains_team"),
+                       "prefill_path": ("one batch through the bulk path (R34)" if args.prefill == "bulk"
+                                        else "per-op Inserts in growing batches + rebuild"),
+                       "bulk_timed": args.bulk,
+                       "l2": "flushed (256 MiB write) between timed steps",
+                       "parallelism": f"range-shard x{world} (strong: global R and batch fixed)" if world > 1 else "1 GPU",
+                       "exchange": (("peer windows (CUDA IPC, fused route kernels, device-side counts)"
+                                     if args.exchange == "peer" else "NCCL all-to-all") if world > 1 else None)},
+            "roofline": ex.get("roofline"),
+            "roofline_kernels": ex.get("roofline_kernels"),
+            "search_gathers": ex.get("gather"),
+            "random_access_roofline": ex.get("rand"),
+            "structure": ex.get("structure"),
+            "mutations_per_step": ex.get("n_mut"),
+            "phase_ms_per_step": ex.get("phases"),
+            "chunk_reads_per_contains": ex.get("reads"),
+            "chunk_reads_l0_per_contains": ex.get("reads_l0"),
+            "cpu_baseline": cpu,
+            "e2e": e2e,
+            "gpu_launches": launches,
+            "library_launches": lib_launches,  # CUB radix-sort kernels (combining mode only)
+            "clocks": clk,
+            "wall_s_timed_region": round(wall_total, 4),
+            "generator_redraws": int(redraws),
+            "validate": ex.get("validate"),
+        }
+        print(json.dumps(line), flush=True)
+
+
+def run_extras(args, S, g, local_g, inputs, W, steps, PROF, st0, st_t, flush, dev):
+    """Run 0's measurements after its timed region: per-kernel phase times (CUDA events
+    between the kernels of PROF extra batches), chunk reads per Contains (counting build,
+    untimed Contains-only replay), the structure's level sizes, the roofline objects, and
+    the validator when asked."""
+    world, rank = S.world, S.rank
+    N = S.N
     Cb = N * 8
+    hbm_peak, peak_kind = load_peaks()
+    n_mut = (st_t["mutations"] - st0["mutations"]) / max(steps, 1)
+    phases, nbat = {"intake": 0, "contains": 0, "update": 0, "upkeep": 0}, 0
+    if PROF:
+        local_g.configure(profile_phases=1)
+        local_g.phase_times()
+        for j in range(PROF):
+            flush.zero_()
+            g.batch(*inputs[W + steps + j])
+        torch.cuda.synchronize()
+        phases, nbat = local_g.phase_times()
+        local_g.configure(profile_phases=0)
+    # chunk reads per Contains: a Contains-only replay of the last batch's keys of this shard
     local_g.configure(count_reads=1)
-    st0 = local_g.stats()
-    key_last = inputs[W + steps + PROF - 1][1]
-    if world > 1:
-        key_last = key_last[(key_last >= g.key_lo) & (key_last < g.key_hi)].contiguous()
-    local_g.batch(torch.zeros(key_last.numel(), dtype=torch.uint8, device=dev), key_last)
+    c0 = local_g.stats()
+    key_last = inputs[-1][1].to(torch.int64)
+    if world > 1:  # the keys of this rank's slice that fall in its own shard, rebased
+        key_last = key_last[(key_last >= S.lo) & (key_last < S.hi)] - S.lo
+    key_last = key_last.to(torch.int32).contiguous()
+    if key_last.numel():
+        local_g.batch(torch.zeros(key_last.numel(), dtype=torch.uint8, device=dev), key_last)
     torch.cuda.synchronize()
-    st1 = local_g.stats()
+    c1 = local_g.stats()
     local_g.configure(count_reads=0)
-    cops = max(1, st1["contains_ops"] - st0["contains_ops"])
-    reads_per_op = (st1["contains_reads"] - st0["contains_reads"]) / cops
-    reads_l0_per_op = (st1["contains_reads_l0"] - st0["contains_reads_l0"]) / cops
+    cops = max(1, c1["contains_ops"] - c0["contains_ops"])
+    reads = (c1["contains_reads"] - c0["contains_reads"]) / cops
+    reads_l0 = (c1["contains_reads_l0"] - c0["contains_reads_l0"]) / cops
+    meta = local_g.meta()
+    l0_bytes = max(0, meta["counters"][0]) * Cb
+    l1_bytes = max(0, meta["counters"][1]) * Cb
+    # ops the search kernel of this rank handles per launch (uniform routing: ~B/world)
+    n_search = S.B / world
+    nb = max(nbat, 1)
+    c_ms, u_ms = phases["contains"] / nb, phases["update"] / nb
+    i_ms, k_ms = phases["intake"] / nb, phases["upkeep"] / nb
 
-    n_search = B1  # the search kernel traverses every valid op of the batch
-    c_ms = phases["contains"] / max(nbat, 1)
-    u_ms = phases["update"] / max(nbat, 1)
-    i_ms = phases["intake"] / max(nbat, 1)
-    k_ms = phases["upkeep"] / max(nbat, 1)
-
-    def roof(bytes_per_launch, ms, kernel):
-        if ms <= 0 or bytes_per_launch <= 0:
-            return None
-        ach = bytes_per_launch / (ms / 1e3) / 1e9
-        return {"bound": "hbm", "achieved": round(ach, 1), "peak": hbm_peak, "unit": "GB/s",
-                "frac": round(ach / hbm_peak, 4), "traffic": None, "peak_kind": peak_kind,
-                "kernel": kernel, "algorithmic_bytes_per_launch": int(bytes_per_launch)}
-    # search kernel: SURVEY 8(d) -- the compulsory DRAM bytes of a traversal are its
-    # bottom-level chunk gathers (upper levels are cache-resident): L0 reads x C_b
-    s_bytes = n_search * reads_l0_per_op * Cb
-    # update kernel: per mutation one chunk read under the lock + the entries written
-    u_bytes = n_mut * (Cb + 8 * (N // 2 + 2))
-    roof_c = roof(s_bytes, c_ms, "search")
-    roof_u = roof(u_bytes, u_ms, "update")
-    traffic, tsrc = load_traffic(args.config) if world == 1 else ({}, None)
-    for r, kname in ((roof_c, "search"), (roof_u, "update")):
-        if r is not None and traffic.get(kname) is not None:
-            r["traffic"] = int(traffic[kname])
-            r["traffic_source"] = f"profiles/{tsrc} (ncu, one launch of this config)"
-    roofline = roof_c if c_ms >= u_ms else roof_u
-    # B6 (SURVEY 8(d)): achievable random-access throughput for this chunk size, measured
-    # now on this GPU -- the denominator of the north star's ">= 40%" target
+    # Which level of the hierarchy bounds the search kernel (SURVEY 8(d)): HBM once level 0
+    # no longer fits the L2; then the compulsory bytes are the level-0 gathers plus the
+    # level-1 gathers that miss (level 1 resident for the fraction L2 / its size).
+    resident = l0_bytes <= L2_BYTES
+    miss1 = 0.0 if l1_bytes <= L2_BYTES else 1.0 - L2_BYTES / l1_bytes
+    upper = max(0.0, reads - reads_l0)
     rand = None
     if not args.no_ubench and rank == 0:
         from paper_conf_ppopp_moscovicicp17_b200.gfsl import ubench
         r_hbm, t_hbm = ubench(Cb, 16 << 30)
         r_l2, t_l2 = ubench(Cb, 32 << 20)
         rand = {"block_bytes": Cb, "R_rand_hbm_GBps": round(r_hbm, 1), "R_rand_l2_GBps": round(r_l2, 1),
-                "chase_latency_hbm_ns": round(t_hbm, 1), "chase_latency_l2_ns": round(t_l2, 1)}
-        for r in (roof_c, roof_u):
-            if r is not None:
-                r["frac_of_random_access_peak"] = round(r["achieved"] / r_hbm, 4)
-                if r.get("traffic"):
-                    ms_k = c_ms if r["kernel"] == "search" else u_ms
-                    r["dram_GBps_measured_traffic"] = round(r["traffic"] / (ms_k / 1e3) / 1e9, 1)
-                    r["frac_traffic_of_random_access_peak"] = round(r["dram_GBps_measured_traffic"] / r_hbm, 4)
-    gather = {"chunk_gathers_per_op": round(reads_per_op, 3),
-              "gather_GBps": round(n_search * reads_per_op * Cb / (c_ms / 1e3) / 1e9, 1) if c_ms > 0 else None,
-              "note": "all chunk gathers of the search kernel incl. L1/L2-resident upper levels"}
+                "chase_latency_hbm_ns": round(t_hbm, 1), "chase_latency_l2_ns": round(t_l2, 1),
+                "how": "gfsl_ubench: random aligned chunk-size gathers over 16 GiB (32 MiB for L2), the "
+                       "search kernel's team shape, 4/8/16 gathers in flight per team (best kept)"}
+    if resident:
+        bound, peak, pk = "l2", (rand["R_rand_l2_GBps"] if rand else None), "measured R_rand_l2 (gfsl_ubench)"
+        s_bytes = n_search * reads * Cb
+        bytes_note = "every chunk gather (all levels) x C_b: the structure is L2-resident"
+    else:
+        bound, peak, pk = "hbm", hbm_peak, peak_kind
+        s_bytes = n_search * (reads_l0 + upper * miss1) * Cb
+        bytes_note = ("(level-0 gathers + upper-level gathers x the level-1 miss fraction "
+                      f"{miss1:.3f} = 1 - L2/level-1 bytes) x C_b per op (SURVEY 8(d))")
+    u_bytes = n_mut * (Cb + 8 * (N // 2 + 2))
+    traffic, tsrc = load_traffic(args.config) if world == 1 else ({}, None)
 
+    def roof(bytes_per_launch, ms, kernel, note):
+        if ms <= 0 or bytes_per_launch <= 0 or not peak:
+            return None
+        ach = bytes_per_launch / (ms / 1e3) / 1e9
+        r = {"bound": bound, "achieved": round(ach, 1), "peak": peak, "unit": "GB/s",
+             "frac": round(ach / peak, 4), "traffic": None, "peak_kind": pk, "kernel": kernel,
+             "algorithmic_bytes_per_launch": int(bytes_per_launch), "algorithmic_bytes": note,
+             "launch_ms": round(ms, 4)}
+        t = traffic.get(kernel)
+        if t is not None:
+            r["traffic"] = int(t)
+            r["traffic_source"] = f"profiles/{tsrc} (ncu dram__bytes_read.sum + dram__bytes_write.sum, one launch)"
+            r["traffic_GBps"] = round(t / (ms / 1e3) / 1e9, 1)
+        if rand and bound == "hbm":
+            r["frac_of_random_access_peak"] = round(ach / rand["R_rand_hbm_GBps"], 4)
+        return r
+
+    roof_c = roof(s_bytes, c_ms, "search", bytes_note)
+    roof_u = roof(u_bytes, u_ms, "update", "per mutation: the chunk read under the lock + the entries "
+                                           "written, C_b + 8 (N/2 + 2) B")
+    roofline = roof_c if c_ms >= u_ms else roof_u
+    gather = {"chunk_gathers_per_op": round(reads, 3),
+              "gather_GBps": round(n_search * reads * Cb / (c_ms / 1e3) / 1e9, 1) if c_ms > 0 else None,
+              "note": "all chunk gathers of the search kernel incl. cache-resident upper levels"}
     rep = None
     if args.validate:
         rep_obj, _, _ = local_g.validate(export=False)
         rep = {"keys": rep_obj.keys, "height": rep_obj.height, "violations": rep_obj.violations}
-    contains_team = local_g.cfg.contains_team or (4 if N == 32 else 2)
+    return {
+        "roofline": roofline, "roofline_kernels": {"search": roof_c, "update": roof_u},
+        "gather": gather, "rand": rand, "n_mut": round(n_mut, 1), "reads": round(reads, 3),
+        "reads_l0": round(reads_l0, 3), "validate": rep,
+        "phases": {"intake": round(i_ms, 4), "search": round(c_ms, 4), "update": round(u_ms, 4),
+                   "upkeep_rebuild": round(k_ms, 4)},
+        "structure": {"level0_chunks": meta["counters"][0], "level1_chunks": meta["counters"][1],
+                      "level0_MB": round(l0_bytes / 2**20, 1), "level1_MB": round(l1_bytes / 2**20, 1),
+                      "height": max([l for l in range(1, 32) if meta["counters"][l] > 0], default=0),
+                      "l2_MB": L2_BYTES >> 20, "shard": [S.lo, S.hi] if world > 1 else None},
+        "contains_team": local_g.cfg.contains_team or (4 if N == 32 else 2),
+    }
 
-    # end to end through the C ABI with host buffers (fresh handle, same sequence)
-    e2e = None
-    if not args.no_e2e and world == 1:
-        g.close()  # the timed handle is done: free its pool for the e2e handles
-        g2 = GFSL(R, capacity=R, chunk_entries=N, contains_team=args.team,
-                 contains_blocks_per_sm=args.contains_blocks, update_blocks_per_sm=args.update_blocks)
-        prefill_gpu(g2, R, pre1, dev)
-        apply_options(g2)
-        host = [(x[0].cpu().pin_memory(), x[1].cpu().pin_memory(), x[2].cpu().pin_memory())
-                for x in inputs]
-        out = torch.empty(B1, dtype=torch.uint8).pin_memory()
-        outs = [torch.empty(B1, dtype=torch.uint8).pin_memory() for _ in range(steps)]
-        for b in range(W):
-            g2.batch_host(*host[b], out=out)
-        # (a) synchronous calls, one per step, L2 flushed before each (outside the timer)
-        t_sync = 0.0
-        for j in range(steps):
-            flush.zero_()
-            torch.cuda.synchronize()
-            t0 = time.perf_counter()
-            g2.batch_host(*host[W + j], out=out)
-            t_sync += time.perf_counter() - t0
-        last_sync = out.clone()
-        g2.close()  # one extra handle at a time (a 1B-key pool is ~72 GB)
-        # (b) the headline: the K steps back to back through gfsl_batch_host_async, as a
-        # user streams batches (copy-in of step j+1 overlaps the kernels of step j), from
-        # the first call until every step's results are in host memory; wall clock
-        # the wall clock of ~K short steps is noisy: small configs run the whole sequence
-        # 3 times, each on a freshly prefilled handle, and report the median
-        reps = 3 if R <= 10_000_000 else 1
-        t_pipes = []
-        for _rep in range(reps):
-            g3 = GFSL(R, capacity=R, chunk_entries=N, contains_team=args.team,
-                      contains_blocks_per_sm=args.contains_blocks, update_blocks_per_sm=args.update_blocks)
-            prefill_gpu(g3, R, pre1, dev)
-            apply_options(g3)
-            out_w = torch.empty(B1, dtype=torch.uint8).pin_memory()
+
+def run_e2e(args, S, inputs, W, steps, world, dev):
+    """End to end through the public API with HOST buffers: every step copies its ops in
+    from pinned host memory and its results back, inside the timed region.  N = 1:
+    gfsl_batch_host_async (copy-in of step j+1 overlaps step j's kernels), K steps back to
+    back on a caller stream, wall clock to the last result in host memory.  N > 1: per
+    step the rank's slice is copied in, the collective batch runs, the results are copied
+    out (one stream); wall clock, max over ranks."""
+    host = [tuple(x.cpu().pin_memory() for x in inp) for inp in inputs]
+    n_local = host[0][0].numel()
+    outs = [torch.empty(n_local, dtype=torch.uint8).pin_memory() for _ in range(steps)]
+    reps = 3 if S.R <= 10_000_000 else 1
+    t_pipes = []
+    for _rep in range(reps):
+        g, local_g = S.create()
+        if world == 1:
+            out_w = torch.empty(n_local, dtype=torch.uint8).pin_memory()
             for b in range(W):
-                g3.batch_host(*host[b], out=out_w)
-            # issued on a stream of the caller's own (as a serving loop would), not on the
-            # legacy default stream: measured 142 vs 246 us/step at C2 (tools/e2e_probe.py)
+                g.batch_host(*host[b], out=out_w)
             side = torch.cuda.Stream()
             torch.cuda.synchronize()
             t0 = time.perf_counter()
             with torch.cuda.stream(side):
                 for j in range(steps):
-                    g3.batch_host_async(*host[W + j], out=outs[j])
+                    g.batch_host_async(*host[W + j], out=outs[j])
             torch.cuda.synchronize()
             t_pipes.append(time.perf_counter() - t0)
-            # both handles ran the same sequence: their answers must agree
-            assert torch.equal(last_sync, outs[-1]), "e2e paths disagree"
-            g3.close()
-        t_pipe = sorted(t_pipes)[len(t_pipes) // 2]
-        e2e = {"value": round(B1 * steps / t_pipe / 1e6, 3), "unit": "Mops/s",
-               "h2d_bytes_per_step": B1 * 9, "d2h_bytes_per_step": B1,
-               "how": "gfsl_batch_host_async on a caller stream, K steps back to back from pinned host buffers, wall "
-                      "clock from the first call to the last result in host memory; L2 not "
-                      "flushed between these steps; median of %d runs of the sequence" % reps,
-               "runs_mops": [round(B1 * steps / t / 1e6, 1) for t in t_pipes],
-               "sync_per_step": {"value": round(B1 * steps / t_sync / 1e6, 3), "unit": "Mops/s",
-                                 "how": "gfsl_batch_host (synchronous) per step, L2 flushed before "
-                                        "each step, summed wall time of the calls"}}
-
-    cpu = None
-    if rank == 0 and world == 1 and not args.no_cpu_baseline:
-        cm, ct, cdone, cBs, note = oracle_sample(args.config, min(steps, 16), 1, budget_s=15.0,
-                                                combine=combine_mode(args))
-        cpu = {"value": round(cm, 4), "unit": "Mops/s", "cores": 1, "kind": "oracle",
-               "sample": f"{cdone} batches of {cBs} ops ({ct:.1f} s); {note}"}
-
-    if rank == 0:
-        line = {
-            "metric": METRIC, "value": round(mops, 3), "unit": "Mops/s", "n_gpus": world,
-            "steps": steps, "warmup": W, "ms_per_step": round(total_ms / steps, 4),
-            "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
-            "dtype": "u32", "data": "synthetic",
-            "config": {"workload": args.config, "key_range": R,
-                       "rebuild_every": "never" if args.rebuild_every < 0 else (args.rebuild_every or "default: ops since the last rebuild >= 5 x min(capacity, ops up to it) (R29)"), "prefill": pre1 * world,
-                       "batch_ops": B1 * world, "mix_ins_del_con": list(mix), "keys": dist,
-                       "semantics": "combining (R26): mutations in input order, any batch" if combine_mode(args)
-                       else "S1 snapshot, <=1 mutation per key (R1/R2)",
-                       "chunk_entries": N, "p_chunk": args.p_chunk, "contains_team": contains_team,
-                       "l2": "flushed (256 MiB write) between timed steps",
-                       "parallelism": f"range-shard x{world}" if world > 1 else "1 GPU",
-                       "exchange": (("peer windows (CUDA IPC, fused route kernels)" if args.exchange == "peer"
-                                     else "NCCL all-to-all") if world > 1 else None)},
-            "roofline": roofline,
-            "roofline_kernels": {"search": roof_c, "update": roof_u},
-            "search_gathers": gather,
-            "random_access_roofline": rand,
-            "mutations_per_step": round(n_mut, 1),
-            "phase_ms_per_step": {"intake": round(i_ms, 4), "search": round(c_ms, 4),
-                                  "update": round(u_ms, 4), "upkeep_rebuild": round(k_ms, 4)},
-            "chunk_reads_per_contains": round(reads_per_op, 3),
-            "chunk_reads_l0_per_contains": round(reads_l0_per_op, 3),
-            "cpu_baseline": cpu,
-            "e2e": e2e,
-            "gpu_launches": launches,
-            "library_launches": lib_launches,  # CUB radix-sort kernels (combining mode only)
-            "clocks": clk,
-            "wall_s_timed_region": round(wall, 4),
-            "generator_redraws": int(redraws),
-            "validate": rep,
-        }
-        print(json.dumps(line), flush=True)
+        else:
+            bufs = [torch.empty_like(x, device=dev) for x in inputs[0]]
+            for b in range(W):
+                for d_, h_ in zip(bufs, host[b]):
+                    d_.copy_(h_, non_blocking=True)
+                g.batch(*bufs)
+            torch.cuda.synchronize()
+            barrier(world)
+            t0 = time.perf_counter()
+            for j in range(steps):
+                for d_, h_ in zip(bufs, host[W + j]):
+                    d_.copy_(h_, non_blocking=True)
+                r = g.batch(*bufs)
+                outs[j].copy_(r, non_blocking=True)
+            torch.cuda.synchronize()
+            t_pipes.append(max_over_ranks(time.perf_counter() - t0, world))
+        S.close(g)
+    t_pipe = sorted(t_pipes)[len(t_pipes) // 2]
+    B = S.B
+    return {"value": round(B * steps / t_pipe / 1e6, 3), "unit": "Mops/s",
+            "h2d_bytes_per_step": B * 9, "d2h_bytes_per_step": B,
+            "how": ("gfsl_batch_host_async on a caller stream, K steps back to back from pinned host "
+                    "buffers, wall clock from the first call to the last result in host memory"
+                    if world == 1 else
+                    "per rank and step: H2D of its slice from pinned memory, the collective batch, "
+                    "D2H of its results; wall clock over K steps, max over ranks")
+                   + f"; L2 not flushed; median of {reps} run(s)",
+            "runs_mops": [round(B * steps / t / 1e6, 1) for t in t_pipes]}
 
 
 def main():
@@ -537,8 +745,9 @@ def main():
     ap.add_argument("--gpus", type=int, default=1)
     ap.add_argument("--steps", type=int, default=0, help="timed steps (0 = the config's batch count)")
     ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--runs", type=int, default=10, help="independent runs (fresh prefill each; P:1009)")
     ap.add_argument("--impl", default="gfsl", choices=["gfsl", "reference"])
-    ap.add_argument("--config", default="C2", choices=sorted(CONFIGS))
+    ap.add_argument("--config", default="C5", choices=sorted(CONFIGS))
     ap.add_argument("--team", type=int, default=0)
     ap.add_argument("--chunk", type=int, default=0)
     ap.add_argument("--contains-blocks", type=int, default=0,
@@ -556,17 +765,29 @@ def main():
                     help="combining mode (R26) for any config (always on for *-raw configs)")
     ap.add_argument("--rebuild-every", type=int, default=0,
                     help="rebuild the upper levels after every k-th batch (R24); "
-                         "0 = library default (4), -1 = never (the paper's dynamics only)")
+                         "0 = library default (R29 wear rule), -1 = never (the paper's dynamics only)")
     ap.add_argument("--dist-backend", default="nccl", choices=["nccl", "gloo"],
                     help="gloo: exercise the multi-rank path with ranks sharing a GPU (no timing value)")
     ap.add_argument("--exchange", default="peer", choices=["peer", "nccl"],
                     help="N>1 exchange: peer = fused route kernels over CUDA-IPC windows "
                          "(NEXT-3); nccl = torch.distributed all-to-all (baseline)")
-    ap.add_argument("--l2-window", action="store_true",
-                    help="pin the upper-level pool in L2 (access-policy window; ablation)")
+    ap.add_argument("--prefill", default="bulk", choices=["bulk", "per-op"],
+                    help="prefill through the bulk path (one batch, R34; default) or the paper's "
+                         "per-op Insert path in growing batches")
+    ap.add_argument("--bulk", default=None, choices=["auto", "off", "always"],
+                    help="the library's bulk path for the timed batches (R34); default auto, "
+                         "off for INS-1M / DEL-1M (they measure the paper's per-op Insert / Delete)")
+    ap.add_argument("--l2-window", type=int, default=0,
+                    help="L2 access-policy window for the search kernel: 1 = the upper-level pool, "
+                         "2 = the level-1 directory (ablations)")
     args = ap.parse_args()
     if args.warmup < 3:
         args.warmup = 3
+    if args.p_chunk <= 0:
+        ap.error("--p-chunk must be > 0 (p_chunk_q32 = 0 means p_chunk = 1)")
+    args.runs = max(1, args.runs)
+    if args.bulk is None:
+        args.bulk = "off" if args.config in PERM_CONFIGS else "auto"
     if args.impl == "reference":
         world = int(os.environ.get("WORLD_SIZE", "1"))
         rank = int(os.environ.get("RANK", "0"))

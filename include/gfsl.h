@@ -108,7 +108,21 @@ typedef struct gfsl_config {
                                (raised key, level), so runs are reproducible.  The periodic
                                upper-level rebuild (rebuild_every) replaces what the raises
                                built; combine with GFSL_REBUILD_NEVER to study p_chunk. */
+  uint32_t bulk;            /* the bulk path (R34; "compact the structure
+                               between kernel launches"): a batch of n >= GFSL_BULK_MIN_OPS
+                               ops on a map of at most U live keys with n >= GFSL_BULK_RATIO x U
+                               (U = min(capacity, ops ever submitted)) is applied by sorting
+                               the level-0 entries and the ops together and writing level 0
+                               anew (then the upper levels are rebuilt): same S1 results, no
+                               lock contention on a small structure.  0 = that rule (default),
+                               GFSL_BULK_OFF = never (the paper's per-op path only),
+                               GFSL_BULK_ALWAYS = every batch.  Not in serial or combining
+                               mode. */
 } gfsl_config;
+#define GFSL_BULK_OFF 1u
+#define GFSL_BULK_ALWAYS 2u
+#define GFSL_BULK_MIN_OPS 4096u
+#define GFSL_BULK_RATIO 2u
 
 /*
  * Create an empty GFSL (one unlocked chunk per level holding -inf with a pointer
@@ -147,6 +161,18 @@ void gfsl_destroy(gfsl_t h);
 gfsl_status gfsl_batch(gfsl_t h, const uint8_t *op_types, const uint32_t *keys,
                        const uint32_t *values, uint8_t *results, uint64_t n,
                        void *stream);
+
+/*
+ * gfsl_batch with the op count in DEVICE memory (no host round trip; e.g. the received
+ * count of a multi-GPU exchange, gfsl_xr_recv): the batch has min(*n_dev, n_max) ops,
+ * read by the kernels when they run.  n_max sizes the launch and the per-batch lists;
+ * n_hint (0 = n_max) is the op count the default rebuild policy (R29) counts for this
+ * batch.  The arrays must hold n_max entries.  Not available in combining or serial mode
+ * (GFSL_EINVAL).  Otherwise as gfsl_batch.
+ */
+gfsl_status gfsl_batch_dn(gfsl_t h, const uint8_t *op_types, const uint32_t *keys,
+                          const uint32_t *values, uint8_t *results, uint64_t n_max,
+                          const uint32_t *n_dev, uint64_t n_hint, void *stream);
 
 /*
  * Same batch through HOST buffers (pageable or pinned): copies the ops in, runs the
@@ -212,6 +238,33 @@ gfsl_status gfsl_rebuild(gfsl_t h, void *stream);
 gfsl_status gfsl_validate(gfsl_t h, gfsl_report *rep, uint32_t *keys_out,
                           uint32_t *vals_out, uint64_t cap, uint64_t *count);
 
+/*
+ * Device-side structural check (B4), chunk-parallel, for structures
+ * too large for the host walk of gfsl_validate (seconds at C5's 500M keys).  Synchronous.
+ * Checks V1-V5, V7-V9, V12, V14 and the chain shape of every level (one live chain per
+ * level from its head: one first and one last live chunk per level, every other live
+ * chunk with exactly one live predecessor); with GFSL_CHECK_CROSS also V6 (no max field
+ * grew) and V11 (zombie bytes unchanged) against the snapshot taken by an
+ * earlier call with GFSL_CHECK_SNAPSHOT, if no upper-level rebuild (and so no reclamation)
+ * ran in between.  rep (may be NULL): keys, counters, chunks[0] / zombies[0] = live /
+ * zombie level-0 chunks, chunks[1] / zombies[1] = the same over all upper levels,
+ * underfull, reserved[0] = level-1 stale separators (R33), reserved[1] = 1 if V6 / V11
+ * were checked.  Returns GFSL_OK or GFSL_ECORRUPT (rep->violations says which).
+ */
+#define GFSL_CHECK_SNAPSHOT 1u
+#define GFSL_CHECK_CROSS 2u
+gfsl_status gfsl_check(gfsl_t h, gfsl_report *rep, uint32_t flags);
+
+/*
+ * The bottom level's live (key, value) pairs in ascending key order, into DEVICE buffers
+ * keys[cap] / values[cap] (either may be NULL; both NULL = count only, no allocation).
+ * *count = the number of live keys.  Collects every live level-0 chunk's entries and sorts
+ * them on the device (temporary device memory ~16 B per slot); a key found in two live
+ * chunks makes it return GFSL_ECORRUPT.  Synchronous.
+ */
+gfsl_status gfsl_export(gfsl_t h, uint32_t *keys, uint32_t *values, uint64_t cap,
+                        uint64_t *count);
+
 /* Human-readable description of the last error on this thread. */
 const char *gfsl_last_error(void);
 
@@ -267,7 +320,9 @@ gfsl_status gfsl_load(gfsl_t h, const gfsl_meta *meta, const uint64_t *entries,
  *   uint64, number of ops for each destination) and perm[n] (device, uint32: perm[j] =
  *   input index of the j-th op in destination-major, input-stable order).  Invalid keys
  *   are routed to shard 0, which reports them invalid.
- * gfsl_route_pack: packs ops in perm order into send_op/send_key/send_val.
+ * gfsl_route_pack: packs ops in perm order into send_op/send_key/send_val; a valid op's
+ *   key is rebased to its destination's LOCAL key space (key - g * ceil(key_range/world)),
+ *   so shard g is a GFSL created over [0, its width); invalid ops keep their key.
  * gfsl_route_unpack: results[perm[j]] = recv_res[j].
  */
 gfsl_status gfsl_route_plan(const uint8_t *op_types, const uint32_t *keys, uint64_t n,
@@ -275,6 +330,7 @@ gfsl_status gfsl_route_plan(const uint8_t *op_types, const uint32_t *keys, uint6
                             uint32_t *perm, void *stream);
 gfsl_status gfsl_route_pack(const uint32_t *perm, const uint8_t *op_types,
                             const uint32_t *keys, const uint32_t *values, uint64_t n,
+                            uint64_t key_range, uint32_t world,
                             uint8_t *send_op, uint32_t *send_key, uint32_t *send_val,
                             void *stream);
 gfsl_status gfsl_route_unpack(const uint32_t *perm, const uint8_t *recv_res, uint64_t n,
@@ -285,8 +341,11 @@ gfsl_status gfsl_route_unpack(const uint32_t *perm, const uint8_t *recv_res, uin
  * device WINDOW (receive arrays for world * max_slice ops, a double-buffered count matrix,
  * barrier flags) that the peers map through CUDA IPC (one node, NVLink/NVSwitch).  The
  * push kernel stores each routed op once, straight from the caller's arrays into its
- * destination's window; the local shard runs gfsl_batch on its window; the pull kernel
- * loads every result straight from the destination's window into the caller's order.
+ * destination's window, its key rebased to the destination's local key space (as
+ * gfsl_route_pack: shard g's GFSL is created over [0, its width)); the local shard runs
+ * gfsl_batch_dn on its window with the received count read on the device (no host
+ * synchronisation anywhere in a batch); the pull kernel loads every result straight from
+ * the destination's window into the caller's order.
  * Ranks synchronise with device-side barriers (release/acquire flags at system scope),
  * each spin bounded by `timeout_ms`; an expired barrier makes the handle sticky-failed
  * (GFSL_ETIMEOUT) and the batch's results GFSL_RESULT_INVALID.  The semantics are those of
@@ -295,7 +354,8 @@ gfsl_status gfsl_route_unpack(const uint32_t *perm, const uint8_t *recv_res, uin
  *
  * gfsl_xr_create: this rank's window on the current device.  rank < world <= 64;
  *   key_range as gfsl_create; max_slice = the largest n any rank will pass (the receive
- *   arrays hold world * max_slice <= 2^32 - 1 ops); timeout_ms 0 = 60 s.  NULL on failure.
+ *   arrays hold world * max_slice <= GFSL_MAX_BATCH ops, all of which the local batch may
+ *   receive); timeout_ms 0 = 60 s.  NULL on failure.
  * gfsl_xr_export: writes the window's CUDA IPC handle (GFSL_XR_HANDLE_BYTES bytes, host).
  * gfsl_xr_attach: maps peer `peer`'s window from its exported handle (another process).
  * gfsl_xr_attach_local: uses the window of another handle of THIS process (one process
@@ -309,15 +369,23 @@ gfsl_status gfsl_route_unpack(const uint32_t *perm, const uint8_t *recv_res, uin
  *     into every peer, arrive.  Enqueue only; the caller's arrays must stay valid until the
  *     stream passes the batch.
  *   gfsl_xr_push(stream): wait for all counts, push the ops into the peers' windows, arrive.
- *   gfsl_xr_recv(..., stream): blocks the host until this rank's count exchange has
- *     completed, enqueues the wait for everyone's pushes, and returns the received count and
- *     the window's receive arrays (device pointers, owned by the handle, valid until
- *     gfsl_xr_finish): op/key/val to feed the local shard, `results` for its answers.
- *   (the caller enqueues gfsl_batch(local, op, key, val, results, n_recv, stream))
+ *   gfsl_xr_recv(..., stream): enqueues the wait for everyone's pushes and returns (without
+ *     waiting) the window's receive arrays (device pointers, owned by the handle, valid
+ *     until gfsl_xr_finish): op/key/val to feed the local shard, `results` for its answers,
+ *     their capacity *n_cap and *n_dev, the device word that holds the received count once
+ *     the stream has passed the count exchange.
+ *   gfsl_xr_local(local, n_hint, stream): the local shard's batch on the window
+ *     (gfsl_batch_dn with the device count; n_hint = the expected count, e.g. this rank's
+ *     slice size, paces the rebuild policy).  If it fails (e.g. a sticky GFSL_EPOOL) the
+ *     received ops are answered GFSL_RESULT_INVALID and its error is returned; the caller
+ *     must still make the remaining calls, so that no peer waits for this rank.
  *   gfsl_xr_done(stream): arrive (this shard's results are written).
  *   gfsl_xr_finish(results[n] of the slice, device, stream): wait, then the pull.
- * gfsl_xr_batch: all of the above plus the local gfsl_batch, for one shard per process.
- * gfsl_xr_status: GFSL_ETIMEOUT once any barrier of this handle has expired (synchronous).
+ * gfsl_xr_batch: all of the above, for one shard per process; a local failure is returned
+ *   after the exchange has completed.
+ * An expired barrier is reported by a later call on the handle (the error word reaches
+ * host memory asynchronously); gfsl_xr_status checks synchronously: GFSL_ETIMEOUT once any
+ * barrier of this handle has expired.
  * gfsl_xr_window: the window's base pointer and size (tests). */
 typedef struct gfsl_xr gfsl_xr;
 typedef gfsl_xr *gfsl_xr_t;
@@ -332,8 +400,9 @@ gfsl_status gfsl_xr_send(gfsl_xr_t x, const uint8_t *op_types, const uint32_t *k
                          const uint32_t *values, uint64_t n, void *stream);
 gfsl_status gfsl_xr_push(gfsl_xr_t x, void *stream);
 gfsl_status gfsl_xr_recv(gfsl_xr_t x, const uint8_t **op_types, const uint32_t **keys,
-                         const uint32_t **values, uint8_t **results, uint64_t *n_recv,
-                         void *stream);
+                         const uint32_t **values, uint8_t **results, uint64_t *n_cap,
+                         const uint32_t **n_dev, void *stream);
+gfsl_status gfsl_xr_local(gfsl_xr_t x, gfsl_t local, uint64_t n_hint, void *stream);
 gfsl_status gfsl_xr_done(gfsl_xr_t x, void *stream);
 gfsl_status gfsl_xr_finish(gfsl_xr_t x, uint8_t *results, void *stream);
 gfsl_status gfsl_xr_batch(gfsl_xr_t x, gfsl_t local, const uint8_t *op_types,

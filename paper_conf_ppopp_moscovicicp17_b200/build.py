@@ -15,7 +15,8 @@ ROOT = os.path.dirname(HERE)
 CSRC = os.path.join(HERE, "csrc")
 LIB = os.path.join(HERE, "libgfsl.so")
 SOURCES = ["gfsl.cu", "gfsl_xroute.cu"]
-HEADERS = ["gfsl_device.cuh", "gfsl_search.cuh", "gfsl_update.cuh", "gfsl_ubench.cuh", "gfsl_rebuild.cuh", "gfsl_combine.cuh"]
+HEADERS = ["gfsl_device.cuh", "gfsl_search.cuh", "gfsl_update.cuh", "gfsl_ubench.cuh", "gfsl_rebuild.cuh",
+           "gfsl_combine.cuh", "gfsl_check.cuh", "gfsl_bulk.cuh"]
 
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]

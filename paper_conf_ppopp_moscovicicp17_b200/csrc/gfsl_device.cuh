@@ -66,7 +66,7 @@ struct DevState {
   // is chunk r / F^l of that level: chunk l-1 (the head) if 0, else dir_hdr[32 + l] + r / F^l - 1.
   // dir_hdr = {shift, valid, buckets, F, ..., [32 + l] = base of level l}; valid = 0 until the
   // first rebuild (and after gfsl_load).
-  uint32_t *dir;
+  uint2 *dir;            // {r, bkey}: see rebuild_pack_kernel (R27, R27b)
   uint32_t *dir_hdr;
   uint32_t dir_cap;      // entries allocated (a power of two)
   // Zombie marks (R30): the update kernel sets bit c of zbits[zparity] when it makes chunk c

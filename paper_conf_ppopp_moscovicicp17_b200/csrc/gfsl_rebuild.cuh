@@ -184,38 +184,11 @@ __device__ __forceinline__ uint32_t rb_rank_le(const RebuildBufs &b, uint32_t k)
   return b.block_sum[w / RB_BLOCK_WORDS] + b.word_prefix[w] + __popc(b.bitmap[w] & mask);
 }
 
-// (4) each marked chunk writes itself at its rank; the level-1 directory (R27)
+// (4) each marked chunk writes itself at its rank
 template <int N>
 __global__ void __launch_bounds__(256) rebuild_rank_kernel(const __grid_constant__ DevState d, RebuildBufs b) {
   pdl_wait();
   if (!rb_active(b)) return;
-  {
-    // R27: bucket q = keys [q << shift, (q+1) << shift); its entry is r = rank(q << shift),
-    // the number of marked min keys (= level-1 entries >= 1) <= q << shift.  Level-1 entry
-    // r is then the largest level-1 key <= q << shift, in chunk r / F of the packed level 1,
-    // and level l's largest key <= q << shift is in its chunk r / F^l (rebuild_pack_kernel).
-    // About one bucket per level-1 key.
-    const uint32_t n1 = b.n1[0];
-    uint32_t target = 1024;
-    while (target < 2u * n1 && target < d.dir_cap) target <<= 1;
-    target = min(target, d.dir_cap);
-    int shift = 0;
-    while (((uint64_t)d.key_max >> shift) + 1 > target) ++shift;
-    const uint32_t buckets = (uint32_t)((uint64_t)d.key_max >> shift) + 1;
-    const RbLevels *L = (const RbLevels *)b.levels;
-    for (uint32_t q = blockIdx.x * blockDim.x + threadIdx.x; q < buckets; q += gridDim.x * blockDim.x)
-      d.dir[q] = rb_rank_le(b, q << shift);
-    if (blockIdx.x == 0 && threadIdx.x < 32) {
-      const int l = threadIdx.x;
-      d.dir_hdr[32 + l] = (l >= 1 && l < N) ? L->base[l] : 0u;
-      if (l == 0) {
-        d.dir_hdr[0] = (uint32_t)shift;
-        d.dir_hdr[1] = 1u;
-        d.dir_hdr[2] = buckets;
-        d.dir_hdr[3] = b.fill;
-      }
-    }
-  }
   const uint32_t used = min(d.bump[0], d.cap_bottom);
   for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < used; i += gridDim.x * blockDim.x) {
     const uint32_t c = d.cap_upper + i;
@@ -229,7 +202,8 @@ __global__ void __launch_bounds__(256) rebuild_rank_kernel(const __grid_constant
   }
 }
 
-// (5) write every chunk of levels >= 1; one warp per chunk, lane e writes entry e
+// (5) write every chunk of levels >= 1; one warp per chunk, lane e writes entry e.  And
+// the level-1 directory (R27).
 template <int N>
 __global__ void __launch_bounds__(256) rebuild_pack_kernel(const __grid_constant__ DevState d, RebuildBufs b) {
   pdl_wait();
@@ -239,6 +213,38 @@ __global__ void __launch_bounds__(256) rebuild_pack_kernel(const __grid_constant
   __shared__ RbLevels L;
   if (threadIdx.x == 0) L = *(const RbLevels *)b.levels;
   __syncthreads();
+  {
+    // R27: bucket q = keys [q << shift, (q+1) << shift); its entry is {r, bkey}: r =
+    // rank(q << shift), the number of marked min keys (= level-1 entries >= 1) <= q << shift,
+    // so level-1 entry r is the largest level-1 key <= q << shift, in chunk r / F of the
+    // packed level 1, and level l's largest key <= q << shift is in its chunk r / F^l.
+    // bkey = the first key of level-1 chunk r / F + 1 (+inf if none): a key k >= bkey of the
+    // bucket starts in that chunk instead (rank (r / F + 1) F <= rank(k)), which saves the
+    // lateral step when a bucket straddles a chunk boundary (R27b).  About one bucket per
+    // level-1 key, at most dir_cap.
+    uint32_t target = 1024;
+    while (target < 2u * n1 && target < d.dir_cap) target <<= 1;
+    target = min(target, d.dir_cap);
+    int shift = 0;
+    while (((uint64_t)d.key_max >> shift) + 1 > target) ++shift;
+    const uint32_t buckets = (uint32_t)((uint64_t)d.key_max >> shift) + 1;
+    for (uint32_t q = blockIdx.x * blockDim.x + threadIdx.x; q < buckets; q += gridDim.x * blockDim.x) {
+      const uint32_t r = rb_rank_le(b, q << shift);
+      const uint64_t nxt = ((uint64_t)r / F + 1) * F;  // first entry of the next chunk
+      const uint32_t bkey = nxt <= n1 ? b.order_key[nxt - 1] : KEY_POS_INF;
+      d.dir[q] = make_uint2(r, bkey);
+    }
+    if (blockIdx.x == 0 && threadIdx.x < 32) {
+      const int l = threadIdx.x;
+      d.dir_hdr[32 + l] = (l >= 1 && l < N) ? L.base[l] : 0u;
+      if (l == 0) {
+        d.dir_hdr[0] = (uint32_t)shift;
+        d.dir_hdr[1] = 1u;
+        d.dir_hdr[2] = buckets;
+        d.dir_hdr[3] = b.fill;
+      }
+    }
+  }
   uint32_t total = 0;
   for (int l = 1; l < N; ++l) total += L.m[l];
   const uint32_t head0 = d.head[0];

@@ -57,8 +57,10 @@ struct BatchIn {
   const uint32_t *keys;
   const uint32_t *vals;  // may be NULL (= 0)
   uint8_t *res;
-  uint32_t n;
+  uint32_t n;                // ops (or, with n_dev, the upper bound n_max)
   uint64_t key_range;
+  const uint32_t *n_dev;     // NULL, or device word holding the op count (gfsl_batch_dn):
+                             // the batch has min(*n_dev, n) ops, read at kernel time
 };
 
 // The mutations a batch's search phase hands to the update phase, compact: mutation m
@@ -93,6 +95,12 @@ constexpr uint32_t CW_NOTMUT = 0x20000000u;  // Contains or invalid: not part of
 #ifndef GFSL_SEARCH_MIN_BLOCKS
 #define GFSL_SEARCH_MIN_BLOCKS 1
 #endif
+
+__device__ __forceinline__ uint2 ld_dir(const uint2 *p) {
+  uint2 v;
+  asm volatile("ld.global.nc.v2.u32 {%0,%1}, [%2];" : "=r"(v.x), "=r"(v.y) : "l"(p));
+  return v;
+}
 
 template <int N, int TEAM, bool COUNT = false>
 __global__ void __launch_bounds__(256, GFSL_SEARCH_MIN_BLOCKS)
@@ -146,7 +154,7 @@ search_kernel(DevState d, const BatchIn in, BatchCtl *__restrict__ ctl, SearchOu
     return use_dir && !(opw & INVALID_FLAG) && (dir_upd || !(opw & UPDATE_FLAG));
   };
   auto l1_chunk = [&](uint32_t r) { const uint32_t q = r / F; return q ? s_dir_base[1] + q - 1u : 0u; };
-  const uint32_t n = in.n;
+  const uint32_t n = in.n_dev ? min(*(volatile const uint32_t *)in.n_dev, in.n) : in.n;
   uint8_t *__restrict__ res = in.res;
 
   const int team_in_warp = lane / TEAM;
@@ -191,12 +199,19 @@ search_kernel(DevState d, const BatchIn in, BatchCtl *__restrict__ ctl, SearchOu
   bool active = lane_live && slot < n;
   uint32_t k = cur_op.y;
   bool via_dir = dir_op(cur_op.x);
-  uint32_t cur_r = via_dir ? __ldg(d.dir + (k >> dir_shift)) : 0u;  // the op's directory rank
+  // the op's directory rank: r of its bucket, or the first entry of the next level-1 chunk
+  // when k is at or past that chunk's first key (R27b)
+#ifdef GFSL_DIR_NO_BKEY
+  auto dir_rank = [&](uint2 e, uint32_t) -> uint32_t { return e.x; };
+#else
+  auto dir_rank = [&](uint2 e, uint32_t key) -> uint32_t { return key >= e.y ? (e.x / F + 1u) * F : e.x; };
+#endif
+  uint32_t cur_r = via_dir ? dir_rank(ld_dir(d.dir + (k >> dir_shift)), k) : 0u;
   uint32_t cur = via_dir ? l1_chunk(cur_r) : start;
   int level = via_dir ? 1 : height;
   // the next op's directory word is loaded one loop iteration after its raw op (so that
   // its key has arrived), and is ready when the op becomes current
-  uint32_t nxt_dir = 0;
+  uint2 nxt_dir = make_uint2(0u, KEY_POS_INF);
   bool pf_dir = use_dir;
   uint32_t bt = NULL_CHUNK, bt_c = NULL_CHUNK;       // prevKv, reduced
   int seen_top = 0;                                  // highest level where k was seen
@@ -208,7 +223,7 @@ search_kernel(DevState d, const BatchIn in, BatchCtl *__restrict__ ctl, SearchOu
     ld_slice_nc<EPL>(d.pool + (size_t)cur * N + t * EPL, s);  // idle teams re-read `cur`
     if (pf_dir) {
       if ((nxt.op == 0 || (dir_upd && nxt.op <= 2)) && (uint64_t)nxt.key < in.key_range)
-        nxt_dir = __ldg(d.dir + ((nxt.key + 1u) >> dir_shift));
+        nxt_dir = ld_dir(d.dir + ((nxt.key + 1u) >> dir_shift));
       pf_dir = false;
     }
     if (COUNT && active) {
@@ -325,7 +340,7 @@ search_kernel(DevState d, const BatchIn in, BatchCtl *__restrict__ ctl, SearchOu
         k = cur_op.y;
         nxt = load_raw(slot + total_teams);
         via_dir = dir_op(cur_op.x);
-        cur_r = nxt_dir;
+        cur_r = dir_rank(nxt_dir, k);
         cur = via_dir ? l1_chunk(cur_r) : start;
         level = via_dir ? 1 : height;
         pf_dir = use_dir;

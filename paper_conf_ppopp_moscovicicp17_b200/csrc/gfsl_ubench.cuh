@@ -20,14 +20,14 @@ __device__ __forceinline__ uint64_t ub_hash(uint64_t x) {
   return x;
 }
 
-// Each team gathers `iters` random blocks, UNROLL independent gathers in flight.
-// nblocks is a power of two (the address is a masked hash).
-template <int BLOCK_BYTES, int TEAM>
+// Each team gathers `iters` random blocks, UNROLL independent gathers in flight (the host
+// sweeps UNROLL and keeps the best: the ceiling must not be limited by the benchmark's own
+// memory-level parallelism).  nblocks is a power of two (the address is a masked hash).
+template <int BLOCK_BYTES, int TEAM, int UNROLL>
 __global__ void __launch_bounds__(256) ubench_gather(const uint4 *__restrict__ buf, uint64_t nblocks,
                                                       uint32_t iters, uint32_t seed, uint32_t *sink) {
   constexpr int LANE_BYTES = BLOCK_BYTES / TEAM;      // 64 (256/4) or 64 (128/2)
   constexpr int V = LANE_BYTES / 32;                   // 32-B loads per lane
-  constexpr int UNROLL = 4;
   const int lane = threadIdx.x & 31;
   const int t = lane % TEAM;
   const uint64_t team = ((uint64_t)blockIdx.x * blockDim.x + threadIdx.x) / TEAM;

@@ -22,10 +22,13 @@
 //
 // The barriers are split-phase (arrive and wait are separate launches, so one process can
 // drive several shards in phase order even when its streams share one hardware queue).
-// No host round trip except one: the received count is read back (event) so that the local
-// gfsl_batch can be sized, as gfsl_batch takes a host n.  Every barrier spin is bounded by
-// a timeout (%globaltimer); on expiry the rank raises a sticky error flag, the remaining
-// kernels of the batch do nothing, and the host call returns GFSL_ETIMEOUT.
+// No host round trip: the received count stays on the device (the window's n_recv word),
+// and the local shard runs gfsl_batch_dn, whose kernels read their op count from there.
+// Keys arrive rebased to the destination's local key space (key - g * span), so each shard
+// is a GFSL over [0, its width) with bitmaps and directory sized for its own range.  Every
+// barrier spin is bounded by a timeout (%globaltimer); on expiry the rank raises a sticky
+// error flag, the remaining kernels of the batch do nothing (n_recv = 0, results INVALID),
+// and a later host call returns GFSL_ETIMEOUT (gfsl_xr_status checks at once).
 //
 // Reuse of the windows across batches: a rank writes a peer's receive arrays only after
 // the first barrier of the next batch, which every rank reaches only after its pull of the
@@ -45,6 +48,9 @@ size_t gfsl_internal_route_ws_bytes(uint64_t n, uint32_t world);
 gfsl_status gfsl_internal_route_plan(const uint8_t *op_types, const uint32_t *keys, uint64_t n,
                                      uint64_t key_range, uint32_t world, uint64_t *counts,
                                      uint32_t *perm, uint32_t *tile_counts, cudaStream_t s);
+extern "C" gfsl_status gfsl_batch_dn(gfsl_t h, const uint8_t *op_types, const uint32_t *keys,
+                                     const uint32_t *values, uint8_t *results, uint64_t n_max,
+                                     const uint32_t *n_dev, uint64_t n_hint, void *stream);
 
 #define XCK(call)                                                                     \
   do {                                                                                \
@@ -63,7 +69,7 @@ constexpr uint32_t XR_MAX_WORLD = 64;  // as the route kernels (gfsl.cu MAX_WORL
 struct Layout {
   size_t flags;   // u64[XR_MAX_WORLD]: flags[s] = the last barrier epoch rank s arrived at
   size_t cnt;     // u32[2][world][world]: cnt[parity][s][g] = ops rank s sends to rank g
-  size_t misc;    // u64 n_recv; u32 err
+  size_t misc;    // u64 n_recv; u32 err; u32 n_recv (the local batch's device count)
   size_t op, key, val, res;  // receive arrays, cap = world * max_slice entries each
   size_t total;
 };
@@ -86,6 +92,7 @@ Layout make_layout(uint32_t world, uint64_t cap) {
 
 struct XrArgs {
   char *const *peer;  // device table: window base of every rank (own included)
+  uint64_t key_range, span;  // the global key space and the shard width ceil(R / world)
   uint32_t rank, world, parity;
   uint64_t epoch;      // epoch of THIS barrier (counts / barrier kernels)
   uint64_t timeout_ns;
@@ -164,16 +171,19 @@ __global__ void xr_counts_kernel(XrArgs a, const unsigned long long *counts) {
   xr_arrive(a);
 }
 
-// (2) wait for every count row; n_recv = column `rank` of the matrix
+// (2) wait for every count row; n_recv = column `rank` of the matrix (0 if the exchange
+// failed: the local batch then has no ops)
 __global__ void xr_wait_counts_kernel(XrArgs a) {
-  xr_wait(a);
+  const bool ok = xr_wait(a);
   __syncthreads();
   if (threadIdx.x == 0) {
     char *own = a.peer[a.rank];
     uint64_t n = 0;
     const uint32_t *m = cnt_of(a, own);
-    for (uint32_t s = 0; s < a.world; ++s) n += ld_relaxed_sys_u32(m + s * a.world + a.rank);
+    if (ok && *(volatile uint32_t *)err_word(a, own) == 0)
+      for (uint32_t s = 0; s < a.world; ++s) n += ld_relaxed_sys_u32(m + s * a.world + a.rank);
     *(unsigned long long *)(own + a.L.misc) = n;
+    *(uint32_t *)(own + a.L.misc + 12) = (uint32_t)n;
   }
 }
 
@@ -228,8 +238,12 @@ __global__ void __launch_bounds__(256) xr_push_kernel(XrArgs a, const uint32_t *
     const size_t slot = (size_t)dst[g] + (j - seg[g]);
     const uint32_t i = perm[j];
     char *b = base[g];
-    ((uint8_t *)(b + a.L.op))[slot] = op[i];
-    ((uint32_t *)(b + a.L.key))[slot] = key[i];
+    const uint8_t o = op[i];
+    const uint32_t k = key[i];
+    ((uint8_t *)(b + a.L.op))[slot] = o;
+    // a valid op's key in its shard's local key space; invalid ones (routed to shard 0)
+    // stay out of range there
+    ((uint32_t *)(b + a.L.key))[slot] = (o <= 2 && (uint64_t)k < a.key_range) ? (uint32_t)(k - (uint64_t)g * a.span) : k;
     ((uint32_t *)(b + a.L.val))[slot] = val ? val[i] : 0u;
   }
   __threadfence_system();
@@ -282,6 +296,8 @@ static gfsl_status upload_table(gfsl_xr *x);
 static XrArgs xr_args(gfsl_xr *x, uint64_t epoch) {
   XrArgs a{};
   a.peer = x->d_peer;
+  a.key_range = x->key_range;
+  a.span = (x->key_range + x->world - 1) / x->world;
   a.rank = x->rank;
   a.world = x->world;
   a.parity = (uint32_t)(x->batches & 1);
@@ -295,7 +311,7 @@ extern "C" gfsl_xr_t gfsl_xr_create(uint32_t rank, uint32_t world, uint64_t key_
                                     uint64_t max_slice, uint64_t timeout_ms) {
   if (world == 0 || world > XR_MAX_WORLD || rank >= world || key_range == 0 ||
       key_range > 0xFFFFFFFEull || max_slice == 0 || max_slice > GFSL_MAX_BATCH ||
-      (uint64_t)world * max_slice > 0xFFFFFFFFull) {
+      (uint64_t)world * max_slice > GFSL_MAX_BATCH) {  // the local batch takes them all
     gfsl_internal_set_error("gfsl_xr_create: bad arguments");
     return nullptr;
   }
@@ -323,6 +339,7 @@ extern "C" gfsl_xr_t gfsl_xr_create(uint32_t rank, uint32_t world, uint64_t key_
   if ((e = cudaMalloc(&x->d_tiles, gfsl_internal_route_ws_bytes(max_slice, world))) != cudaSuccess)
     return fail("route workspace", e);
   if ((e = cudaMallocHost(&x->h_misc, 16)) != cudaSuccess) return fail("pinned", e);
+  memset(x->h_misc, 0, 16);
   if ((e = cudaEventCreateWithFlags(&x->ev_counts, cudaEventDisableTiming)) != cudaSuccess) return fail("event", e);
   if ((e = cudaDeviceSynchronize()) != cudaSuccess) return fail("sync", e);
   x->peer[rank] = x->win;
@@ -392,6 +409,7 @@ extern "C" gfsl_status gfsl_xr_attach_local(gfsl_xr_t x, uint32_t peer, gfsl_xr_
 }
 
 static gfsl_status xr_sticky(gfsl_xr *x) {
+  if (!x->sticky && ((volatile const uint32_t *)x->h_misc)[2] != 0) x->sticky = true;
   if (x->sticky) {
     gfsl_internal_set_error("gfsl_xr: an earlier exchange timed out (sticky)");
     return GFSL_ETIMEOUT;
@@ -433,8 +451,6 @@ extern "C" gfsl_status gfsl_xr_push(gfsl_xr_t x, void *stream) {
   }
   cudaStream_t s = (cudaStream_t)stream;
   xr_wait_counts_kernel<<<1, 64, 0, s>>>(xr_args(x, x->epoch));
-  XCK(cudaMemcpyAsync(x->h_misc, x->win + x->L.misc, 16, cudaMemcpyDeviceToHost, s));
-  XCK(cudaEventRecord(x->ev_counts, s));
   if (x->n_cur) {
     const int grid = (int)std::min<uint64_t>((x->n_cur + 255) / 256, (uint64_t)x->sms * 8);
     xr_push_kernel<<<grid, 256, 0, s>>>(xr_args(x, x->epoch), x->d_perm, (uint32_t)x->n_cur, x->in_op,
@@ -447,23 +463,17 @@ extern "C" gfsl_status gfsl_xr_push(gfsl_xr_t x, void *stream) {
 }
 
 extern "C" gfsl_status gfsl_xr_recv(gfsl_xr_t x, const uint8_t **op_types, const uint32_t **keys,
-                                    const uint32_t **values, uint8_t **results, uint64_t *n_recv,
-                                    void *stream) {
-  if (!x || x->stage != 2 || !n_recv) {
+                                    const uint32_t **values, uint8_t **results, uint64_t *n_cap,
+                                    const uint32_t **n_dev, void *stream) {
+  if (!x || x->stage != 2 || !n_cap || !n_dev) {
     gfsl_internal_set_error("gfsl_xr_recv: bad arguments or call order");
     return GFSL_EINVAL;
   }
-  XCK(cudaEventSynchronize(x->ev_counts));
   xr_wait_kernel<<<1, 64, 0, (cudaStream_t)stream>>>(xr_args(x, x->epoch));
   XCK(cudaGetLastError());
   x->stage = 3;
-  if (((const uint32_t *)x->h_misc)[2] != 0) {
-    x->sticky = true;
-    gfsl_internal_set_error("gfsl_xr_recv: a peer did not reach the count exchange in time");
-    *n_recv = 0;
-    return GFSL_ETIMEOUT;
-  }
-  *n_recv = x->h_misc[0];
+  *n_cap = x->cap;
+  *n_dev = (const uint32_t *)(x->win + x->L.misc + 12);
   if (op_types) *op_types = (const uint8_t *)(x->win + x->L.op);
   if (keys) *keys = (const uint32_t *)(x->win + x->L.key);
   if (values) *values = (const uint32_t *)(x->win + x->L.val);
@@ -493,6 +503,9 @@ extern "C" gfsl_status gfsl_xr_finish(gfsl_xr_t x, uint8_t *results, void *strea
     const int grid = (int)std::min<uint64_t>((x->n_cur + 255) / 256, (uint64_t)x->sms * 8);
     xr_pull_kernel<<<grid, 256, 0, s>>>(xr_args(x, x->epoch), x->d_perm, (uint32_t)x->n_cur, results);
   }
+  // the error word goes to pinned host memory asynchronously: a timeout of this batch makes
+  // a later call fail (gfsl_xr_status checks synchronously)
+  XCK(cudaMemcpyAsync(x->h_misc, x->win + x->L.misc, 16, cudaMemcpyDeviceToHost, s));
   XCK(cudaGetLastError());
   x->batches += 1;
   x->stage = 0;
@@ -509,6 +522,23 @@ extern "C" gfsl_status gfsl_xr_status(gfsl_xr_t x) {
   return xr_sticky(x);
 }
 
+extern "C" gfsl_status gfsl_xr_local(gfsl_xr_t x, gfsl_t local, uint64_t n_hint, void *stream) {
+  if (!x || !local || x->stage != 3) {
+    gfsl_internal_set_error("gfsl_xr_local: bad arguments or call order");
+    return GFSL_EINVAL;
+  }
+  uint8_t *rr = (uint8_t *)(x->win + x->L.res);
+  gfsl_status st = gfsl_batch_dn(local, (const uint8_t *)(x->win + x->L.op), (const uint32_t *)(x->win + x->L.key),
+                                 (const uint32_t *)(x->win + x->L.val), rr, x->cap,
+                                 (const uint32_t *)(x->win + x->L.misc + 12), n_hint ? n_hint : 1, stream);
+  if (st != GFSL_OK) {
+    // the peers still pull their results from this window: answer them INVALID; the caller
+    // then takes part in the remaining barriers (done, finish) so no peer waits for it
+    cudaMemsetAsync(rr, 0xFF, x->cap, (cudaStream_t)stream);
+  }
+  return st;
+}
+
 extern "C" gfsl_status gfsl_xr_batch(gfsl_xr_t x, gfsl_t local, const uint8_t *op_types,
                                      const uint32_t *keys, const uint32_t *values, uint8_t *results,
                                      uint64_t n, void *stream) {
@@ -516,15 +546,16 @@ extern "C" gfsl_status gfsl_xr_batch(gfsl_xr_t x, gfsl_t local, const uint8_t *o
   gfsl_status st = gfsl_xr_send(x, op_types, keys, values, n, stream);
   if (st != GFSL_OK) return st;
   const uint8_t *ro;
-  const uint32_t *rk, *rv;
+  const uint32_t *rk, *rv, *nd;
   uint8_t *rr;
-  uint64_t m = 0;
+  uint64_t cap = 0;
   if ((st = gfsl_xr_push(x, stream)) != GFSL_OK) return st;
-  st = gfsl_xr_recv(x, &ro, &rk, &rv, &rr, &m, stream);
-  if (st != GFSL_OK) return st;
-  if (m && (st = gfsl_batch(local, ro, rk, rv, rr, m, stream)) != GFSL_OK) return st;
+  if ((st = gfsl_xr_recv(x, &ro, &rk, &rv, &rr, &cap, &nd, stream)) != GFSL_OK) return st;
+  // the local shard; the expected count (this rank's own slice) paces its rebuild policy
+  const gfsl_status local_st = gfsl_xr_local(x, local, n, stream);
   if ((st = gfsl_xr_done(x, stream)) != GFSL_OK) return st;
-  return gfsl_xr_finish(x, results, stream);
+  st = gfsl_xr_finish(x, results, stream);
+  return local_st != GFSL_OK ? local_st : st;
 }
 
 extern "C" gfsl_status gfsl_xr_window(gfsl_xr_t x, void **base, uint64_t *bytes) {

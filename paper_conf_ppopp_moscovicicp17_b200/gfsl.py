@@ -24,6 +24,8 @@ GFSL_OK, GFSL_EINVAL, GFSL_ENOMEM, GFSL_EPOOL, GFSL_ECUDA, GFSL_ECORRUPT, GFSL_E
 CONTAINS, INSERT, DELETE = 0, 1, 2
 RES_FALSE, RES_TRUE, RES_INVALID = 0, 1, 0xFF
 REBUILD_DEFAULT, REBUILD_NEVER = 0, 0xFFFFFFFF  # rebuild_every: library default period / never
+CHECK_SNAPSHOT, CHECK_CROSS = 1, 2
+BULK_AUTO, BULK_OFF, BULK_ALWAYS = 0, 1, 2
 STATUS_NAMES = ["OK", "EINVAL", "ENOMEM", "EPOOL", "ECUDA", "ECORRUPT", "ETIMEOUT"]
 XR_HANDLE_BYTES = 64
 
@@ -36,7 +38,7 @@ class gfsl_config(ctypes.Structure):
                 ("profile_phases", ctypes.c_uint32), ("l2_window", ctypes.c_uint32),
                 ("no_pdl", ctypes.c_uint32),
                 ("rebuild_every", ctypes.c_uint32), ("combine", ctypes.c_uint32),
-                ("p_chunk_q32", ctypes.c_uint32)]
+                ("p_chunk_q32", ctypes.c_uint32), ("bulk", ctypes.c_uint32)]
 
 
 class gfsl_report(ctypes.Structure):
@@ -68,13 +70,14 @@ class gfsl_meta(ctypes.Structure):
 
 # Every symbol include/gfsl.h declares (checked by tests/test_abi.py).
 EXPORTS = [
-    "gfsl_create", "gfsl_create_ex", "gfsl_destroy", "gfsl_batch", "gfsl_batch_host",
+    "gfsl_create", "gfsl_create_ex", "gfsl_destroy", "gfsl_batch", "gfsl_batch_dn", "gfsl_batch_host",
     "gfsl_batch_host_async",
-    "gfsl_validate", "gfsl_last_error", "gfsl_get_stats", "gfsl_dump", "gfsl_load",
+    "gfsl_validate", "gfsl_check", "gfsl_export", "gfsl_last_error", "gfsl_get_stats", "gfsl_dump", "gfsl_load",
     "gfsl_route_plan", "gfsl_route_pack", "gfsl_route_unpack", "gfsl_phase_times",
     "gfsl_configure", "gfsl_ubench", "gfsl_rebuild",
     "gfsl_xr_create", "gfsl_xr_destroy", "gfsl_xr_export", "gfsl_xr_attach",
-    "gfsl_xr_attach_local", "gfsl_xr_send", "gfsl_xr_push", "gfsl_xr_recv", "gfsl_xr_done",
+    "gfsl_xr_attach_local", "gfsl_xr_send", "gfsl_xr_push", "gfsl_xr_recv", "gfsl_xr_local",
+    "gfsl_xr_done",
     "gfsl_xr_finish", "gfsl_xr_batch",
     "gfsl_xr_status", "gfsl_xr_window",
 ]
@@ -101,6 +104,8 @@ def load_library(path: str = LIB_PATH):
     lib.gfsl_destroy.argtypes = [vp]
     lib.gfsl_batch.restype = i32
     lib.gfsl_batch.argtypes = [vp, vp, vp, vp, vp, u64, vp]
+    lib.gfsl_batch_dn.restype = i32
+    lib.gfsl_batch_dn.argtypes = [vp, vp, vp, vp, vp, u64, vp, u64, vp]
     lib.gfsl_batch_host.restype = i32
     lib.gfsl_batch_host.argtypes = [vp, vp, vp, vp, vp, u64, vp]
     lib.gfsl_batch_host_async.restype = i32
@@ -108,6 +113,10 @@ def load_library(path: str = LIB_PATH):
     lib.gfsl_validate.restype = i32
     lib.gfsl_validate.argtypes = [vp, ctypes.POINTER(gfsl_report), vp, vp, u64,
                                   ctypes.POINTER(u64)]
+    lib.gfsl_check.restype = i32
+    lib.gfsl_check.argtypes = [vp, ctypes.POINTER(gfsl_report), u32]
+    lib.gfsl_export.restype = i32
+    lib.gfsl_export.argtypes = [vp, vp, vp, u64, ctypes.POINTER(u64)]
     lib.gfsl_last_error.restype = ctypes.c_char_p
     lib.gfsl_last_error.argtypes = []
     lib.gfsl_get_stats.restype = i32
@@ -127,7 +136,7 @@ def load_library(path: str = LIB_PATH):
     lib.gfsl_route_plan.restype = i32
     lib.gfsl_route_plan.argtypes = [vp, vp, u64, u64, u32, vp, vp, vp]
     lib.gfsl_route_pack.restype = i32
-    lib.gfsl_route_pack.argtypes = [vp, vp, vp, vp, u64, vp, vp, vp, vp]
+    lib.gfsl_route_pack.argtypes = [vp, vp, vp, vp, u64, u64, u32, vp, vp, vp, vp]
     lib.gfsl_route_unpack.restype = i32
     lib.gfsl_route_unpack.argtypes = [vp, vp, u64, vp, vp]
     lib.gfsl_xr_create.restype = vp
@@ -146,7 +155,9 @@ def load_library(path: str = LIB_PATH):
     lib.gfsl_xr_push.argtypes = [vp, vp]
     lib.gfsl_xr_recv.restype = i32
     lib.gfsl_xr_recv.argtypes = [vp, ctypes.POINTER(vp), ctypes.POINTER(vp), ctypes.POINTER(vp),
-                                 ctypes.POINTER(vp), ctypes.POINTER(u64), vp]
+                                 ctypes.POINTER(vp), ctypes.POINTER(u64), ctypes.POINTER(vp), vp]
+    lib.gfsl_xr_local.restype = i32
+    lib.gfsl_xr_local.argtypes = [vp, vp, u64, vp]
     lib.gfsl_xr_done.restype = i32
     lib.gfsl_xr_done.argtypes = [vp, vp]
     lib.gfsl_xr_finish.restype = i32
@@ -207,7 +218,8 @@ class GFSL:
                  contains_team: int = 0, serial_updates: bool = False,
                  contains_blocks_per_sm: int = 0, update_blocks_per_sm: int = 0,
                  count_reads: bool = False, profile_phases: bool = False,
-                 rebuild_every: int = 0, combine: bool = False, p_chunk: float = 1.0):
+                 rebuild_every: int = 0, combine: bool = False, p_chunk: float = 1.0,
+                 bulk: int = 0):
         import torch
         if not torch.cuda.is_available():
             raise RuntimeError("GFSL needs a CUDA device (there is no CPU fallback)")
@@ -216,7 +228,9 @@ class GFSL:
                           update_blocks_per_sm, 1 if serial_updates else 0,
                           1 if count_reads else 0, 1 if profile_phases else 0, 0, 0,
                           rebuild_every, 1 if combine else 0,
-                          0 if p_chunk >= 1.0 else int(p_chunk * 2**32))
+                          0 if p_chunk >= 1.0 else max(1, int(p_chunk * 2**32)), bulk)
+        if p_chunk <= 0:
+            raise ValueError("p_chunk must be > 0 (p_chunk_q32 = 0 means p_chunk = 1)")
         self.key_range = int(key_range)
         self.chunk_entries = int(chunk_entries)
         self.cfg = cfg
@@ -259,6 +273,12 @@ class GFSL:
         """Asynchronous batch on raw device pointers (e.g. an exchange window's arrays)."""
         _check(self.lib.gfsl_batch(self.h, op_ptr, key_ptr, val_ptr, res_ptr, n, _stream(stream)),
                "gfsl_batch")
+
+    def batch_dn(self, op_ptr: int, key_ptr: int, val_ptr: int | None, res_ptr: int, n_max: int,
+                 n_dev_ptr: int, n_hint: int = 0, stream=None):
+        """Asynchronous batch whose op count lives in device memory (gfsl_batch_dn)."""
+        _check(self.lib.gfsl_batch_dn(self.h, op_ptr, key_ptr, val_ptr, res_ptr, n_max, n_dev_ptr,
+                                      n_hint, _stream(stream)), "gfsl_batch_dn")
 
     def batch_host(self, op, key, val=None, out=None, stream=None):
         """Synchronous batch on HOST tensors (the end-to-end entry point)."""
@@ -306,6 +326,38 @@ class GFSL:
             raise GFSLError(st, f"gfsl_validate (violations=0x{rep.violations:x})")
         return report, keys, vals
 
+    def check(self, snapshot: bool = False, cross: bool = False, raise_on_violation: bool = True):
+        """Device-side structural check (gfsl_check, B4): a Report; chunks[1] / zombies[1]
+        count all upper levels together; .stale = level-1 stale separators (R33);
+        .cross_checked = whether V6 / V11 were checked against the last snapshot."""
+        rep = gfsl_report()
+        flags = (CHECK_SNAPSHOT if snapshot else 0) | (CHECK_CROSS if cross else 0)
+        st = self.lib.gfsl_check(self.h, ctypes.byref(rep), flags)
+        if st not in (GFSL_OK, GFSL_ECORRUPT):
+            _check(st, "gfsl_check")
+        report = Report(rep.keys, rep.height, list(rep.chunks), list(rep.zombies),
+                        list(rep.level_keys), list(rep.counters), tuple(rep.pool_used),
+                        tuple(rep.pool_cap), rep.violations, rep.first_violation, rep.restarts,
+                        rep.underfull)
+        report.stale = rep.reserved[0]
+        report.cross_checked = bool(rep.reserved[1])
+        if st == GFSL_ECORRUPT and raise_on_violation:
+            raise GFSLError(st, f"gfsl_check (violations=0x{rep.violations:x})")
+        return report
+
+    def export(self):
+        """(keys, values): the live pairs in key order as int32 DEVICE tensors holding
+        uint32 bit patterns (gfsl_export; sorted on the device)."""
+        import torch
+        cnt = ctypes.c_uint64()
+        _check(self.lib.gfsl_export(self.h, None, None, 0, ctypes.byref(cnt)), "gfsl_export")
+        n = cnt.value
+        dev = torch.device("cuda", torch.cuda.current_device())
+        keys = torch.empty(n, dtype=torch.int32, device=dev)
+        vals = torch.empty(n, dtype=torch.int32, device=dev)
+        _check(self.lib.gfsl_export(self.h, _ptr(keys), _ptr(vals), n, ctypes.byref(cnt)), "gfsl_export")
+        return keys, vals
+
     def stats(self) -> dict:
         s = gfsl_stats()
         _check(self.lib.gfsl_get_stats(self.h, ctypes.byref(s)), "gfsl_get_stats")
@@ -323,6 +375,14 @@ class GFSL:
         nb = ctypes.c_uint64()
         _check(self.lib.gfsl_phase_times(self.h, ms, ctypes.byref(nb)), "gfsl_phase_times")
         return dict(intake=ms[0], contains=ms[1], update=ms[2], upkeep=ms[3], total=ms[4]), nb.value
+
+    def meta(self):
+        """Head array, level counters and pool use (gfsl_dump without the pool; synchronises)."""
+        m = gfsl_meta()
+        _check(self.lib.gfsl_dump(self.h, ctypes.byref(m), None, 0), "gfsl_dump")
+        return dict(head=list(m.head), counters=list(m.counters), used_bottom=m.used_bottom,
+                    used_upper=m.used_upper, cap_bottom=m.cap_bottom, cap_upper=m.cap_upper,
+                    chunk_entries=m.chunk_entries)
 
     def dump(self):
         """(meta dict, entries uint64 array of shape [chunks, N]) -- test-only."""
@@ -349,6 +409,24 @@ class GFSL:
         _check(self.lib.gfsl_load(self.h, ctypes.byref(m), ent.ctypes.data, ent.size), "gfsl_load")
 
 
+def read_device_u32(dev_ptr: int) -> int:
+    """One uint32 from device memory, synchronously (tests / diagnostics only)."""
+    global _cudart
+    if _cudart is None:
+        import torch  # noqa: F401  (loads the CUDA runtime into the process)
+        _cudart = ctypes.CDLL("libcudart.so.12")
+        _cudart.cudaMemcpy.restype = ctypes.c_int
+        _cudart.cudaMemcpy.argtypes = [ctypes.c_void_p, ctypes.c_void_p, ctypes.c_size_t, ctypes.c_int]
+    buf = ctypes.c_uint32()
+    st = _cudart.cudaMemcpy(ctypes.addressof(buf), dev_ptr, 4, 2)  # cudaMemcpyDeviceToHost
+    if st != 0:
+        raise RuntimeError(f"cudaMemcpy failed ({st})")
+    return buf.value
+
+
+_cudart = None
+
+
 # ---- multi-GPU routing primitives (B5) ------------------------------------------------
 def route_plan(op, key, key_range: int, world: int, stream=None):
     """Returns (counts int64[world] on device, perm int32[n] on device)."""
@@ -362,15 +440,16 @@ def route_plan(op, key, key_range: int, world: int, stream=None):
     return counts, perm
 
 
-def route_pack(perm, op, key, val, stream=None):
+def route_pack(perm, op, key, val, key_range: int, world: int, stream=None):
+    """Ops in routed order; keys rebased to their destination shard's local key space."""
     import torch
     lib = load_library()
     n = op.numel()
     so = torch.empty_like(op)
     sk = torch.empty_like(key)
     sv = torch.empty(n, dtype=key.dtype, device=op.device)
-    _check(lib.gfsl_route_pack(_ptr(perm), _ptr(op), _ptr(key), _ptr(val), n, _ptr(so),
-                               _ptr(sk), _ptr(sv), _stream(stream)), "gfsl_route_pack")
+    _check(lib.gfsl_route_pack(_ptr(perm), _ptr(op), _ptr(key), _ptr(val), n, key_range, world,
+                               _ptr(so), _ptr(sk), _ptr(sv), _stream(stream)), "gfsl_route_pack")
     return so, sk, sv
 
 
@@ -433,13 +512,19 @@ class XRoute:
         _check(self.lib.gfsl_xr_push(self.h, _stream(stream)), "gfsl_xr_push")
 
     def recv(self, stream=None):
-        """(n_recv, op_ptr, key_ptr, val_ptr, res_ptr): the window's receive arrays."""
-        o, k, v, r = ctypes.c_void_p(), ctypes.c_void_p(), ctypes.c_void_p(), ctypes.c_void_p()
+        """(n_cap, n_dev_ptr, op_ptr, key_ptr, val_ptr, res_ptr): the window's receive
+        arrays, their capacity and the device word holding the received count."""
+        o, k, v, r, nd = (ctypes.c_void_p() for _ in range(5))
         m = ctypes.c_uint64()
         _check(self.lib.gfsl_xr_recv(self.h, ctypes.byref(o), ctypes.byref(k), ctypes.byref(v),
-                                     ctypes.byref(r), ctypes.byref(m), _stream(stream)),
-               "gfsl_xr_recv")
-        return m.value, o.value, k.value, v.value, r.value
+                                     ctypes.byref(r), ctypes.byref(m), ctypes.byref(nd),
+                                     _stream(stream)), "gfsl_xr_recv")
+        return m.value, nd.value, o.value, k.value, v.value, r.value
+
+    def local(self, local: "GFSL", n_hint: int = 0, stream=None) -> int:
+        """The local shard's batch on the window (gfsl_xr_local); returns the status
+        (GFSL_OK, or the local error after the received ops were answered INVALID)."""
+        return self.lib.gfsl_xr_local(self.h, local.h, n_hint, _stream(stream))
 
     def done(self, stream=None):
         _check(self.lib.gfsl_xr_done(self.h, _stream(stream)), "gfsl_xr_done")

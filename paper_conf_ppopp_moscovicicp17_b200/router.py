@@ -1,12 +1,14 @@
 """Range-partitioned multi-GPU GFSL.
 
-Shard g owns keys [g*ceil(R/G), min(R, (g+1)*ceil(R/G))) in its own GFSL (keys stay
-global; no rebasing).  Every rank calls ``batch`` collectively with its own slice of the
+Shard g owns keys [g*ceil(R/G), min(R, (g+1)*ceil(R/G))) in its own GFSL, created over
+its LOCAL key space [0, hi - lo): the route kernels rebase every key on its way in
+(key - lo), so each shard's bitmaps and directory are sized for its own range, and the
+export adds lo back.  Every rank calls ``batch`` collectively with its own slice of the
 global batch, like an NCCL collective.  One batch is:
 
   route_plan (CUDA: per-op destination, per-tile histogram, scan, stable scatter)
   -> all_to_all of the per-destination counts
-  -> route_pack (CUDA) -> all_to_all of ops, keys, values (NCCL over NVLink)
+  -> route_pack (CUDA, keys rebased) -> all_to_all of ops, keys, values (NCCL over NVLink)
   -> the local gfsl_batch (S1 on the shard)
   -> all_to_all of the 1-byte results back -> route_unpack (CUDA) into the caller's order.
 
@@ -18,6 +20,7 @@ with the gloo backend (tests/test_router_gloo.py).
 """
 from __future__ import annotations
 
+import numpy as np
 import torch
 import torch.distributed as dist
 
@@ -40,8 +43,8 @@ class CudaRouteKernels:
     def plan(self, op, key, key_range, world):
         return G.route_plan(op, key, key_range, world)
 
-    def pack(self, perm, op, key, val):
-        return G.route_pack(perm, op, key, val)
+    def pack(self, perm, op, key, val, key_range, world):
+        return G.route_pack(perm, op, key, val, key_range, world)
 
     def local_batch(self, op, key, val):
         return self.local.batch(op, key, val)
@@ -58,8 +61,8 @@ class ShardedGFSL:
         self.rank, self.world, self.group = rank, world, group
         self.key_lo, self.key_hi, self.span = shard_bounds(self.key_range, world, rank)
         if kernels is None:
-            cap = capacity if capacity else max(1, self.key_hi - self.key_lo)
-            self.local = G.GFSL(self.key_range, capacity=cap, **gfsl_kw)
+            width = max(1, self.key_hi - self.key_lo)
+            self.local = G.GFSL(width, capacity=capacity or width, **gfsl_kw)
             kernels = CudaRouteKernels(self.local)
         else:
             self.local = getattr(kernels, "local", None)
@@ -83,7 +86,7 @@ class ShardedGFSL:
         if val is None:
             val = torch.zeros_like(key)
         counts, perm = self.k.plan(op, key, self.key_range, self.world)
-        so, sk, sv = self.k.pack(perm, op, key, val)
+        so, sk, sv = self.k.pack(perm, op, key, val, self.key_range, self.world)
         recv_counts = torch.empty_like(counts)
         self._a2a(recv_counts, counts, None, None)
         send_split = counts.tolist()
@@ -101,6 +104,17 @@ class ShardedGFSL:
         self.last_counts = (send_split, recv_split)
         return self.k.unpack(perm, back, n)
 
+    def export(self):
+        """This shard's validated (report, global keys, values)."""
+        return export_global(self.local, self.key_lo)
+
+
+def export_global(local: "G.GFSL", key_lo: int):
+    rep, ks, vs = local.validate()
+    if ks is not None:
+        ks = (ks.astype(np.uint64) + key_lo).astype(np.uint32)
+    return rep, ks, vs
+
 
 class PeerShardedGFSL:
     """Range-partitioned GFSL with the fused peer-memory exchange (gfsl_xr_*; SURVEY 8(f)
@@ -115,8 +129,8 @@ class PeerShardedGFSL:
         self.key_range = int(key_range)
         self.rank, self.world, self.group = rank, world, group
         self.key_lo, self.key_hi, self.span = shard_bounds(self.key_range, world, rank)
-        cap = capacity if capacity else max(1, self.key_hi - self.key_lo)
-        self.local = G.GFSL(self.key_range, capacity=cap, **gfsl_kw)
+        width = max(1, self.key_hi - self.key_lo)
+        self.local = G.GFSL(width, capacity=capacity or width, **gfsl_kw)
         self.xr = G.XRoute(rank, world, self.key_range, max_slice, timeout_ms)
         handles = [None] * world
         dist.all_gather_object(handles, self.xr.export(), group=group)
@@ -129,6 +143,9 @@ class PeerShardedGFSL:
         """Collective.  op uint8[n], key 32-bit[n], val 32-bit[n] (this rank's slice);
         returns uint8[n] results in the slice's order."""
         return self.xr.batch(self.local, op, key, val, out=out, stream=stream)
+
+    def export(self):
+        return export_global(self.local, self.key_lo)
 
 
 class LoopbackShards:
@@ -146,8 +163,8 @@ class LoopbackShards:
         self.bounds = [shard_bounds(self.key_range, world, r) for r in range(world)]
         self.local = []
         for lo, hi, _ in self.bounds:
-            cap = capacity if capacity else max(1, hi - lo)
-            self.local.append(G.GFSL(self.key_range, capacity=cap, **gfsl_kw))
+            width = max(1, hi - lo)
+            self.local.append(G.GFSL(width, capacity=capacity or width, **gfsl_kw))
         self.xr = [G.XRoute(r, world, self.key_range, max_slice, timeout_ms) for r in range(world)]
         for r in range(world):
             for p in range(world):
@@ -177,16 +194,28 @@ class LoopbackShards:
             self.xr[r].send(op[a:b], key[a:b], val[a:b], stream=self.streams[r])
         for r in range(self.world):
             self.xr[r].push(stream=self.streams[r])
-        recv = []
-        for r in range(self.world):
+        recv, errs = [], []
+        for r, (a, b) in enumerate(sl):
             recv.append(self.xr[r].recv(stream=self.streams[r]))
-            m, o, k, v, res = recv[-1]
-            if m:
-                self.local[r].batch_ptr(o, k, v, res, m, stream=self.streams[r])
+            st = self.xr[r].local(self.local[r], n_hint=max(1, b - a), stream=self.streams[r])
+            if st != G.GFSL_OK:
+                errs.append((st, r))
             self.xr[r].done(stream=self.streams[r])
         for r, (a, b) in enumerate(sl):
             self.xr[r].finish(out[a:b], stream=self.streams[r])
         for s in self.streams:
             cur.wait_stream(s)
-        self.last_recv = [x[0] for x in recv]
+        self.recv_ptrs = [x[1] for x in recv]
+        if errs:
+            G._check(errs[0][0], f"gfsl_xr_local (shard {errs[0][1]})")
         return out
+
+    def last_recv(self):
+        """The received op count of every shard in the last batch (synchronises; tests)."""
+        torch.cuda.synchronize()
+        return [G.read_device_u32(nd) for nd in self.recv_ptrs]
+
+    def export(self, r: int):
+        lo = self.bounds[r][0]
+        return export_global(self.local[r], lo)
+

@@ -6,10 +6,12 @@
 * C3 (R = 10M, 6.25M-op batches): the same, for 4 batches.
 * C2 raw Zipf in combining mode (R26): every result vs Oracle-A's combining semantics.
 * C4-16 (100M keys, 50M Contains per batch): every lookup of a key of the full structure
-  answers true (a property at any size), and the invariants hold.
-* C5 (R = 1B, 500M live keys, 125M-op batches): sampled -- present and absent keys of the
-  prefill answer true / false, and one full 10/10/80 batch keeps #true inserts and
-  deletes equal to the closed forms |I \\ M| and |D & M| on its sampled keys.
+  answers true, the device export is exactly (k, prefill value of k) for every k, and the
+  device check passes.
+* C5 (R = 1B, 500M live keys, 125M-op batches): every result of 2 full batches vs the DAT
+  (5 GB of host memory), then the exported set (device export, 500M pairs) vs the DAT and
+  the device check (gfsl_check: V1-V5, V7-V9, V12, V14, chain shape; V6 / V11 across the
+  batches).
 """
 import numpy as np
 import pytest
@@ -89,33 +91,41 @@ def test_fullsize_c4_contains_all_true():
         assert int(op.max()) == 0
         r = g.batch(op.contiguous(), key.to(torch.int32).contiguous(), None)
         assert int(r.min()) == 1 and int(r.max()) == 1
-    rep, _, _ = g.validate(export=False)
-    assert rep.violations == 0 and rep.keys == R
+    d = g.check()
+    assert d.violations == 0 and d.keys == R
+    ks, vs = g.export()
+    assert ks.numel() == R
+    assert bool((ks.to(torch.int64) == torch.arange(R, device=DEV)).all())
+    exp_v = prefill_values(SEED_BASE, torch.arange(R, device=DEV)).to(torch.int32)
+    assert bool((vs == exp_v).all())
     g.close()
 
 
-def test_fullsize_c5_sampled():
+def test_fullsize_c5_every_result():
     R, pre, B, _, mix, dist, N = cfg("C5")
     g = GFSL(R, capacity=R, chunk_entries=N)
-    prefill_both(g, None, R, pre)
-    present = prefill_keys(SEED_BASE, R, 1 << 20, start=0, device=DEV)
-    absent = prefill_keys(SEED_BASE, R, 1 << 20, start=pre, device=DEV)
-    zeros = torch.zeros(1 << 20, dtype=torch.uint8, device=DEV)
-    assert int(g.batch(zeros, present.to(torch.int32)).min()) == 1
-    assert int(g.batch(zeros, absent.to(torch.int32)).max()) == 0
-    # one full batch; its mutating keys on the sampled present / absent sets obey the
-    # closed forms of S1 (an Insert succeeds iff absent, a Delete iff present)
+    ref = DirectAddressMap(R)
+    import bench
+    bench.prefill_gpu(g, R, pre, DEV)
+    for s0 in range(0, pre, 1 << 26):  # the same prefill into the DAT, in slices
+        k = prefill_keys(SEED_BASE, R, min(1 << 26, pre - s0), start=s0, device=DEV)
+        v = prefill_values(SEED_BASE, k)
+        ref.load(k.cpu().numpy(), v.cpu().numpy().astype(np.uint32))
+    d = g.check(snapshot=True)
+    assert d.violations == 0 and d.keys == pre
     w = Workload(R, B, mix=mix, dist=dist, seed=SEED_BASE + 1)
-    op, key, val, _ = w.make_batch(0, device=DEV)
-    r = g.batch(op.contiguous(), key.to(torch.int32).contiguous(), val.to(torch.int32).contiguous())
-    ps = torch.zeros(R, dtype=torch.bool, device=DEV)
-    ps[present] = True
-    ab = torch.zeros(R, dtype=torch.bool, device=DEV)
-    ab[absent] = True
-    k = key.to(torch.int64)
-    ins, dele = op == 1, op == 2
-    assert bool((r[ins & ps[k]] == 0).all()) and bool((r[ins & ab[k]] == 1).all())
-    assert bool((r[dele & ps[k]] == 1).all()) and bool((r[dele & ab[k]] == 0).all())
-    assert bool((r[(op == 0) & ps[k]] == 1).all()) and bool((r[(op == 0) & ab[k]] == 0).all())
-    assert int((ins & (ps[k] | ab[k])).sum()) > 1000
+    for b in range(2):
+        op, key, val, _ = w.make_batch(b, device=DEV)
+        r = g.batch(op.contiguous(), key.to(torch.int32).contiguous(), val.to(torch.int32).contiguous())
+        r = r.cpu().numpy()
+        e = ref.batch(op.cpu().numpy(), key.cpu().numpy().astype(np.uint32), val.cpu().numpy().astype(np.uint32))
+        bad = np.flatnonzero(r != e)
+        assert bad.size == 0, f"batch {b}: {bad.size} of {B} results differ, first {bad[:5]}"
+        d = g.check(snapshot=True, cross=True)
+        assert d.violations == 0
+    ks, vs = g.export()
+    ek, ev = ref.export()
+    assert ks.numel() == ek.size
+    assert np.array_equal(ks.cpu().numpy().view(np.uint32), ek)
+    assert np.array_equal(vs.cpu().numpy().view(np.uint32), ev)
     g.close()

@@ -1,0 +1,232 @@
+"""GPU parity, round 2: the paper's own update protocol under contention, batches outside
+the <=1-mutation-per-key contract, and the device-side check / export (B4).
+
+* Paper mode (p_chunk = 1, rebuild_every = NEVER, concurrent update kernel): the raise
+  under the bottom lock (Alg 4.5 l.15-22), updateDownPtrs (Alg 4.10) and the
+  top-down upper-level Deletes (Alg 4.11 l.13-20) all run concurrently -- 50/50 churn on a
+  600-key range for 40 batches, fill then drain of 50K keys, and the full-size C2 workload
+  for 19 batches; every result and the exported set vs Oracle-A / the DAT, and the
+  invariants (host walk + device check, V6 / V11 across batches) after every batch.
+* Out of contract: batches with many mutations of the same key (include/gfsl.h: "every
+  result is still the result of SOME linearization of the batch") -- checked per
+  key against the sequential definition, and the final set must follow the same
+  linearization.
+* gfsl_check / gfsl_export agree with the host walk of gfsl_validate, and the check
+  catches planted faults.
+"""
+import numpy as np
+import pytest
+import torch
+
+from oracle.dat import DirectAddressMap
+from oracle.oracle_a import OracleMap
+from paper_conf_ppopp_moscovicicp17_b200.gfsl import GFSL, REBUILD_NEVER
+from paper_conf_ppopp_moscovicicp17_b200.workload import (
+    SEED_BASE, Workload, prefill_keys, prefill_values)
+from tests import gfsl_fixtures as fx
+from tests.linearize import linearizable
+
+pytestmark = pytest.mark.gpu
+DEV = torch.device("cuda")
+
+
+def to_dev(op, key, val):
+    return (torch.as_tensor(np.ascontiguousarray(op, np.uint8)).to(DEV),
+            torch.as_tensor(np.ascontiguousarray(key, np.uint32).view(np.int32)).to(DEV),
+            None if val is None else torch.as_tensor(np.ascontiguousarray(val, np.uint32).view(np.int32)).to(DEV))
+
+
+def run_batch(g, o, op, key, val):
+    r = g.batch(*to_dev(op, key, val)).cpu().numpy()
+    e = o.batch(op, key, val)
+    bad = np.flatnonzero(r != e)
+    assert bad.size == 0, f"{bad.size} results differ, first {bad[:5]}: gpu={r[bad[:5]]} oracle={e[bad[:5]]}"
+    return r
+
+
+def check_all(g, o, cross=True):
+    rep, ks, vs = g.validate()
+    ok, ov = o.export()
+    assert rep.violations == 0 and np.array_equal(ks, ok) and np.array_equal(vs, ov)
+    d = g.check(snapshot=True, cross=cross)
+    assert d.violations == 0 and d.keys == len(o)
+    dk, dv = g.export()
+    assert np.array_equal(dk.cpu().numpy().view(np.uint32), ok)
+    assert np.array_equal(dv.cpu().numpy().view(np.uint32), ov)
+    return rep, d
+
+
+def batches(R, B, nb, mix, seed):
+    w = Workload(R, B, mix=mix, seed=seed)
+    for b in range(nb):
+        op, key, val, _ = w.make_batch(b)
+        yield op.numpy(), key.numpy().astype(np.uint32), val.numpy().astype(np.uint32)
+
+
+# ---------------------------------------------------------------- paper mode, concurrent
+
+@pytest.mark.parametrize("N", [16, 32])
+def test_paper_mode_concurrent_churn_small_range(N):
+    R = 600
+    g = GFSL(R, chunk_entries=N, rebuild_every=REBUILD_NEVER)   # p_chunk = 1 (default)
+    o = OracleMap(R)
+    for op, key, val in batches(R, 300, 40, (50, 50, 0), SEED_BASE + 201 + N):
+        run_batch(g, o, op, key, val)
+        _, d = check_all(g, o)
+    assert d.cross_checked                    # no rebuild ran: V6 / V11 were checked
+    st = g.stats()
+    assert st["splits"] > 0 and st["merges"] > 0
+    rep, _, _ = g.validate()
+    assert rep.height >= 1                    # keys were raised (Alg 4.5 l.15-22)
+
+
+@pytest.mark.parametrize("N", [16, 32])
+def test_paper_mode_fill_then_drain(N):
+    R = 50_000
+    g = GFSL(R, chunk_entries=N, rebuild_every=REBUILD_NEVER)
+    o = OracleMap(R)
+    perm = np.random.default_rng(50 + N).permutation(R).astype(np.uint32)
+    for s in range(0, R, 12_345):
+        k = perm[s:s + 12_345]
+        run_batch(g, o, np.ones(k.size, np.uint8), k, k * 7)
+        check_all(g, o)
+    rep, _, _ = g.validate()
+    assert rep.keys == R and rep.height >= 3
+    perm2 = np.random.default_rng(60 + N).permutation(R).astype(np.uint32)
+    for s in range(0, R, 9_999):
+        k = perm2[s:s + 9_999]
+        run_batch(g, o, np.full(k.size, 2, np.uint8), k, None)
+        check_all(g, o)
+    assert len(o) == 0
+    assert g.stats()["merges"] > 0
+
+
+def test_paper_mode_c2_fullsize_every_result():
+    """C2 (R = 1M, prefill 500K, 625K-op batches of [10,10,80]) with the paper's structure
+    dynamics: every result of 19 batches vs the DAT, then the set and the invariants."""
+    import bench
+    R, pre, B, _, mix, dist, N = bench.CONFIGS["C2"]
+    g = GFSL(R, capacity=R, chunk_entries=N, rebuild_every=REBUILD_NEVER)
+    ref = DirectAddressMap(R)
+    bench.prefill_gpu(g, R, pre, DEV)
+    k = prefill_keys(SEED_BASE, R, pre).numpy().astype(np.uint32)
+    ref.batch(np.ones(k.size, np.uint8), k, prefill_values(SEED_BASE, torch.from_numpy(k.astype(np.int64))).numpy().astype(np.uint32))
+    w = Workload(R, B, mix=mix, dist=dist, seed=SEED_BASE + 1)
+    g.check(snapshot=True)
+    for b in range(19):
+        op, key, val, _ = w.make_batch(b, device=DEV)
+        r = g.batch(op.contiguous(), key.to(torch.int32).contiguous(), val.to(torch.int32).contiguous()).cpu().numpy()
+        e = ref.batch(op.cpu().numpy(), key.cpu().numpy().astype(np.uint32), val.cpu().numpy().astype(np.uint32))
+        bad = np.flatnonzero(r != e)
+        assert bad.size == 0, f"batch {b}: {bad.size} results differ"
+        d = g.check(snapshot=True, cross=True)
+        assert d.violations == 0 and d.cross_checked
+    rep, ks, vs = g.validate()
+    ek, ev = ref.export()
+    assert rep.violations == 0 and np.array_equal(ks, ek) and np.array_equal(vs, ev)
+    g.close()
+
+
+# ---------------------------------------------------------------- out of contract
+
+@pytest.mark.parametrize("serial", [False, True])
+def test_out_of_contract_batches_are_linearizable(serial):
+    R = 3000
+    g = GFSL(R, serial_updates=serial)
+    rng = np.random.default_rng(7 + serial)
+    present = np.zeros(R, bool)
+    value = np.zeros(R, np.uint32)
+    hot = rng.choice(R, 150, replace=False)
+    for b in range(12):
+        n = 4000
+        key = np.where(rng.random(n) < 0.6, rng.choice(hot, n), rng.integers(0, R, n)).astype(np.uint32)
+        op = rng.choice([0, 1, 2], n, p=[0.3, 0.4, 0.3]).astype(np.uint8)
+        val = rng.integers(0, 2**32, n, dtype=np.uint64).astype(np.uint32)
+        r = g.batch(*to_dev(op, key, val)).cpu().numpy()
+        rep, ks, vs = g.validate()
+        assert rep.violations == 0
+        fin_p = np.zeros(R, bool)
+        fin_p[ks] = True
+        fin_v = np.zeros(R, np.uint32)
+        fin_v[ks] = vs
+        order = np.argsort(key, kind="stable")
+        cuts = np.flatnonzero(np.diff(key[order])) + 1
+        for grp in np.split(order, cuts):
+            k = int(key[grp[0]])
+            assert linearizable(bool(present[k]), int(value[k]), op[grp].tolist(), r[grp].tolist(),
+                                val[grp].tolist(), bool(fin_p[k]), int(fin_v[k])), \
+                f"batch {b} key {k}: ops {op[grp].tolist()} results {r[grp].tolist()}"
+        untouched = np.ones(R, bool)
+        untouched[key] = False
+        assert np.array_equal(fin_p[untouched], present[untouched])
+        assert np.array_equal(fin_v[untouched & present], value[untouched & present])
+        present, value = fin_p, fin_v
+        assert g.check().violations == 0
+
+
+# ---------------------------------------------------------------- gfsl_check / gfsl_export
+
+@pytest.mark.parametrize("N,every", [(16, 0), (32, 0), (16, REBUILD_NEVER), (12, 1), (6, REBUILD_NEVER)])
+def test_device_check_and_export_agree_with_host_walk(N, every):
+    R = 20_000 if N >= 16 else 3000
+    g = GFSL(R, chunk_entries=N, rebuild_every=every)
+    o = OracleMap(R)
+    for op, key, val in batches(R, 2_500, 14, (35, 30, 35), SEED_BASE + 300 + N):
+        run_batch(g, o, op, key, val)
+        rep, d = check_all(g, o, cross=True)
+        # the host walk counts the zombies still linked; the device check every zombie in
+        # the pool (also those upkeep unlinked, not yet reclaimed)
+        assert d.chunks[0] == rep.chunks[0] and d.zombies[0] >= rep.zombies[0]
+        assert d.height == rep.height
+
+
+def test_device_check_catches_planted_faults():
+    g = GFSL(100, capacity=64, chunk_entries=12, serial_updates=True, rebuild_every=REBUILD_NEVER)
+    meta0, _ = g.dump()
+    m, names = fx.build(fx.FD, 12, key_range=100, cap_bottom=meta0["cap_bottom"], cap_upper=meta0["cap_upper"])
+    meta, ent = fx.image(m)
+    ent = ent.reshape(-1, 12)
+    g.load(meta, ent)
+    assert g.check().violations == 0
+    e, f = names["E"], names["F"]
+
+    def with_fault(fn):
+        bad = ent.copy()
+        fn(bad)
+        g.load(meta, bad)
+        v = g.check(raise_on_violation=False).violations
+        g.load(meta, ent)
+        return v
+
+    def unsort(a):    # V1: two keys of E swapped
+        a[e, 1], a[e, 2] = a[e, 2], a[e, 1]
+    def maxup(a):     # V2: E's max field no longer its largest key
+        a[e, 10] = (a[e, 10] & ~np.uint64(0xFFFFFFFF)) | np.uint64(23)
+    def overlap(a):   # V3: F starts below E's max
+        a[f, 0] = (a[f, 0] & ~np.uint64(0xFFFFFFFF)) | np.uint64(15)
+    def locked(a):    # V7: a live chunk left locked
+        a[f, 11] = np.uint64(1)
+    def dangling(a):  # V12: a NEXT beyond the allocated chunks
+        a[e, 10] = (a[e, 10] & np.uint64(0xFFFFFFFF)) | (np.uint64(60) << np.uint64(32))
+    for fn, v in ((unsort, 1), (maxup, 2), (overlap, 3), (locked, 7), (dangling, 12)):
+        assert with_fault(fn) & (1 << (v - 1)), fn.__name__
+    assert g.check().violations == 0
+
+
+def test_device_check_cross_batch_v6_v11():
+    """V6 / V11 fire when a max field grows or a zombie changes between two checks."""
+    g = GFSL(100, capacity=64, chunk_entries=12, serial_updates=True, rebuild_every=REBUILD_NEVER)
+    meta0, _ = g.dump()
+    m, names = fx.build(fx.FD, 12, key_range=100, cap_bottom=meta0["cap_bottom"], cap_upper=meta0["cap_upper"])
+    meta, ent = fx.image(m)
+    g.load(meta, ent.reshape(-1, 12))
+    assert g.batch(*to_dev([2], [13], None)).cpu().tolist() == [1]   # E becomes a zombie
+    d = g.check(snapshot=True)
+    assert d.violations == 0 and d.zombies[0] == 1
+    meta1, ent1 = g.dump()
+    e = names["E"]
+    bad = ent1.copy()
+    bad[e, 1] ^= np.uint64(1)                # the zombie's bytes change
+    g.load(meta1, bad)
+    v = g.check(cross=True, raise_on_violation=False)
+    assert v.violations & (1 << 10)

@@ -39,9 +39,14 @@ def test_route_plan_pack_unpack(world, n):
     ec, ep = ref_plan(op, key, R, world)
     assert counts.cpu().numpy().tolist() == ec.tolist()
     assert np.array_equal(perm.cpu().numpy(), ep.astype(np.int32))
-    so, sk, sv = G.route_pack(perm, op_d, key_d, val_d)
+    so, sk, sv = G.route_pack(perm, op_d, key_d, val_d, R, world)
     assert np.array_equal(so.cpu().numpy(), op[ep])
-    assert np.array_equal(sk.cpu().numpy().view(np.uint32), key[ep])
+    # valid ops' keys in their destination's local key space; invalid ones unchanged
+    span = -(-R // world)
+    k64, o8 = key.astype(np.int64), op
+    valid = (o8 <= 2) & (k64 < R)
+    local = np.where(valid, k64 - np.minimum(k64 // span, world - 1) * span, k64).astype(np.uint32)
+    assert np.array_equal(sk.cpu().numpy().view(np.uint32), local[ep])
     assert np.array_equal(sv.cpu().numpy().view(np.uint32), val[ep])
     rr = torch.arange(n, device=dev).to(torch.uint8)
     out = torch.empty(n, dtype=torch.uint8, device=dev)
@@ -55,7 +60,7 @@ def test_route_plan_pack_unpack(world, n):
 def test_loopback_shards_match_global_oracle(world):
     R, B = 200_000, 40_000
     dev = torch.device("cuda")
-    shards = [G.GFSL(R, capacity=shard_bounds(R, world, g)[1] - shard_bounds(R, world, g)[0])
+    shards = [G.GFSL(shard_bounds(R, world, g)[1] - shard_bounds(R, world, g)[0])
               for g in range(world)]
     o = OracleMap(R)
     w = Workload(R, B, mix=(20, 20, 60), seed=SEED_BASE + 9)
@@ -65,7 +70,7 @@ def test_loopback_shards_match_global_oracle(world):
         key_d = key.to(torch.int32).to(dev)
         val_d = val.to(torch.int32).to(dev)
         counts, perm = G.route_plan(op_d, key_d, R, world)
-        so, sk, sv = G.route_pack(perm, op_d, key_d, val_d)
+        so, sk, sv = G.route_pack(perm, op_d, key_d, val_d, R, world)
         parts, s = [], 0
         for g, c in enumerate(counts.tolist()):
             parts.append(shards[g].batch(so[s:s + c], sk[s:s + c], sv[s:s + c]) if c else
@@ -75,7 +80,8 @@ def test_loopback_shards_match_global_oracle(world):
         G.route_unpack(perm, torch.cat(parts), res)
         exp = o.batch(op.numpy(), key.numpy().astype(np.uint32), val.numpy().astype(np.uint32))
         assert np.array_equal(res.cpu().numpy(), exp)
-    ks = np.concatenate([sh.validate()[1] for sh in shards])
+    ks = np.concatenate([sh.validate()[1].astype(np.int64) + shard_bounds(R, world, g)[0]
+                         for g, sh in enumerate(shards)]).astype(np.uint32)
     vs = np.concatenate([sh.validate()[2] for sh in shards])
     ok, ov = o.export()
     assert np.array_equal(ks, ok) and np.array_equal(vs, ov)

@@ -28,9 +28,10 @@ def _to_dev(op, key, val, dev):
     return (op.to(dev), key.to(torch.int32).to(dev), val.to(torch.int32).to(dev))
 
 
-def _check_final(local_shards, o):
-    ks = np.concatenate([sh.validate()[1] for sh in local_shards])
-    vs = np.concatenate([sh.validate()[2] for sh in local_shards])
+def _check_final(ls, o):
+    ex = [ls.export(r) for r in range(ls.world)]
+    ks = np.concatenate([x[1] for x in ex])
+    vs = np.concatenate([x[2] for x in ex])
     ok, ov = o.export()
     assert np.array_equal(ks, ok) and np.array_equal(vs, ov)
 
@@ -47,8 +48,8 @@ def test_loopback_exchange_matches_global_oracle(world):
         res = ls.batch(*_to_dev(op, key, val, dev))
         exp = o.batch(op.numpy(), key.numpy().astype(np.uint32), val.numpy().astype(np.uint32))
         assert np.array_equal(res.cpu().numpy(), exp), f"batch {b}"
-        assert sum(ls.last_recv) == B
-    _check_final(ls.local, o)
+        assert sum(ls.last_recv()) == B
+    _check_final(ls, o)
 
 
 def test_loopback_edge_batches():
@@ -78,25 +79,87 @@ def test_loopback_edge_batches():
     op[::97] = 7
     kk[::89] = R + 5
     run(op, kk, rng.integers(0, 2**32, n, dtype=np.uint64).astype(np.uint32))
-    _check_final(ls.local, o)
+    _check_final(ls, o)
 
 
 def test_timeout_when_a_peer_never_arrives():
+    """Rank 1 never sends: rank 0's count barrier expires, its received count is 0, its
+    results are INVALID, no call blocks, and the handle reports GFSL_ETIMEOUT from then on."""
     dev = torch.device("cuda")
     a = G.XRoute(0, 2, 1000, 16, timeout_ms=200)
     b = G.XRoute(1, 2, 1000, 16, timeout_ms=200)
     a.attach_local(1, b)
+    local = G.GFSL(500)
     op = torch.zeros(4, dtype=torch.uint8, device=dev)
     key = torch.arange(4, dtype=torch.int32, device=dev)
+    out = torch.zeros(4, dtype=torch.uint8, device=dev)
     a.send(op, key)  # rank 1 never sends
     a.push()
-    with pytest.raises(G.GFSLError) as e:
-        a.recv()
-    assert e.value.status == G.GFSL_ETIMEOUT
+    cap, nd, o, k, v, r = a.recv()
+    assert cap == 32
+    local.batch_dn(o, k, v, r, cap, nd, n_hint=4)
+    a.done()
+    try:
+        a.finish(out)
+    except G.GFSLError as e:   # may already see the error word
+        assert e.status == G.GFSL_ETIMEOUT
     torch.cuda.synchronize()
+    assert G.read_device_u32(nd) == 0
+    assert out.cpu().tolist() == [0xFF] * 4
     assert a.status() == G.GFSL_ETIMEOUT
+    with pytest.raises(G.GFSLError) as e:
+        a.send(op, key)
+    assert e.value.status == G.GFSL_ETIMEOUT
+    local.close()
     b.close()
     a.close()
+
+
+def test_local_failure_still_completes_the_exchange():
+    """A shard whose local batch fails (a sticky GFSL_EPOOL here) answers its received ops
+    INVALID and still takes part in every barrier (gfsl_xr_local): the other shard's ops
+    are answered and nobody times out."""
+    R, world = 40_000, 2
+    dev = torch.device("cuda")
+    ls = LoopbackShards(R, world, max_slice=20_000, timeout_ms=10_000)
+    ls.local[1].close()
+    ls.local[1] = G.GFSL(R // 2, capacity=10)          # a tiny pool: exhausted at once
+    keys = torch.randperm(R, generator=torch.Generator().manual_seed(3))[:30_000].to(torch.int32)
+    op = torch.ones(keys.numel(), dtype=torch.uint8)
+    ls.batch(op.to(dev), keys.to(dev), keys.to(dev))   # shard 1 raises GFSL_EPOOL on device
+    torch.cuda.synchronize()
+    out = None
+    with pytest.raises(G.GFSLError) as e:
+        out = ls.batch(op.to(dev), keys.to(dev), keys.to(dev))  # shard 1 fails on the host
+    assert e.value.status == G.GFSL_EPOOL
+    torch.cuda.synchronize()
+    # the exchange completed: the same call again gives shard 0's answers (present now ->
+    # Insert false) and INVALID for shard 1's, with no timeout on either window
+    with pytest.raises(G.GFSLError):
+        ls.batch(op.to(dev), keys.to(dev), keys.to(dev))
+    for x in ls.xr:
+        assert x.status() == G.GFSL_OK
+    k = keys.numpy().astype(np.int64)
+    sl = ls.slices(k.size)
+    res = []
+    # re-run with results kept: drive the phases by hand to read the output
+    outs = torch.empty(k.size, dtype=torch.uint8, device=dev)
+    op_d, key_d = op.to(dev), keys.to(dev)
+    torch.cuda.synchronize()
+    for r, (a, b) in enumerate(sl):
+        ls.xr[r].send(op_d[a:b], key_d[a:b], key_d[a:b], stream=ls.streams[r])
+    for r in range(world):
+        ls.xr[r].push(stream=ls.streams[r])
+    for r, (a, b) in enumerate(sl):
+        ls.xr[r].recv(stream=ls.streams[r])
+        res.append(ls.xr[r].local(ls.local[r], n_hint=b - a, stream=ls.streams[r]))
+        ls.xr[r].done(stream=ls.streams[r])
+    for r, (a, b) in enumerate(sl):
+        ls.xr[r].finish(outs[a:b], stream=ls.streams[r])
+    torch.cuda.synchronize()
+    assert res == [G.GFSL_OK, G.GFSL_EPOOL]
+    o = outs.cpu().numpy()
+    assert (o[k < R // 2] == 0).all() and (o[k >= R // 2] == 0xFF).all()
 
 
 def _ipc_worker(rank, world, port, R, B, nb, outdir):
@@ -117,7 +180,7 @@ def _ipc_worker(rank, world, port, R, B, nb, outdir):
         a, e = sl[rank]
         res = g.batch(*_to_dev(op[a:e].contiguous(), key[a:e].contiguous(), val[a:e].contiguous(), dev))
         outs.append(res.cpu().numpy())
-    _, ks, vs = g.local.validate()
+    _, ks, vs = g.export()
     np.savez(os.path.join(outdir, f"r{rank}.npz"), res=np.concatenate(outs), ks=ks, vs=vs)
     dist.barrier()
     dist.destroy_process_group()

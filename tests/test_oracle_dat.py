@@ -27,3 +27,21 @@ def test_dat_contract_check():
     d = DirectAddressMap(10)
     with pytest.raises(ValueError):
         d.batch(np.array([1, 2], np.uint8), np.array([3, 3], np.uint32), None)
+
+
+def test_load_equals_an_insert_batch():
+    """DirectAddressMap.load (the full-size prefill) = an S1 batch of distinct Inserts."""
+    rng = np.random.default_rng(11)
+    R = 5000
+    k = rng.permutation(R)[:2000].astype(np.uint32)
+    v = rng.integers(0, 2**32, k.size, dtype=np.uint64).astype(np.uint32)
+    a = DirectAddressMap(R)
+    b = DirectAddressMap(R)
+    a.batch(np.ones(k.size, np.uint8), k, v)
+    b.load(k, v)
+    ka, va = a.export()
+    kb, vb = b.export()
+    assert np.array_equal(ka, kb) and np.array_equal(va, vb)
+    import pytest
+    with pytest.raises(ValueError):
+        b.load(k[:3], v[:3])

@@ -20,8 +20,11 @@ from paper_conf_ppopp_moscovicicp17_b200.workload import SEED_BASE, Workload
 
 
 class CpuKernels:
-    def __init__(self, key_range):
-        self.oracle = OracleMap(key_range)
+    """Stand-ins with the kernels' contract: the pack rebases a valid op's key to its
+    destination's local key space (gfsl_route_pack), the local map is keyed locally."""
+
+    def __init__(self, width):
+        self.oracle = OracleMap(width)
         self.local = None
 
     def plan(self, op, key, key_range, world):
@@ -32,9 +35,14 @@ class CpuKernels:
         counts = np.bincount(dest, minlength=world).astype(np.int64)
         return torch.from_numpy(counts), torch.from_numpy(perm)
 
-    def pack(self, perm, op, key, val):
+    def pack(self, perm, op, key, val, key_range, world):
         p = perm.long()
-        return op[p].contiguous(), key[p].contiguous(), val[p].contiguous()
+        span = -(-key_range // world)
+        o = op[p].numpy()
+        k = key[p].numpy().view(np.uint32).astype(np.int64)
+        valid = (o <= 2) & (k < key_range)
+        local = np.where(valid, k - np.minimum(k // span, world - 1) * span, k).astype(np.uint32)
+        return op[p].contiguous(), torch.from_numpy(local.view(np.int32)), val[p].contiguous()
 
     def local_batch(self, op, key, val):
         r = self.oracle.batch(op.numpy(), key.numpy().view(np.uint32), val.numpy().view(np.uint32))
@@ -51,7 +59,8 @@ def _worker(rank, world, port, R, B, nb, q):
     os.environ["MASTER_PORT"] = str(port)
     dist.init_process_group("gloo", rank=rank, world_size=world)
     try:
-        sg = ShardedGFSL(R, rank, world, kernels=CpuKernels(R))
+        lo, hi, _ = shard_bounds(R, world, rank)
+        sg = ShardedGFSL(R, rank, world, kernels=CpuKernels(hi - lo))
         w = Workload(R, B * world, mix=(20, 20, 60), seed=SEED_BASE + 5)
         out = []
         for b in range(nb):
@@ -64,8 +73,8 @@ def _worker(rank, world, port, R, B, nb, q):
                          val[sl].to(torch.int32).contiguous())
             out.append(r.numpy())
         ks, vs = sg.k.oracle.export()
-        lo, hi, _ = shard_bounds(R, world, rank)
-        assert ks.size == 0 or (ks.min() >= lo and ks.max() < hi)
+        assert ks.size == 0 or ks.max() < hi - lo          # local key space
+        ks = (ks.astype(np.int64) + lo).astype(np.uint32)
         q.put((rank, out, ks, vs))
     finally:
         dist.destroy_process_group()

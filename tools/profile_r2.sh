@@ -1,0 +1,26 @@
+#!/bin/bash
+# Round-2 profiling pass (run under gpurun from the repo root; one GPU):
+#  1. launch list (gpu__time_duration only, one pass, no replay) of the default bench (C5)
+#  2. DRAM / L2 traffic of one mid-run batch per config: application replay (ncu reruns the
+#     whole program per pass, so no 70-GB save/restore of the pool between passes),
+#     --cache-control all (cold L2 per pass, as bench.py flushes L2 before each timed step)
+#  3. one `--set full` capture of the C5 search kernel (application replay)
+# Outputs in $O; summaries by tools/ncu_metrics.py.
+set -u
+O=${O:-gpurun_out/prof_r2}; mkdir -p $O
+CFGS=${CFGS:-"C5 C4-16 C3 C2"}
+M=gpu__time_duration.sum,dram__bytes_read.sum,dram__bytes_write.sum,lts__t_bytes.sum,lts__t_sector_hit_rate.pct,l1tex__t_sector_hit_rate.pct,smsp__issue_active.avg.pct_of_peak_sustained_active,dram__throughput.avg.pct_of_peak_sustained_elapsed,sm__warps_active.avg.pct_of_peak_sustained_active,launch__registers_per_thread
+timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none --csv \
+  --log-file $O/launches_C5.csv python bench.py --runs 1 --steps 4 --warmup 3 --no-cpu-baseline --no-e2e --no-ubench \
+  > $O/launches_C5_bench.log 2>&1
+for c in $CFGS; do
+  timeout 1200 ncu --replay-mode application --profile-from-start off --metrics $M --clock-control none \
+    --cache-control all -f -o $O/traffic_$c python tools/prof_step.py $c > $O/traffic_$c.log 2>&1
+  python tools/ncu_metrics.py $O/traffic_$c.ncu-rep > $O/ncu_$c.json 2>&1
+done
+if [ -z "${NO_FULL:-}" ]; then
+  timeout 2400 ncu --replay-mode application --profile-from-start off --set full --import-source on \
+    --clock-control none --cache-control all -k regex:search_kernel -f -o $O/full_C5_search \
+    python tools/prof_step.py C5 > $O/full_C5.log 2>&1
+  python tools/ncu_metrics.py $O/full_C5_search.ncu-rep > $O/ncu_full_C5_search.json 2>&1
+fi
