@@ -43,10 +43,14 @@ L2_BYTES = 126 << 20          # B200 L2 (B200_PROFILING.md)
 L2_FLUSH_BYTES = 256 << 20
 
 # name: (R, prefill, batch, n_batches, mix, dist, N)
-# N = chunk entries.  The paper's runs use N = 32; on B200 a chunk read costs L1
-# data-pipe wavefronts in proportion to its bytes, and N = 16 (128-B chunks, 2-lane teams)
-# is faster on every config measured, so it is the default here; the
-# C4 pair compares the two, and --chunk 32 runs any config at the paper's size.
+# N = chunk entries.  The paper's runs use N = 32.  On B200 the choice follows
+# the memory level that bounds the search: while the upper levels are
+# L2-resident (C1-C4) a chunk read costs L1 data-pipe wavefronts in proportion to its
+# bytes and N = 16 (128-B chunks) wins; at C5 (1B keys) the level-1 gathers go to HBM,
+# whose random-request rate -- not bytes -- is the limit, and N = 32 halves both the
+# level-0 chunk count and level 1 (208 MB instead of 509 MB: more of it stays in L2):
+# measured +26% at C5 in one gpurun call.  The C4 pair compares the two; --chunk N
+# overrides any config.
 CONFIGS = {
     "C1": (10_000, 5_000, 6_250, 16, (10, 10, 80), "uniform", 16),
     "C2": (1_000_000, 500_000, 625_000, 16, (10, 10, 80), "uniform", 16),
@@ -57,7 +61,7 @@ CONFIGS = {
     "C3-zipf": (10_000_000, 5_000_000, 6_250_000, 16, (10, 10, 80), "zipf", 16),
     "C4-32": (100_000_000, 100_000_000, 50_000_000, 10, (0, 0, 100), "uniform", 32),
     "C4-16": (100_000_000, 100_000_000, 50_000_000, 10, (0, 0, 100), "uniform", 16),
-    "C5": (1_000_000_000, 500_000_000, 125_000_000, 8, (10, 10, 80), "uniform", 16),
+    "C5": (1_000_000_000, 500_000_000, 125_000_000, 8, (10, 10, 80), "uniform", 32),
     # NEXT-4: the paper's other workloads (Fig 5.3 mixes, Fig 5.4b/c single-op runs)
     "M1-1-98": (1_000_000, 500_000, 625_000, 16, (1, 1, 98), "uniform", 16),
     "M5-5-90": (1_000_000, 500_000, 625_000, 16, (5, 5, 90), "uniform", 16),
@@ -166,9 +170,22 @@ class ClockSampler:
 
     def result(self):
         self.pause()
-        return {"sm_mhz": statistics.median(self.samples) if self.samples else None,
-                "sm_max_mhz": self.max_mhz, "reasons": sorted(self.reasons),
-                "samples": len(self.samples)}
+        out = {"sm_mhz": statistics.median(self.samples) if self.samples else None,
+               "sm_max_mhz": self.max_mhz, "reasons": sorted(self.reasons),
+               "samples": len(self.samples)}
+        if self.ok:  # which board this ran on (box-to-box variance of HBM random access)
+            nv = self.nv
+            for k, f in (("mem_mhz", lambda: nv.nvmlDeviceGetClockInfo(self.hdl, nv.NVML_CLOCK_MEM)),
+                         ("mem_max_mhz", lambda: nv.nvmlDeviceGetMaxClockInfo(self.hdl, nv.NVML_CLOCK_MEM)),
+                         ("ecc", lambda: nv.nvmlDeviceGetEccMode(self.hdl)[0]),
+                         ("uuid", lambda: nv.nvmlDeviceGetUUID(self.hdl)),
+                         ("vbios", lambda: nv.nvmlDeviceGetVbiosVersion(self.hdl))):
+                try:
+                    v = f()
+                    out[k] = v.decode() if isinstance(v, bytes) else v
+                except Exception:
+                    pass
+        return out
 
 
 def dist_setup(backend="nccl"):

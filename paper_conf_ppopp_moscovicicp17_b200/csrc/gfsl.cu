@@ -34,7 +34,7 @@
 using namespace gfsl_dev;
 
 #ifndef GFSL_DIR_CAP_LOG2
-#define GFSL_DIR_CAP_LOG2 22  // level-1 directory buckets at most 2^22 (32 MiB of {r, bkey})
+#define GFSL_DIR_CAP_LOG2 24  // level-1 directory buckets at most 2^24 (16 MiB of bytes + 2 MiB of bases)
 #endif
 
 // ------------------------------------------------------------------------------------
@@ -193,7 +193,7 @@ static void fill_window(gfsl *h, cudaLaunchAttribute &a) {
   a.id = cudaLaunchAttributeAccessPolicyWindow;
   // l2_window = 2: the level-1 directory only (R27; 8 B x its buckets); else the upper pool
   const bool dir = h->cfg.l2_window == 2;
-  const size_t used = dir ? (size_t)h->d.dir_cap * 8 : (size_t)std::min(h->h_bump[1] + 64u, h->d.cap_upper) * h->N * 8;
+  const size_t used = dir ? (size_t)h->d.dir_cap : (size_t)std::min(h->h_bump[1] + 64u, h->d.cap_upper) * h->N * 8;
   const size_t bytes = std::min(used, h->window_max);
   a.val.accessPolicyWindow.base_ptr = dir ? (void *)h->d.dir : (void *)h->d.pool;
   a.val.accessPolicyWindow.num_bytes = bytes;
@@ -459,6 +459,7 @@ static void free_all(gfsl *h) {
   cudaFree(h->d.zbits);
   cudaFree(h->d.fl);
   cudaFree(h->d.dir);
+  cudaFree(h->d.dir_base);
   cudaFree(h->d.dir_hdr);
   cudaFree(h->snap_max);
   cudaFree(h->snap_zh);
@@ -554,11 +555,17 @@ extern "C" gfsl_t gfsl_create_ex(uint64_t key_range, uint64_t capacity, const gf
     if ((e = cudaMalloc(&h->d.fl, 8 * 4)) != cudaSuccess) return fail("cudaMalloc(freelist)", e);
     if ((e = cudaMalloc(&h->rc_tiles, ((size_t)cap_b / RC_TILE + 2) * 4)) != cudaSuccess) return fail("cudaMalloc(reclaim)", e);
     cudaMemset(h->d.fl, 0, 8 * 4);
-    // R27: level-1 directory, about one bucket per level-1 key, at most 2^22 (32 MiB)
+    // R27 / R27b: level-1 directory, about four buckets per level-1 key, at most
+    // 2^GFSL_DIR_CAP_LOG2: one byte per bucket plus one 32-bit base per 32 buckets
     uint32_t dcap = 1024;
     while (dcap < (1u << GFSL_DIR_CAP_LOG2) && (uint64_t)dcap < key_range + 1) dcap <<= 1;
     h->d.dir_cap = dcap;
-    if ((e = cudaMalloc(&h->d.dir, (size_t)dcap * 8)) != cudaSuccess) return fail("cudaMalloc(dir)", e);
+#ifdef GFSL_DIR_U32
+    if ((e = cudaMalloc(&h->d.dir, (size_t)dcap * 4)) != cudaSuccess) return fail("cudaMalloc(dir)", e);
+#else
+    if ((e = cudaMalloc(&h->d.dir, (size_t)dcap)) != cudaSuccess) return fail("cudaMalloc(dir)", e);
+#endif
+    if ((e = cudaMalloc(&h->d.dir_base, (size_t)dcap / 32 * 4)) != cudaSuccess) return fail("cudaMalloc(dir)", e);
     if ((e = cudaMalloc(&h->d.dir_hdr, 64 * 4)) != cudaSuccess) return fail("cudaMalloc(dir)", e);
     cudaMemset(h->d.dir_hdr, 0, 64 * 4);
     // R30: zombie marks, two bitmaps over every chunk index

@@ -60,15 +60,19 @@ struct DevState {
   uint32_t *fl;          // [0] free chunks in the current list, [1] taken, [2] buffer,
                          // [3..5] reclaim scratch
   unsigned long long *debug_times;  // GFSL_DEBUG_TIMING builds: per-team (start, end, ops)
-  // Directory (R27): dir[b] = how many level-1 keys of the last rebuild are <= (b << shift)
-  // (the rank r of the bucket's low key).  The rebuilt level l holds every F^(l-1)-th
-  // level-1 key F per chunk, so the chunk of level l that holds the largest key <= b << shift
-  // is chunk r / F^l of that level: chunk l-1 (the head) if 0, else dir_hdr[32 + l] + r / F^l - 1.
-  // dir_hdr = {shift, valid, buckets, F, ..., [32 + l] = base of level l}; valid = 0 until the
-  // first rebuild (and after gfsl_load).
-  uint2 *dir;            // {r, bkey}: see rebuild_pack_kernel (R27, R27b)
+  // Directory (R27): the rank r(b) = how many level-1 keys of the last rebuild are
+  // <= (b << shift), stored compactly so that it stays L2-resident under the random-gather
+  // traffic of a 1B-key structure (R27b): r(b) = dir_base[b >> 5] + dir[b], one byte per
+  // bucket (a delta saturated at 255: a smaller rank is still a valid start, one more
+  // lateral step) and one 32-bit base per 32 buckets.  The rebuilt level l holds every
+  // F^(l-1)-th level-1 key F per chunk, so the chunk of level l that holds the largest key
+  // <= b << shift is chunk r / F^l of that level: chunk l-1 (the head) if 0, else
+  // dir_hdr[32 + l] + r / F^l - 1.  dir_hdr = {shift, valid, buckets, F, ..., [32 + l] =
+  // base of level l}; valid = 0 until the first rebuild (and after gfsl_load).
+  uint8_t *dir;
+  uint32_t *dir_base;
   uint32_t *dir_hdr;
-  uint32_t dir_cap;      // entries allocated (a power of two)
+  uint32_t dir_cap;      // buckets allocated (a power of two, multiple of 32)
   // Zombie marks (R30): the update kernel sets bit c of zbits[zparity] when it makes chunk c
   // a zombie; the upkeep sweep after the batch only has to follow NEXT pointers whose target
   // bit is set, instead of reading every successor's lock word.  Two bitmaps of zwords words

@@ -23,6 +23,10 @@
 
 namespace gfsl_dev {
 
+#ifndef GFSL_DIR_PER_KEY
+#define GFSL_DIR_PER_KEY 4u  // directory buckets per level-1 key (R27b)
+#endif
+
 struct RebuildBufs {
   uint32_t *bitmap;       // [words]      key marks (all zero between rebuilds)
   uint32_t *word_prefix;  // [words]      exclusive popcount prefix within a 1024-word block
@@ -214,25 +218,27 @@ __global__ void __launch_bounds__(256) rebuild_pack_kernel(const __grid_constant
   if (threadIdx.x == 0) L = *(const RbLevels *)b.levels;
   __syncthreads();
   {
-    // R27: bucket q = keys [q << shift, (q+1) << shift); its entry is {r, bkey}: r =
-    // rank(q << shift), the number of marked min keys (= level-1 entries >= 1) <= q << shift,
-    // so level-1 entry r is the largest level-1 key <= q << shift, in chunk r / F of the
-    // packed level 1, and level l's largest key <= q << shift is in its chunk r / F^l.
-    // bkey = the first key of level-1 chunk r / F + 1 (+inf if none): a key k >= bkey of the
-    // bucket starts in that chunk instead (rank (r / F + 1) F <= rank(k)), which saves the
-    // lateral step when a bucket straddles a chunk boundary (R27b).  About one bucket per
-    // level-1 key, at most dir_cap.
+    // R27: bucket q = keys [q << shift, (q+1) << shift); r(q) = rank(q << shift), the
+    // number of marked min keys (= level-1 entries >= 1) <= q << shift, so level-1 entry
+    // r(q) is the largest level-1 key <= q << shift, in chunk r / F of the packed level 1,
+    // and level l's largest key <= q << shift is in its chunk r / F^l.  R27b: about four
+    // buckets per level-1 key (at most dir_cap), one byte each: r(q) = base[q / 32] +
+    // min(255, r(q) - base[q / 32]), base[g] = r(32 g).
     uint32_t target = 1024;
-    while (target < 2u * n1 && target < d.dir_cap) target <<= 1;
+    while (target < GFSL_DIR_PER_KEY * n1 && target < d.dir_cap) target <<= 1;
     target = min(target, d.dir_cap);
     int shift = 0;
     while (((uint64_t)d.key_max >> shift) + 1 > target) ++shift;
     const uint32_t buckets = (uint32_t)((uint64_t)d.key_max >> shift) + 1;
     for (uint32_t q = blockIdx.x * blockDim.x + threadIdx.x; q < buckets; q += gridDim.x * blockDim.x) {
       const uint32_t r = rb_rank_le(b, q << shift);
-      const uint64_t nxt = ((uint64_t)r / F + 1) * F;  // first entry of the next chunk
-      const uint32_t bkey = nxt <= n1 ? b.order_key[nxt - 1] : KEY_POS_INF;
-      d.dir[q] = make_uint2(r, bkey);
+#ifdef GFSL_DIR_U32
+      ((uint32_t *)d.dir)[q] = r;
+#else
+      const uint32_t base = (q & 31u) ? rb_rank_le(b, (q & ~31u) << shift) : r;
+      d.dir[q] = (uint8_t)min(255u, r - base);
+      if ((q & 31u) == 0) d.dir_base[q >> 5] = base;
+#endif
     }
     if (blockIdx.x == 0 && threadIdx.x < 32) {
       const int l = threadIdx.x;

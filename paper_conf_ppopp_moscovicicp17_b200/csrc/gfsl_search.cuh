@@ -96,12 +96,6 @@ constexpr uint32_t CW_NOTMUT = 0x20000000u;  // Contains or invalid: not part of
 #define GFSL_SEARCH_MIN_BLOCKS 1
 #endif
 
-__device__ __forceinline__ uint2 ld_dir(const uint2 *p) {
-  uint2 v;
-  asm volatile("ld.global.nc.v2.u32 {%0,%1}, [%2];" : "=r"(v.x), "=r"(v.y) : "l"(p));
-  return v;
-}
-
 template <int N, int TEAM, bool COUNT = false>
 __global__ void __launch_bounds__(256, GFSL_SEARCH_MIN_BLOCKS)
 search_kernel(DevState d, const BatchIn in, BatchCtl *__restrict__ ctl, SearchOut so) {
@@ -199,19 +193,22 @@ search_kernel(DevState d, const BatchIn in, BatchCtl *__restrict__ ctl, SearchOu
   bool active = lane_live && slot < n;
   uint32_t k = cur_op.y;
   bool via_dir = dir_op(cur_op.x);
-  // the op's directory rank: r of its bucket, or the first entry of the next level-1 chunk
-  // when k is at or past that chunk's first key (R27b)
-#ifdef GFSL_DIR_NO_BKEY
-  auto dir_rank = [&](uint2 e, uint32_t) -> uint32_t { return e.x; };
+  // the op's directory rank (R27b): base of its 32-bucket group + its byte
+  auto dir_rank = [&](uint2 e, uint32_t) -> uint32_t { return e.x + e.y; };
+  auto ld_dir = [&](uint32_t key) -> uint2 {
+    const uint32_t q = key >> dir_shift;
+#ifdef GFSL_DIR_U32
+    return make_uint2(__ldg((const uint32_t *)d.dir + q), 0u);
 #else
-  auto dir_rank = [&](uint2 e, uint32_t key) -> uint32_t { return key >= e.y ? (e.x / F + 1u) * F : e.x; };
+    return make_uint2(__ldg(d.dir_base + (q >> 5)), (uint32_t)__ldg(d.dir + q));
 #endif
-  uint32_t cur_r = via_dir ? dir_rank(ld_dir(d.dir + (k >> dir_shift)), k) : 0u;
+  };
+  uint32_t cur_r = via_dir ? dir_rank(ld_dir(k), k) : 0u;
   uint32_t cur = via_dir ? l1_chunk(cur_r) : start;
   int level = via_dir ? 1 : height;
   // the next op's directory word is loaded one loop iteration after its raw op (so that
   // its key has arrived), and is ready when the op becomes current
-  uint2 nxt_dir = make_uint2(0u, KEY_POS_INF);
+  uint2 nxt_dir = make_uint2(0u, 0u);
   bool pf_dir = use_dir;
   uint32_t bt = NULL_CHUNK, bt_c = NULL_CHUNK;       // prevKv, reduced
   int seen_top = 0;                                  // highest level where k was seen
@@ -223,7 +220,7 @@ search_kernel(DevState d, const BatchIn in, BatchCtl *__restrict__ ctl, SearchOu
     ld_slice_nc<EPL>(d.pool + (size_t)cur * N + t * EPL, s);  // idle teams re-read `cur`
     if (pf_dir) {
       if ((nxt.op == 0 || (dir_upd && nxt.op <= 2)) && (uint64_t)nxt.key < in.key_range)
-        nxt_dir = ld_dir(d.dir + ((nxt.key + 1u) >> dir_shift));
+        nxt_dir = ld_dir(nxt.key + 1u);
       pf_dir = false;
     }
     if (COUNT && active) {

@@ -95,6 +95,21 @@ def load_library(path: str = LIB_PATH):
             f"{path} is missing: build it with `python -m paper_conf_ppopp_moscovicicp17_b200.build`"
             " (there is no CPU fallback)")
     lib = ctypes.CDLL(path)
+    if os.environ.get("GFSL_LIB"):
+        # an experimental build of another revision (tools/ A/B runs): declare only the
+        # entry points it has
+        class _Tolerant:
+            def __init__(self, l):
+                object.__setattr__(self, "_l", l)
+
+            def __getattr__(self, name):
+                try:
+                    return getattr(self._l, name)
+                except AttributeError:
+                    return type("Missing", (), {})()
+
+        real = lib
+        lib = _Tolerant(real)
     vp, u64, u32, i32 = ctypes.c_void_p, ctypes.c_uint64, ctypes.c_uint32, ctypes.c_int
     lib.gfsl_create.restype = vp
     lib.gfsl_create.argtypes = [u64, u64]
@@ -168,8 +183,8 @@ def load_library(path: str = LIB_PATH):
     lib.gfsl_xr_status.argtypes = [vp]
     lib.gfsl_xr_window.restype = i32
     lib.gfsl_xr_window.argtypes = [vp, ctypes.POINTER(vp), ctypes.POINTER(u64)]
-    _lib = lib
-    return lib
+    _lib = lib._l if hasattr(lib, "_l") else lib
+    return _lib
 
 
 class GFSLError(RuntimeError):

@@ -12,11 +12,14 @@ ap = argparse.ArgumentParser()
 ap.add_argument("config")
 ap.add_argument("--team", type=int, default=0)
 ap.add_argument("--warmup", type=int, default=2)
+ap.add_argument("--prefill", default="bulk", choices=["bulk", "per-op"])
+ap.add_argument("--chunk", type=int, default=0)
 a = ap.parse_args()
 R, pre, B, nb, mix, dist, N = CONFIGS[a.config]
+N = a.chunk or N
 dev = torch.device("cuda")
 g = GFSL(R, capacity=R, chunk_entries=N, contains_team=a.team)
-prefill_gpu(g, R, pre, dev)
+prefill_gpu(g, R, pre, dev, per_op=a.prefill == "per-op")
 w = Workload(R, B, mix=mix, dist=dist, seed=SEED_BASE + 1)
 batches = [make_inputs(w, b, dev) for b in range(a.warmup + 1)]
 for b in range(a.warmup):
