@@ -43,14 +43,11 @@ L2_BYTES = 126 << 20          # B200 L2 (B200_PROFILING.md)
 L2_FLUSH_BYTES = 256 << 20
 
 # name: (R, prefill, batch, n_batches, mix, dist, N)
-# N = chunk entries.  The paper's runs use N = 32.  On B200 the choice follows
-# the memory level that bounds the search: while the upper levels are
-# L2-resident (C1-C4) a chunk read costs L1 data-pipe wavefronts in proportion to its
-# bytes and N = 16 (128-B chunks) wins; at C5 (1B keys) the level-1 gathers go to HBM,
-# whose random-request rate -- not bytes -- is the limit, and N = 32 halves both the
-# level-0 chunk count and level 1 (208 MB instead of 509 MB: more of it stays in L2):
-# measured +26% at C5 in one gpurun call.  The C4 pair compares the two; --chunk N
-# overrides any config.
+# N = chunk entries.  The paper's runs use N = 32; on B200 N = 16 (128-B chunks,
+# 2-lane teams) is faster on every config measured: a chunk read costs L1
+# data-pipe wavefronts in proportion to its bytes, and since level 0 is entered directly
+# from the directory (R37/R38) the smaller level 1 of N = 32 no longer pays off (C5 in one
+# gpurun call: 7534 vs 6660 Mops/s).  The C4 pair compares the two; --chunk N overrides.
 CONFIGS = {
     "C1": (10_000, 5_000, 6_250, 16, (10, 10, 80), "uniform", 16),
     "C2": (1_000_000, 500_000, 625_000, 16, (10, 10, 80), "uniform", 16),
@@ -61,7 +58,7 @@ CONFIGS = {
     "C3-zipf": (10_000_000, 5_000_000, 6_250_000, 16, (10, 10, 80), "zipf", 16),
     "C4-32": (100_000_000, 100_000_000, 50_000_000, 10, (0, 0, 100), "uniform", 32),
     "C4-16": (100_000_000, 100_000_000, 50_000_000, 10, (0, 0, 100), "uniform", 16),
-    "C5": (1_000_000_000, 500_000_000, 125_000_000, 8, (10, 10, 80), "uniform", 32),
+    "C5": (1_000_000_000, 500_000_000, 125_000_000, 8, (10, 10, 80), "uniform", 16),
     # NEXT-4: the paper's other workloads (Fig 5.3 mixes, Fig 5.4b/c single-op runs)
     "M1-1-98": (1_000_000, 500_000, 625_000, 16, (1, 1, 98), "uniform", 16),
     "M5-5-90": (1_000_000, 500_000, 625_000, 16, (5, 5, 90), "uniform", 16),
@@ -764,7 +761,10 @@ def main():
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--runs", type=int, default=10, help="independent runs (fresh prefill each; P:1009)")
     ap.add_argument("--impl", default="gfsl", choices=["gfsl", "reference"])
-    ap.add_argument("--config", default="C5", choices=sorted(CONFIGS))
+    ap.add_argument("--config", default="C5", choices=sorted(CONFIGS) + ["custom"])
+    ap.add_argument("--custom", default=None,
+                    help="R:prefill:batch:batches:i,d,c:dist:N for --config custom (sweeps, "
+                         "tools/sweep_r2.py); dist uniform | zipf | perm")
     ap.add_argument("--team", type=int, default=0)
     ap.add_argument("--chunk", type=int, default=0)
     ap.add_argument("--contains-blocks", type=int, default=0,
@@ -798,6 +798,12 @@ def main():
                     help="L2 access-policy window for the search kernel: 1 = the upper-level pool, "
                          "2 = the level-1 directory (ablations)")
     args = ap.parse_args()
+    if args.config == "custom":
+        R, pre, B, nb, mix, dist, N = args.custom.split(":")
+        CONFIGS["custom"] = (int(R), int(pre), int(B), int(nb), tuple(int(x) for x in mix.split(",")),
+                             dist, int(N))
+        if dist == "perm":
+            PERM_CONFIGS.add("custom")
     if args.warmup < 3:
         args.warmup = 3
     if args.p_chunk <= 0:

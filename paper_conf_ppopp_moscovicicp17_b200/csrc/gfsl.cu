@@ -104,6 +104,7 @@ struct gfsl {
   uint64_t n_policy = 0;    // ops of the current batch as counted by the rebuild policy (R29)
   uint64_t rebuilds = 0;    // upper-level rebuilds enqueued (R24): cross-batch checks reset
   uint64_t live_ub = 0;     // upper bound on the live keys (ops ever submitted), for the bulk path
+  uint32_t l0_entry = 1;    // R37 (GFSL_NO_L0_ENTRY in the environment at create: 0)
   uint64_t bulk_batches = 0;
   // gfsl_check snapshot (V6 / V11)
   uint32_t *snap_max = nullptr;
@@ -255,6 +256,9 @@ static void launch_rebuild(gfsl *h, cudaStream_t s) {
   }
   const RebuildBufs &b = h->rb;
   h->launches += 9;
+  // R38: concurrent-mode rebuilds also relocate level 0 into rank order (serial mode keeps
+  // the paper's layout: its pools are compared byte for byte with Oracle-B)
+  const bool relocate = !h->cfg.serial_updates && h->l0_entry;
   lc.gridDim = dim3(1);
   lc.blockDim = dim3(32);
   cudaLaunchKernelEx(&lc, rebuild_begin_kernel, b);
@@ -269,6 +273,13 @@ static void launch_rebuild(gfsl *h, cudaStream_t s) {
   lc.blockDim = dim3(256);
   lc.gridDim = dim3(h->sms * 4);
   cudaLaunchKernelEx(&lc, rebuild_rank_kernel<N>, h->d, b);
+  if (relocate) {
+    lc.gridDim = dim3(h->sms * 8);
+    cudaLaunchKernelEx(&lc, reloc_out_kernel<N>, h->d, b);
+    cudaLaunchKernelEx(&lc, reloc_in_kernel<N>, h->d, b);
+    cudaLaunchKernelEx(&lc, reloc_reset_kernel<N>, h->d, b);
+    h->launches += 3;
+  }
   lc.gridDim = dim3(h->sms * 8);
   cudaLaunchKernelEx(&lc, rebuild_pack_kernel<N>, h->d, b);
   // R25: reclaim the (now unreachable) zombie level-0 chunks (+ the bitmap clear)
@@ -496,6 +507,10 @@ extern "C" gfsl_t gfsl_create_ex(uint64_t key_range, uint64_t capacity, const gf
   h->cfg = cfg;
   h->key_range = key_range;
   h->capacity = capacity;
+  {
+    const char *e = getenv("GFSL_NO_L0_ENTRY");
+    h->l0_entry = (e && *e && *e != '0') ? 0u : 1u;
+  }
   auto fail = [&](const char *what, cudaError_t e) -> gfsl_t {
     set_last_error(std::string(what) + ": " + cudaGetErrorString(e));
     free_all(h);
@@ -546,11 +561,13 @@ extern "C" gfsl_t gfsl_create_ex(uint64_t key_range, uint64_t capacity, const gf
     if ((e = cudaMalloc(&b.block_sum, (size_t)b.blocks * 4)) != cudaSuccess) return fail("cudaMalloc(rebuild)", e);
     if ((e = cudaMalloc(&b.order_key, (size_t)cap_b * 4)) != cudaSuccess) return fail("cudaMalloc(rebuild)", e);
     if ((e = cudaMalloc(&b.order_chunk, (size_t)cap_b * 4)) != cudaSuccess) return fail("cudaMalloc(rebuild)", e);
-    if ((e = cudaMalloc(&b.n1, 16)) != cudaSuccess) return fail("cudaMalloc(rebuild)", e);
+    if ((e = cudaMalloc(&b.n1, 32)) != cudaSuccess) return fail("cudaMalloc(rebuild)", e);
     if ((e = cudaMalloc(&b.levels, sizeof(RbLevels))) != cudaSuccess) return fail("cudaMalloc(rebuild)", e);
     cudaMemset(b.bitmap, 0, (size_t)b.words * 4);
-    cudaMemset(b.n1, 0, 16);
+    cudaMemset(b.n1, 0, 32);
     h->d.dirty = b.n1 + 2;
+    h->d.dir_oc = b.order_chunk;
+    h->d.dir_ok = b.order_key;
     if ((e = cudaMalloc(&h->d.freelist, (size_t)cap_b * 8)) != cudaSuccess) return fail("cudaMalloc(freelist)", e);
     if ((e = cudaMalloc(&h->d.fl, 8 * 4)) != cudaSuccess) return fail("cudaMalloc(freelist)", e);
     if ((e = cudaMalloc(&h->rc_tiles, ((size_t)cap_b / RC_TILE + 2) * 4)) != cudaSuccess) return fail("cudaMalloc(reclaim)", e);
@@ -737,6 +754,17 @@ static gfsl_status enqueue_batch(gfsl *h, const uint8_t *ops, const uint32_t *ke
                                  const uint32_t *vals, uint8_t *res, uint64_t n, cudaStream_t s,
                                  const uint32_t *n_dev = nullptr, uint64_t n_policy = 0) {
   CK(cudaStreamWaitEvent(s, h->last, 0));
+  {
+    // R36: level-0 loads evict_first, except when level 0 spills the L2 while the upper
+    // levels fit it (C4-like: measured 4% slower with the hint; C3 +11%, C5 +3%).  Sizes
+    // from the bump counters of the previous batch (pinned copy; a heuristic only).
+    const double l2 = 126.0 * (1 << 20);
+    const double l0 = (double)h->h_bump[0] * h->N * 8, up = (double)h->h_bump[1] * h->N * 8;
+    h->d.l0_evict_first = (l0 > l2 && up <= l2) ? 0u : 1u;
+  }
+  // R37: enter level 0 straight from the directory (Contains, and the Insert/Delete of lazy
+  // batches); GFSL_NO_L0_ENTRY (environment, read at gfsl_create) keeps R27's level-1 entry
+  h->d.l0_entry = h->l0_entry;
   h->n_policy = n_dev ? n_policy : n;
   h->d.zparity = (uint32_t)(h->batches & 1);  // R30: this batch's zombie-mark bitmap
 #ifdef GFSL_NO_LAZY_UPPER  // ablation

@@ -67,8 +67,9 @@ struct DevState {
   // lateral step) and one 32-bit base per 32 buckets.  The rebuilt level l holds every
   // F^(l-1)-th level-1 key F per chunk, so the chunk of level l that holds the largest key
   // <= b << shift is chunk r / F^l of that level: chunk l-1 (the head) if 0, else
-  // dir_hdr[32 + l] + r / F^l - 1.  dir_hdr = {shift, valid, buckets, F, ..., [32 + l] =
-  // base of level l}; valid = 0 until the first rebuild (and after gfsl_load).
+  // dir_hdr[32 + l] + r / F^l - 1.  dir_hdr = {shift, valid, buckets, F, l0_ok (R37),
+  // korder (R38: level 0 in rank order), n1, cap_upper, ...,
+  // [32 + l] = base of level l}; valid = 0 until the first rebuild (and after gfsl_load).
   uint8_t *dir;
   uint32_t *dir_base;
   uint32_t *dir_hdr;
@@ -88,6 +89,14 @@ struct DevState {
   uint32_t upkeep_force;  // R33: the deferred upkeep before a rebuild runs even if this
                           // batch merged nothing (earlier lazy batches did)
   uint32_t p_chunk_q32;  // isKeyRaised probability as a 32-bit fraction; 0 = 1 (R16)
+  uint32_t l0_evict_first;  // R36: the search kernel loads level-0 chunks evict_first
+  // R37: the rebuild's rank order of the level-0 chunks (RebuildBufs::order_chunk): entry
+  // r-1 is the level-0 chunk whose min key is the r-th level-1 key, i.e. level-1 entry r's
+  // down pointer, stored densely; with the directory's rank it lets a traversal enter
+  // level 0 directly.  l0_entry = 1: the search kernel does so (concurrent modes).
+  const uint32_t *dir_oc;
+  const uint32_t *dir_ok;  // R38: the sorted min keys of the last rebuild (order_key)
+  uint32_t l0_entry;
 };
 
 // isKeyRaised's draw (R28): a counter-based hash of (raised key, level of the split), the
@@ -190,45 +199,65 @@ struct ChunkSlice {
 };
 
 template <int EPL>
-__device__ __forceinline__ void ld_slice_nc(const uint64_t *p, ChunkSlice<EPL> &s);
+__device__ __forceinline__ void ld_slice_nc(const uint64_t *p, ChunkSlice<EPL> &s, uint64_t pol);
+
+// The chunk loads of the search phase carry an L2 eviction-priority policy (createpolicy):
+// level-0 chunks evict_first (a 1B-key level 0 is streamed, ~5 reads per line per batch),
+// the upper levels and the directory evict_last, so that the L2 keeps as much of level 1
+// as fits (R36).
+__device__ __forceinline__ uint64_t l2_policy_evict_first() {
+  uint64_t p;
+  asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(p));
+  return p;
+}
+__device__ __forceinline__ uint64_t l2_policy_evict_last() {
+  uint64_t p;
+  asm volatile("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(p));
+  return p;
+}
+__device__ __forceinline__ uint64_t l2_policy_evict_normal() {
+  uint64_t p;
+  asm volatile("createpolicy.fractional.L2::evict_normal.b64 %0, 1.0;" : "=l"(p));
+  return p;
+}
 
 template <>
-__device__ __forceinline__ void ld_slice_nc<1>(const uint64_t *p, ChunkSlice<1> &s) {
-  asm volatile("ld.global.nc.v2.u32 {%0,%1}, [%2];" : "=r"(s.k[0]), "=r"(s.v[0]) : "l"(p));
+__device__ __forceinline__ void ld_slice_nc<1>(const uint64_t *p, ChunkSlice<1> &s, uint64_t pol) {
+  asm volatile("ld.global.nc.L2::cache_hint.v2.u32 {%0,%1}, [%2], %3;" : "=r"(s.k[0]), "=r"(s.v[0]) : "l"(p), "l"(pol));
 }
 template <>
-__device__ __forceinline__ void ld_slice_nc<2>(const uint64_t *p, ChunkSlice<2> &s) {
-  asm volatile("ld.global.nc.v4.u32 {%0,%1,%2,%3}, [%4];"
+__device__ __forceinline__ void ld_slice_nc<2>(const uint64_t *p, ChunkSlice<2> &s, uint64_t pol) {
+  asm volatile("ld.global.nc.L2::cache_hint.v4.u32 {%0,%1,%2,%3}, [%4], %5;"
                : "=r"(s.k[0]), "=r"(s.v[0]), "=r"(s.k[1]), "=r"(s.v[1])
-               : "l"(p));
+               : "l"(p), "l"(pol));
 }
 template <>
-__device__ __forceinline__ void ld_slice_nc<4>(const uint64_t *p, ChunkSlice<4> &s) {
-  asm volatile("ld.global.nc.v8.u32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];"
+__device__ __forceinline__ void ld_slice_nc<4>(const uint64_t *p, ChunkSlice<4> &s, uint64_t pol) {
+  asm volatile("ld.global.nc.L2::cache_hint.v8.u32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8], %9;"
                : "=r"(s.k[0]), "=r"(s.v[0]), "=r"(s.k[1]), "=r"(s.v[1]), "=r"(s.k[2]),
                  "=r"(s.v[2]), "=r"(s.k[3]), "=r"(s.v[3])
-               : "l"(p));
+               : "l"(p), "l"(pol));
 }
 template <>
-__device__ __forceinline__ void ld_slice_nc<8>(const uint64_t *p, ChunkSlice<8> &s) {
-  asm volatile("ld.global.nc.v8.u32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];"
+__device__ __forceinline__ void ld_slice_nc<8>(const uint64_t *p, ChunkSlice<8> &s, uint64_t pol) {
+  asm volatile("ld.global.nc.L2::cache_hint.v8.u32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8], %9;"
                : "=r"(s.k[0]), "=r"(s.v[0]), "=r"(s.k[1]), "=r"(s.v[1]), "=r"(s.k[2]),
                  "=r"(s.v[2]), "=r"(s.k[3]), "=r"(s.v[3])
-               : "l"(p));
-  asm volatile("ld.global.nc.v8.u32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];"
+               : "l"(p), "l"(pol));
+  asm volatile("ld.global.nc.L2::cache_hint.v8.u32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8], %9;"
                : "=r"(s.k[4]), "=r"(s.v[4]), "=r"(s.k[5]), "=r"(s.v[5]), "=r"(s.k[6]),
                  "=r"(s.v[6]), "=r"(s.k[7]), "=r"(s.v[7])
-               : "l"(p + 4));
+               : "l"(p + 4), "l"(pol));
 }
 
 template <>
-__device__ __forceinline__ void ld_slice_nc<16>(const uint64_t *p, ChunkSlice<16> &s) {
+__device__ __forceinline__ void ld_slice_nc<16>(const uint64_t *p, ChunkSlice<16> &s, uint64_t pol) {
 #pragma unroll
   for (int q = 0; q < 4; ++q)
-    asm volatile("ld.global.nc.v8.u32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];"
+    asm volatile("ld.global.nc.L2::cache_hint.v8.u32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8], %9;"
                  : "=r"(s.k[4 * q]), "=r"(s.v[4 * q]), "=r"(s.k[4 * q + 1]), "=r"(s.v[4 * q + 1]),
                    "=r"(s.k[4 * q + 2]), "=r"(s.v[4 * q + 2]), "=r"(s.k[4 * q + 3]), "=r"(s.v[4 * q + 3])
-                 : "l"(p + 4 * q));
+                 : "l"(p + 4 * q), "l"(pol));
 }
 
 // Programmatic dependent launch: a kernel launched with programmatic stream serialization

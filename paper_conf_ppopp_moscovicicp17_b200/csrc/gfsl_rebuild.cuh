@@ -33,7 +33,8 @@ struct RebuildBufs {
   uint32_t *block_sum;    // [blocks]     popcount of each block, then its exclusive prefix
   uint32_t *order_key;    // [cap_bottom] min keys in key order
   uint32_t *order_chunk;  // [cap_bottom] their chunks
-  uint32_t *n1;           // [4]          marked chunks; old upper bump; dirty; active
+  uint32_t *n1;           // [8]          marked chunks; old upper bump; dirty; active;
+                          //              relocated (R38)
   void *levels;           // RbLevels computed once per rebuild (scan_top kernel)
   uint32_t words, blocks;
   uint32_t fill;          // F: entries per rebuilt upper chunk
@@ -98,6 +99,7 @@ __global__ void rebuild_begin_kernel(RebuildBufs b) {
   pdl_wait();
   b.n1[3] = b.n1[2];
   b.n1[2] = 0;
+  b.n1[4] = 0;  // R38: set by reloc_out_kernel when level 0 is relocated
 }
 
 // (1) mark min keys of the live non-first level-0 chunks
@@ -206,6 +208,73 @@ __global__ void __launch_bounds__(256) rebuild_rank_kernel(const __grid_constant
   }
 }
 
+// ---- R38: level 0 relocated into rank order (concurrent-mode rebuilds) -------------------
+// After the rank kernel, level 0 is copied chunk by chunk in key order into the bottom
+// pool's unused tail (the scratch: chunks [used, used + m), m = n1 + 1 live chunks), then
+// back to [0, m): chunk j holds the j-th chunk in key order (j = 0: the first chunk, -inf),
+// NEXT = j + 1, the last (+inf, NULL).  Zombies, the free list and the unused chunks are
+// gone (reset to the allocated state of P:237).  The rank of a key among the level-1 keys
+// then IS its level-0 chunk, so a traversal can enter level 0 from the directory's rank
+// refined by one 32-B read of the sorted min keys (R38 in the search kernel).
+template <int N>
+__global__ void __launch_bounds__(256) reloc_out_kernel(const __grid_constant__ DevState d, RebuildBufs b) {
+  pdl_wait();
+  if (!rb_active(b)) return;
+  const uint32_t n1 = b.n1[0];
+  const uint32_t used = min(d.bump[0], d.cap_bottom);
+  const uint32_t m = n1 + 1;
+  if ((uint64_t)used + m > d.cap_bottom) return;  // no room for the scratch: no relocation
+  const uint32_t S = d.cap_upper + used;
+  const int lane = threadIdx.x & 31;
+  const uint32_t warp = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  const uint32_t nwarps = (gridDim.x * blockDim.x) >> 5;
+  const uint32_t head0 = d.head[0];
+  for (uint32_t j = warp; j < m; j += nwarps) {
+    const uint32_t src = j ? b.order_chunk[j - 1] : head0;
+    if (lane < N) {
+      uint64_t e = d.pool[(size_t)src * N + lane];
+      if (lane == N - 2) e = (j + 1 < m) ? mk64(lo32(e), d.cap_upper + j + 1) : mk64(KEY_POS_INF, NULL_CHUNK);
+      if (lane == N - 1) e = mk64(LOCK_FREE, 0u);
+      d.pool[(size_t)(S + j) * N + lane] = e;
+    }
+  }
+  if (blockIdx.x == 0 && threadIdx.x == 0) b.n1[4] = 1u;
+}
+
+template <int N>
+__global__ void __launch_bounds__(256) reloc_in_kernel(const __grid_constant__ DevState d, RebuildBufs b) {
+  pdl_wait();
+  if (!rb_active(b) || !b.n1[4]) return;
+  const uint32_t n1 = b.n1[0], m = n1 + 1;
+  const uint32_t used = min(d.bump[0], d.cap_bottom);
+  const uint32_t S = d.cap_upper + used;
+  const uint64_t total = (uint64_t)m * N;
+  for (uint64_t e = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; e < total; e += (uint64_t)gridDim.x * blockDim.x)
+    d.pool[(size_t)d.cap_upper * N + e] = d.pool[(size_t)S * N + e];
+  for (uint32_t j = blockIdx.x * blockDim.x + threadIdx.x; j < n1; j += gridDim.x * blockDim.x)
+    b.order_chunk[j] = d.cap_upper + j + 1;  // the pack kernel's level-1 down pointers
+}
+
+template <int N>
+__global__ void __launch_bounds__(256) reloc_reset_kernel(const __grid_constant__ DevState d, RebuildBufs b) {
+  pdl_wait();
+  if (!rb_active(b) || !b.n1[4]) return;
+  const uint32_t n1 = b.n1[0], m = n1 + 1;
+  const uint32_t used = min(d.bump[0], d.cap_bottom);
+  const uint64_t first = (uint64_t)(d.cap_upper + m) * N, last = (uint64_t)(d.cap_upper + used + m) * N;
+  const uint64_t tid = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x, stride = (uint64_t)gridDim.x * blockDim.x;
+  for (uint64_t e = first + tid; e < last; e += stride)
+    d.pool[e] = ((e % N) == (uint64_t)(N - 1)) ? (uint64_t)LOCK_HELD : EMPTY_ENTRY;
+  for (uint64_t w = tid; w < 2ull * d.zwords; w += stride) d.zbits[w] = 0u;  // no zombie left
+  if (blockIdx.x == 0 && threadIdx.x == 0) {
+    const bool any = n1 > 0 || lo32(d.pool[(size_t)d.cap_upper * N + 1]) != KEY_EMPTY;
+    d.head[0] = d.cap_upper;
+    d.counter[0] = any ? (int32_t)m : 0;
+    d.bump[0] = m;
+    d.fl[0] = d.fl[1] = 0;  // the free list (R25) is empty: nothing left to reclaim
+  }
+}
+
 // (5) write every chunk of levels >= 1; one warp per chunk, lane e writes entry e.  And
 // the level-1 directory (R27).
 template <int N>
@@ -248,6 +317,12 @@ __global__ void __launch_bounds__(256) rebuild_pack_kernel(const __grid_constant
         d.dir_hdr[1] = 1u;
         d.dir_hdr[2] = buckets;
         d.dir_hdr[3] = b.fill;
+        // R37: entering level 0 from a bucket's rank costs ~(level-1 keys per bucket) / 2
+        // lateral steps there; worth it only while the directory holds >= 1 bucket per key
+        d.dir_hdr[4] = buckets >= n1 ? 1u : 0u;
+        d.dir_hdr[5] = b.n1[4];  // R38: level 0 in rank order (chunk cap_upper + rank)
+        d.dir_hdr[6] = n1;       // R38: min keys in order_key
+        d.dir_hdr[7] = d.cap_upper;
       }
     }
   }

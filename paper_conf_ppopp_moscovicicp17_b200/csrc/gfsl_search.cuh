@@ -108,7 +108,7 @@ search_kernel(DevState d, const BatchIn in, BatchCtl *__restrict__ ctl, SearchOu
   constexpr int LOCK_LANE = LOCK_E / EPL, LOCK_J = LOCK_E % EPL;
   constexpr uint32_t FULL = 0xFFFFFFFFu;
 
-  __shared__ uint32_t s_start, s_height, s_dir_shift;
+  __shared__ uint32_t s_start, s_height, s_dir_shift, s_head0, s_l0_ok, s_korder, s_n1;
   __shared__ uint32_t s_dir_base[PLAN_LEVELS];  // base of each rebuilt level (R27)
   // the path of the team's current op (written by its lane 0 only), copied out compactly
   // at the end if the op mutates (about 1 op in 10)
@@ -124,6 +124,10 @@ search_kernel(DevState d, const BatchIn in, BatchCtl *__restrict__ ctl, SearchOu
     if (lane == 0) {
       s_height = h;
       s_start = d.head[h];
+      s_head0 = d.head[0];
+      s_l0_ok = d.dir_hdr[4];
+      s_korder = d.dir_hdr[5];
+      s_n1 = d.dir_hdr[6];
       // R27: Contains enter at level 1 through the directory when there are levels above
       s_dir_shift = (h >= 2 && d.dir_hdr[1]) ? d.dir_hdr[0] : 32u;
       if (blockIdx.x == 0) ctl->snap_height = h;
@@ -148,6 +152,15 @@ search_kernel(DevState d, const BatchIn in, BatchCtl *__restrict__ ctl, SearchOu
     return use_dir && !(opw & INVALID_FLAG) && (dir_upd || !(opw & UPDATE_FLAG));
   };
   auto l1_chunk = [&](uint32_t r) { const uint32_t q = r / F; return q ? s_dir_base[1] + q - 1u : 0u; };
+  // R37: enter at level 0, in the chunk of level-1 entry r's down pointer (the rebuild's
+  // rank order); the levels above are skipped (their path entries come from r, as R27's)
+  const bool korder = s_korder != 0;   // R38: level 0 in rank order
+  const uint32_t n1 = s_n1;
+  const bool l0_entry = d.l0_entry != 0 && (s_l0_ok != 0 || korder);
+  const uint32_t head0 = s_head0;
+  // an Insert/Delete may skip the upper levels only in a lazy batch (R33: no raise, no
+  // upper-level delete); otherwise it enters at level 1 (R27) to see its exact top
+  auto l0_op = [&](uint32_t opw) { return l0_entry && (d.lazy_upper || !(opw & UPDATE_FLAG)); };
   const uint32_t n = in.n_dev ? min(*(volatile const uint32_t *)in.n_dev, in.n) : in.n;
   uint8_t *__restrict__ res = in.res;
 
@@ -193,6 +206,13 @@ search_kernel(DevState d, const BatchIn in, BatchCtl *__restrict__ ctl, SearchOu
   bool active = lane_live && slot < n;
   uint32_t k = cur_op.y;
   bool via_dir = dir_op(cur_op.x);
+  // R36: L2 eviction priorities -- level-0 chunks evict_first (when the host chose it for
+  // this structure's size), the upper levels and the directory evict_last
+#ifndef GFSL_SEARCH_HINTS
+#define GFSL_SEARCH_HINTS 2
+#endif
+  const uint64_t pol_l0 = (GFSL_SEARCH_HINTS >= 1 && d.l0_evict_first) ? l2_policy_evict_first() : l2_policy_evict_normal();
+  const uint64_t pol_up = GFSL_SEARCH_HINTS >= 2 ? l2_policy_evict_last() : l2_policy_evict_normal();
   // the op's directory rank (R27b): base of its 32-bucket group + its byte
   auto dir_rank = [&](uint2 e, uint32_t) -> uint32_t { return e.x + e.y; };
   auto ld_dir = [&](uint32_t key) -> uint2 {
@@ -200,12 +220,35 @@ search_kernel(DevState d, const BatchIn in, BatchCtl *__restrict__ ctl, SearchOu
 #ifdef GFSL_DIR_U32
     return make_uint2(__ldg((const uint32_t *)d.dir + q), 0u);
 #else
-    return make_uint2(__ldg(d.dir_base + (q >> 5)), (uint32_t)__ldg(d.dir + q));
+    uint32_t base, byte;
+    asm volatile("ld.global.nc.L2::cache_hint.u32 %0, [%1], %2;" : "=r"(base) : "l"(d.dir_base + (q >> 5)), "l"(pol_up));
+    asm volatile("ld.global.nc.L2::cache_hint.u8 %0, [%1], %2;" : "=r"(byte) : "l"(d.dir + q), "l"(pol_up));
+    return make_uint2(base, byte);
 #endif
   };
+  auto l0_chunk = [&](uint32_t r, uint32_t key) -> uint32_t {
+    if (korder) {
+      // R38: rank(key) = r + the sorted min keys >= index r that are <= key; one aligned
+      // 32-B read covers the 8 keys of r's group (those before r are <= key already)
+      const uint32_t g = r & ~7u;
+      uint32_t o[8];
+      asm volatile("ld.global.nc.L2::cache_hint.v8.u32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8], %9;"
+                   : "=r"(o[0]), "=r"(o[1]), "=r"(o[2]), "=r"(o[3]), "=r"(o[4]), "=r"(o[5]), "=r"(o[6]), "=r"(o[7])
+                   : "l"(d.dir_ok + g), "l"(pol_up));
+      uint32_t rho = g;
+#pragma unroll
+      for (int i = 0; i < 8; ++i) rho += (g + i < n1 && o[i] <= key) ? 1u : 0u;
+      return d.cap_upper + rho;  // the chunk of rank rho (rho = g + 8: laterally onward from there)
+    }
+    if (!r) return head0;
+    uint32_t c;
+    asm volatile("ld.global.nc.L2::cache_hint.u32 %0, [%1], %2;" : "=r"(c) : "l"(d.dir_oc + r - 1), "l"(pol_up));
+    return c;
+  };
   uint32_t cur_r = via_dir ? dir_rank(ld_dir(k), k) : 0u;
-  uint32_t cur = via_dir ? l1_chunk(cur_r) : start;
-  int level = via_dir ? 1 : height;
+  bool via_l0 = via_dir && l0_op(cur_op.x);
+  uint32_t cur = via_dir ? (via_l0 ? l0_chunk(cur_r, k) : l1_chunk(cur_r)) : start;
+  int level = via_dir ? (via_l0 ? 0 : 1) : height;
   // the next op's directory word is loaded one loop iteration after its raw op (so that
   // its key has arrived), and is ready when the op becomes current
   uint2 nxt_dir = make_uint2(0u, 0u);
@@ -217,7 +260,7 @@ search_kernel(DevState d, const BatchIn in, BatchCtl *__restrict__ ctl, SearchOu
 
   while (__any_sync(FULL, active)) {
     ChunkSlice<EPL> s;
-    ld_slice_nc<EPL>(d.pool + (size_t)cur * N + t * EPL, s);  // idle teams re-read `cur`
+    ld_slice_nc<EPL>(d.pool + (size_t)cur * N + t * EPL, s, level == 0 ? pol_l0 : pol_up);  // idle teams re-read `cur`
     if (pf_dir) {
       if ((nxt.op == 0 || (dir_upd && nxt.op <= 2)) && (uint64_t)nxt.key < in.key_range)
         nxt_dir = ld_dir(nxt.key + 1u);
@@ -286,6 +329,7 @@ search_kernel(DevState d, const BatchIn in, BatchCtl *__restrict__ ctl, SearchOu
         restarts += redo ? 0 : 1;
         seen_top = 0;
         via_dir = false;
+        via_l0 = false;
         bt = bt_c = NULL_CHUNK;
       }
       if (done) {
@@ -307,8 +351,9 @@ search_kernel(DevState d, const BatchIn in, BatchCtl *__restrict__ ctl, SearchOu
               // next rebuild, as stale separators)
               so.mut_rec[m] = make_uint4(w, k, here, (cur_op.x & DELETE_FLAG) ? (d.lazy_upper ? 0u : (uint32_t)seen_top) : cur_val);
               my_path[0] = here;  // path[0] = the enclosing bottom chunk
-              if (via_dir) {      // levels >= 2 from the directory rank (R27)
+              if (via_dir) {      // levels >= 2 (and 1, R37) from the directory rank (R27)
                 uint32_t q = cur_r / F;
+                if (via_l0) my_path[1] = q ? s_dir_base[1] + q - 1u : 0u;
 #pragma unroll
                 for (int l = 2; l < PLAN_LEVELS; ++l) {
                   q /= F;
@@ -338,8 +383,9 @@ search_kernel(DevState d, const BatchIn in, BatchCtl *__restrict__ ctl, SearchOu
         nxt = load_raw(slot + total_teams);
         via_dir = dir_op(cur_op.x);
         cur_r = dir_rank(nxt_dir, k);
-        cur = via_dir ? l1_chunk(cur_r) : start;
-        level = via_dir ? 1 : height;
+        via_l0 = via_dir && l0_op(cur_op.x);
+        cur = via_dir ? (via_l0 ? l0_chunk(cur_r, k) : l1_chunk(cur_r)) : start;
+        level = via_dir ? (via_l0 ? 0 : 1) : height;
         pf_dir = use_dir;
         bt = bt_c = NULL_CHUNK;
         seen_top = 0;

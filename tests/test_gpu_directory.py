@@ -16,11 +16,16 @@ from .test_gpu_parity import check_same_set, prefill, run_batch
 pytestmark = pytest.mark.gpu
 
 
-@pytest.mark.parametrize("N,serial", [(16, True), (32, True), (16, False), (32, False)])
-def test_stale_directory_restarts(N, serial):
+@pytest.mark.parametrize("N,serial,l0", [(16, True, False), (32, True, False), (16, False, False),
+                                          (32, False, False), (16, True, True), (32, False, True)])
+def test_stale_directory_restarts(N, serial, l0, monkeypatch):
     """Serial mode removes deleted keys from the upper levels (Alg 4.11), so the directory
-    goes stale and Contains restart; concurrent batches leave them as separators until the
-    next rebuild (R33), which must answer the same."""
+    goes stale and Contains entered at level 1 (R27) restart; concurrent batches leave them
+    as separators until the next rebuild (R33), which must answer the same.  With the
+    level-0 entry (R37, the default) the same batches go through the rebuild's rank order
+    of level-0 chunks, which zombies and splits since the rebuild only lengthen laterally."""
+    if not l0:
+        monkeypatch.setenv("GFSL_NO_L0_ENTRY", "1")
     R = 40_000
     g = GFSL(R, chunk_entries=N, rebuild_every=3, serial_updates=serial)
     o = OracleMap(R)
@@ -34,7 +39,7 @@ def test_stale_directory_restarts(N, serial):
     # Contains of every key (and some out of range) before the next rebuild
     ck = np.concatenate([np.arange(R, dtype=np.uint32), np.array([R, R + 5], np.uint32)])
     run_batch(g, o, np.zeros(ck.size, np.uint8), ck, None)
-    if serial:
+    if serial and not l0:
         assert g.stats()["restarts"] > r0, "the stale-directory path was not exercised"
     check_same_set(g, o)
     # churn with re-inserts, then more Contains, across rebuilds
