@@ -37,9 +37,12 @@ __device__ __forceinline__ uint64_t bk_payload(uint32_t value, uint32_t idx, uin
 __device__ __forceinline__ uint32_t bk_kind(uint64_t p) { return (uint32_t)(p >> 62); }
 __device__ __forceinline__ uint32_t bk_idx(uint64_t p) { return (uint32_t)(p >> 32) & 0x1FFFFFFFu; }
 
+#ifndef GFSL_BULK_FILL10
+#define GFSL_BULK_FILL10 7  // tenths of DSIZE
+#endif
 template <int N>
 constexpr uint32_t bk_fill() {
-  return (uint32_t)(((N - 2) * 7 + 5) / 10);  // round(0.7 DSIZE): 10 at N = 16, 21 at N = 32
+  return (uint32_t)(((N - 2) * GFSL_BULK_FILL10 + 5) / 10);  // round(0.7 DSIZE): 10 at N = 16, 21 at N = 32
 }
 
 // (1) ops at [0, n), the live level-0 entries at [n, n + used_b * DSIZE); invalid ops are

@@ -61,6 +61,10 @@ struct BatchIn {
   uint64_t key_range;
   const uint32_t *n_dev;     // NULL, or device word holding the op count (gfsl_batch_dn):
                              // the batch has min(*n_dev, n) ops, read at kernel time
+  // Key-ordered intake (R39), or NULL: slot j is the j-th op in key order -- op sw[j] &
+  // OPI_MASK, its op code (capped at 3 = invalid) in bits 29-30 of sw[j], its key skey[j]
+  const uint32_t *skey;
+  const uint32_t *sw;
 };
 
 // The mutations a batch's search phase hands to the update phase, compact: mutation m
@@ -157,6 +161,7 @@ search_kernel(DevState d, const BatchIn in, BatchCtl *__restrict__ ctl, SearchOu
   const bool korder = s_korder != 0;   // R38: level 0 in rank order
   const uint32_t n1 = s_n1;
   const bool l0_entry = d.l0_entry != 0 && (s_l0_ok != 0 || korder);
+  const bool fine_dir = s_l0_ok != 0;  // >= 1 directory bucket per level-1 key
   const uint32_t head0 = s_head0;
   // an Insert/Delete may skip the upper levels only in a lazy batch (R33: no raise, no
   // upper-level delete); otherwise it enters at level 1 (R27) to see its exact top
@@ -179,24 +184,33 @@ search_kernel(DevState d, const BatchIn in, BatchCtl *__restrict__ ctl, SearchOu
   // The prefetched op stays raw (loaded, not yet looked at) until it becomes current, so
   // its loads overlap the current traversal.
   // An Insert's value is loaded when the op becomes current (it is needed only at its end).
+  // R39: with a key-ordered intake, slot j carries its input index
   struct RawOp {
-    uint32_t op, key;
+    uint32_t op, key, idx;
   };
   auto load_raw = [&](uint32_t i) -> RawOp {
-    RawOp r{3u, 0u};
+    RawOp r{3u, 0u, i};
     if (lane_live && i < n) {
-      r.op = __ldg(in.ops + i);
-      r.key = __ldg(in.keys + i);
+      if (in.sw) {
+        const uint32_t w = __ldg(in.sw + i);
+        r.op = (w >> 29) & 3u;
+        r.idx = w & OPI_MASK;
+        r.key = __ldg(in.skey + i);
+      } else {
+        r.op = __ldg(in.ops + i);
+        r.key = __ldg(in.keys + i);
+      }
     }
     return r;
   };
   auto load_val = [&](uint32_t i, const RawOp &r) -> uint32_t {
-    return (t == 0 && in.vals && r.op == 1 && lane_live && i < n) ? __ldg(in.vals + i) : 0u;
+    return (t == 0 && in.vals && r.op == 1 && lane_live && i < n) ? __ldg(in.vals + r.idx) : 0u;
   };
   auto decode = [&](uint32_t i, const RawOp &r) -> uint2 {
+    (void)i;
     const bool valid = r.op <= 2 && (uint64_t)r.key < in.key_range;
     const uint32_t fl = !valid ? INVALID_FLAG : (r.op == 2 ? (DELETE_FLAG | UPDATE_FLAG) : (r.op == 1 ? UPDATE_FLAG : 0u));
-    return make_uint2(i | fl, valid ? r.key + 1u : 1u);
+    return make_uint2(r.idx | fl, valid ? r.key + 1u : 1u);
   };
   uint32_t slot = warp_global * TPW + team_in_warp;  // this team's current op slot
   RawOp raw = load_raw(slot);
@@ -228,17 +242,32 @@ search_kernel(DevState d, const BatchIn in, BatchCtl *__restrict__ ctl, SearchOu
   };
   auto l0_chunk = [&](uint32_t r, uint32_t key) -> uint32_t {
     if (korder) {
-      // R38: rank(key) = r + the sorted min keys >= index r that are <= key; one aligned
-      // 32-B read covers the 8 keys of r's group (those before r are <= key already)
-      const uint32_t g = r & ~7u;
-      uint32_t o[8];
-      asm volatile("ld.global.nc.L2::cache_hint.v8.u32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8], %9;"
-                   : "=r"(o[0]), "=r"(o[1]), "=r"(o[2]), "=r"(o[3]), "=r"(o[4]), "=r"(o[5]), "=r"(o[6]), "=r"(o[7])
-                   : "l"(d.dir_ok + g), "l"(pol_up));
-      uint32_t rho = g;
+      // R38: rank(key) = r + the sorted min keys >= index r that are <= key (those before
+      // r are <= key already).  A fine directory (>= 1 bucket per key) needs a short look-
+      // ahead: one aligned 32-B read of r's group of 8; a coarse one (C5: ~3 keys per
+      // bucket) three aligned 16-B reads from r rounded down to 4, >= 9 keys past r.
+      if (fine_dir) {
+        const uint32_t g = r & ~7u;
+        uint32_t o[8];
+        asm volatile("ld.global.nc.L2::cache_hint.v8.u32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8], %9;"
+                     : "=r"(o[0]), "=r"(o[1]), "=r"(o[2]), "=r"(o[3]), "=r"(o[4]), "=r"(o[5]), "=r"(o[6]), "=r"(o[7])
+                     : "l"(d.dir_ok + g), "l"(pol_up));
+        uint32_t rho = g;
 #pragma unroll
-      for (int i = 0; i < 8; ++i) rho += (g + i < n1 && o[i] <= key) ? 1u : 0u;
-      return d.cap_upper + rho;  // the chunk of rank rho (rho = g + 8: laterally onward from there)
+        for (int i = 0; i < 8; ++i) rho += (g + i < n1 && o[i] <= key) ? 1u : 0u;
+        return d.cap_upper + rho;  // the chunk of rank rho (rho = g + 8: laterally onward)
+      }
+      const uint32_t s0 = r & ~3u;
+      uint32_t o[12];
+#pragma unroll
+      for (int q = 0; q < 3; ++q)
+        asm volatile("ld.global.nc.L2::cache_hint.v4.u32 {%0,%1,%2,%3}, [%4], %5;"
+                     : "=r"(o[4 * q]), "=r"(o[4 * q + 1]), "=r"(o[4 * q + 2]), "=r"(o[4 * q + 3])
+                     : "l"(d.dir_ok + s0 + 4 * q), "l"(pol_up));
+      uint32_t rho = s0;
+#pragma unroll
+      for (int i = 0; i < 12; ++i) rho += (s0 + i < n1 && o[i] <= key) ? 1u : 0u;
+      return d.cap_upper + rho;  // the chunk of rank rho (rho = s0 + 12: laterally onward)
     }
     if (!r) return head0;
     uint32_t c;
@@ -417,6 +446,13 @@ struct MutMap {
     for (int step = BatchCtl::MUT_REGIONS / 2; step >= 1; step >>= 1)
       if (excl[r + step] <= s) r += step;
     return (uint32_t)r * cap + (s - excl[r]);
+  }
+  // The same for a caller whose slots only grow (a work queue's items, no spread): the
+  // region cursor moves forward, O(1) amortised instead of a 5-step binary search.
+  __device__ __forceinline__ uint32_t rec_fwd(uint32_t s, uint32_t &rg) const {
+    if (spread) return rec(s);
+    while (rg + 1 < (uint32_t)BatchCtl::MUT_REGIONS && excl[rg + 1] <= s) ++rg;
+    return rg * cap + (s - excl[rg]);
   }
 };
 

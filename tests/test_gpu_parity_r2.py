@@ -230,3 +230,28 @@ def test_device_check_cross_batch_v6_v11():
     g.load(meta1, bad)
     v = g.check(cross=True, raise_on_violation=False)
     assert v.violations & (1 << 10)
+
+
+@pytest.mark.parametrize("spread", [False, True])
+def test_key_ordered_intake_matches_oracle(spread, monkeypatch):
+    """R39: the intake sorted by key (forced on a small structure here) changes the order in
+    which the search phase takes the ops, never a result: every result, the set and the
+    invariants equal Oracle-A's, with invalid ops and extreme keys mixed in."""
+    monkeypatch.setenv("GFSL_KEY_ORDER", "1")
+    if spread:
+        monkeypatch.setenv("GFSL_KO_SPREAD", "1")
+    R = 200_000
+    g = GFSL(R)
+    o = OracleMap(R)
+    k = np.random.default_rng(4).permutation(R)[: R // 2].astype(np.uint32)
+    run_batch(g, o, np.ones(k.size, np.uint8), k, k)     # bulk (R34) + rebuild (R38)
+    for b, (op, key, val) in enumerate(batches(R, 60_000, 8, (20, 20, 60), SEED_BASE + 333)):
+        op = op.copy()
+        if b == 2:
+            op[::97] = 7
+            key = key.copy()
+            key[::89] = R + 11
+            key[5] = R - 1
+            key[6] = 0
+        run_batch(g, o, op, key, val)
+        check_all(g, o)

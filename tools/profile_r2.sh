@@ -20,7 +20,9 @@ for c in $CFGS; do
 done
 if [ -z "${NO_FULL:-}" ]; then
   timeout 2400 ncu --replay-mode application --profile-from-start off --set full --import-source on \
-    --clock-control none --cache-control all -k regex:search_kernel -f -o $O/full_C5_search \
+    --clock-control none --cache-control all -k "regex:search_kernel|update_kernel" -f -o $O/full_C5 \
     python tools/prof_step.py C5 > $O/full_C5.log 2>&1
-  python tools/ncu_metrics.py $O/full_C5_search.ncu-rep > $O/ncu_full_C5_search.json 2>&1
+  python tools/ncu_metrics.py $O/full_C5.ncu-rep > $O/ncu_full_C5.json 2>&1
+  ncu -i $O/full_C5.ncu-rep --page details --csv > $O/full_C5_details.csv 2>&1
+  ncu -i $O/full_C5.ncu-rep --page source --csv -k regex:update_kernel > $O/full_C5_update_source.csv 2>&1
 fi

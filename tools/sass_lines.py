@@ -15,9 +15,14 @@ rep, kname, nregex = sys.argv[1], sys.argv[2], sys.argv[3]
 lib = sys.argv[4] if len(sys.argv) > 4 else "paper_conf_ppopp_moscovicicp17_b200/libgfsl.so"
 tmp = tempfile.mkdtemp()
 subprocess.run(["cuobjdump", "-xelf", "all", os.path.abspath(lib)], cwd=tmp, capture_output=True)
-cubin = [f for f in os.listdir(tmp) if f.endswith(".cubin")][0]
-sass = subprocess.run(["nvdisasm", "-g", "-c", os.path.join(tmp, cubin)], capture_output=True, text=True).stdout.split("\n")
-start = [i for i, l in enumerate(sass) if l.startswith(".text." + kname)][0]
+sass, start = None, None
+for cubin in sorted(f for f in os.listdir(tmp) if f.endswith(".cubin")):
+    lines = subprocess.run(["nvdisasm", "-g", "-c", os.path.join(tmp, cubin)], capture_output=True,
+                           text=True).stdout.split("\n")
+    hits = [i for i, l in enumerate(lines) if l.startswith(".text." + kname)]
+    if hits:
+        sass, start = lines, hits[0]
+        break
 cur, off2line = None, {}
 for l in sass[start + 1:]:
     if l.startswith(".text."):
