@@ -97,7 +97,12 @@ constexpr uint32_t CW_DEL = 0x40000000u;     // Delete (else Insert)
 constexpr uint32_t CW_NOTMUT = 0x20000000u;  // Contains or invalid: not part of any chain
 
 #ifndef GFSL_SEARCH_MIN_BLOCKS
-#define GFSL_SEARCH_MIN_BLOCKS 1
+// 4 blocks per SM (<= 64 registers, no spill): with level 0 entered directly (R37/R38) a
+// traversal is ~1-2 dependent gathers, latency-bound (ncu at C5: 0.45 eligible warps per
+// scheduler at 3 blocks), so more resident warps win -- one gpurun call, 3 -> 4 blocks:
+// C5 7664 -> 8088, C4-16 15575 -> 21173, C3 8109 -> 8808, C2 4962 -> 5449 Mops/s (5 and 6
+// blocks, 48 / 40 registers, lose at C4 / C5)
+#define GFSL_SEARCH_MIN_BLOCKS 4
 #endif
 
 template <int N, int TEAM, bool COUNT = false>
