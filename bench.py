@@ -644,10 +644,22 @@ def run_extras(args, S, g, local_g, inputs, W, steps, PROF, st0, st_t, flush, de
                 "chase_latency_hbm_ns": round(t_hbm, 1), "chase_latency_l2_ns": round(t_l2, 1),
                 "how": "gfsl_ubench: random aligned chunk-size gathers over 16 GiB (32 MiB for L2), the "
                        "search kernel's team shape, 4/8/16 gathers in flight per team (best kept)"}
+    # R37/R38: a traversal entered at level 0 reads no upper level; its index lookup is one
+    # 32-B sector of the sorted min keys (4 B per level-0 chunk), compulsory from DRAM for
+    # the part of that array the L2 cannot hold beside the 16-MiB directory
+    idx_bytes = 4.0 * max(0, meta["counters"][0])
+    idx_miss = 0.0 if idx_bytes <= 0 else max(0.0, 1.0 - (L2_BYTES - (18 << 20)) / idx_bytes)
+    l0_entry = upper < 0.05
     if resident:
         bound, peak, pk = "l2", (rand["R_rand_l2_GBps"] if rand else None), "measured R_rand_l2 (gfsl_ubench)"
         s_bytes = n_search * reads * Cb
         bytes_note = "every chunk gather (all levels) x C_b: the structure is L2-resident"
+    elif l0_entry:
+        bound, peak, pk = "hbm", hbm_peak, peak_kind
+        s_bytes = n_search * (reads_l0 * Cb + idx_miss * 32)
+        bytes_note = ("level-0 gathers x C_b + one 32-B sector of the sorted min keys x its L2 miss "
+                      f"fraction {idx_miss:.3f} per op (level 0 entered from the directory, R37/R38; "
+                      "SURVEY 8(d)'s level-0 bytes plus the index that replaced level 1)")
     else:
         bound, peak, pk = "hbm", hbm_peak, peak_kind
         s_bytes = n_search * (reads_l0 + upper * miss1) * Cb
