@@ -803,9 +803,9 @@ def main():
     ap.add_argument("--prefill", default="bulk", choices=["bulk", "per-op"],
                     help="prefill through the bulk path (one batch, R34; default) or the paper's "
                          "per-op Insert path in growing batches")
-    ap.add_argument("--bulk", default=None, choices=["auto", "off", "always"],
-                    help="the library's bulk path for the timed batches (R34); default auto, "
-                         "off for INS-1M / DEL-1M (they measure the paper's per-op Insert / Delete)")
+    ap.add_argument("--bulk", default="auto", choices=["auto", "off", "always"],
+                    help="the library's bulk path for the timed batches (R34; auto = the library "
+                         "default rule); off = the paper's per-op Insert / Delete only")
     ap.add_argument("--l2-window", type=int, default=0,
                     help="L2 access-policy window for the search kernel: 1 = the upper-level pool, "
                          "2 = the level-1 directory (ablations)")
@@ -821,8 +821,6 @@ def main():
     if args.p_chunk <= 0:
         ap.error("--p-chunk must be > 0 (p_chunk_q32 = 0 means p_chunk = 1)")
     args.runs = max(1, args.runs)
-    if args.bulk is None:
-        args.bulk = "off" if args.config in PERM_CONFIGS else "auto"
     if args.impl == "reference":
         world = int(os.environ.get("WORLD_SIZE", "1"))
         rank = int(os.environ.get("RANK", "0"))

@@ -122,7 +122,7 @@ typedef struct gfsl_config {
 #define GFSL_BULK_OFF 1u
 #define GFSL_BULK_ALWAYS 2u
 #define GFSL_BULK_MIN_OPS 4096u
-#define GFSL_BULK_RATIO 2u
+#define GFSL_BULK_RATIO 16u
 
 /*
  * Create an empty GFSL (one unlocked chunk per level holding -inf with a pointer
