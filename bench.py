@@ -442,6 +442,7 @@ class Setup:
             prefill_gpu(local, self.R, self.pre, self.dev, key_lo=self.lo, key_hi=self.hi,
                         per_op=self.args.prefill == "per-op")
         local.configure(bulk={"auto": 0, "off": 1, "always": 2}[a.bulk],
+                        group=1 if a.group == "on" else 0,
                         combine=1 if combine_mode(a) else 0,
                         p_chunk_q32=max(1, int(a.p_chunk * 2**32)) if a.p_chunk < 1.0 else 0,
                         l2_window=a.l2_window, no_pdl=1 if a.no_pdl else 0,
@@ -560,6 +561,7 @@ def run_gpu(args, world, rank, local_rank):
                        "prefill_path": ("one batch through the bulk path (R34)" if args.prefill == "bulk"
                                         else "per-op Inserts in growing batches + rebuild"),
                        "bulk_timed": args.bulk,
+                       "grouped_updates": args.group,
                        "l2": "flushed (256 MiB write) between timed steps",
                        "parallelism": f"range-shard x{world} (strong: global R and batch fixed)" if world > 1 else "1 GPU",
                        "exchange": (("peer windows (CUDA IPC, fused route kernels, device-side counts)"
@@ -806,6 +808,9 @@ def main():
     ap.add_argument("--bulk", default="auto", choices=["auto", "off", "always"],
                     help="the library's bulk path for the timed batches (R34; auto = the library "
                          "default rule); off = the paper's per-op Insert / Delete only")
+    ap.add_argument("--group", default="off", choices=["on", "off"],
+                    help="chunk-grouped mutations (R40, opt-in): the ops of a batch that target "
+                         "one bottom chunk are applied in one lock session; off (default) = one per op")
     ap.add_argument("--l2-window", type=int, default=0,
                     help="L2 access-policy window for the search kernel: 1 = the upper-level pool, "
                          "2 = the level-1 directory (ablations)")

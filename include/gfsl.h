@@ -118,7 +118,16 @@ typedef struct gfsl_config {
                                GFSL_BULK_OFF = never (the paper's per-op path only),
                                GFSL_BULK_ALWAYS = every batch.  Not in serial or combining
                                mode. */
+  uint32_t group;           /* chunk-grouped mutations (R40; opt-in): in concurrent
+                               batches with the lazy upper levels, the Insert/Delete ops of a
+                               batch that target the same bottom chunk are applied together in
+                               one lock session of that chunk (one read, one merged write, one
+                               split / merge decision, one release) instead of one session per
+                               op.  Same results.  0 = off (default: one lock session per op,
+                               the paper's protocol; measured faster on B200),
+                               GFSL_GROUP_ON = grouped. */
 } gfsl_config;
+#define GFSL_GROUP_ON 1u
 #define GFSL_BULK_OFF 1u
 #define GFSL_BULK_ALWAYS 2u
 #define GFSL_BULK_MIN_OPS 4096u
@@ -281,7 +290,8 @@ typedef struct gfsl_stats {
   uint64_t mutations;       /* Insert/Delete ops that changed the map */
   uint64_t kernel_launches; /* libgfsl kernels enqueued by gfsl_batch calls so far */
   uint64_t library_launches;/* library (CUB radix sort, combining mode) kernels, estimated */
-  uint64_t reserved[2];
+  uint64_t grouped;         /* Insert/Delete ops applied in a chunk group of >= 2 (R40) */
+  uint64_t reserved[1];
 } gfsl_stats;
 gfsl_status gfsl_get_stats(gfsl_t h, gfsl_stats *out);
 

@@ -64,6 +64,9 @@ struct gfsl {
   BatchCtl *ctl = nullptr;
   uint32_t *plan_path = nullptr, *mut_of = nullptr;
   uint4 *mut_rec = nullptr;
+  uint32_t *gnext = nullptr;  // R40: [list_cap] group links of the records
+  uint32_t *ghead = nullptr;  // R40: [cap_bottom] per level-0 chunk, EMPTY_GROUP between batches
+  bool group_now = false;     // R40: this batch's records are grouped by chunk
   uint64_t list_cap = 0;
   uint32_t *h_error = nullptr;  // mapped host memory, device alias in d.error
   cudaEvent_t last = nullptr;
@@ -171,7 +174,8 @@ static SearchOut search_out(gfsl *h) {
     return SearchOut{h->mut_rec, h->plan_path, h->mut_of, h->ctl->ccnt, h->region_cap, h->ck[0], h->cw[0], full,
                      0u};
   return SearchOut{h->mut_rec, h->plan_path, h->cfg.serial_updates ? h->mut_of : nullptr,
-                   h->ctl->mcnt, h->region_cap, nullptr, nullptr, full, h->spread_now ? 1u : 0u};
+                   h->ctl->mcnt, h->region_cap, nullptr, nullptr, full, h->spread_now ? 1u : 0u,
+                   h->group_now ? h->ghead : nullptr, h->group_now ? h->gnext : nullptr};
 }
 // What the update kernel reads: the same records, or the net mutations of combining mode.
 static SearchOut update_in(gfsl *h) {
@@ -446,6 +450,8 @@ static void free_all(gfsl *h) {
   cudaFree(h->plan_path);
   cudaFree(h->mut_of);
   cudaFree(h->mut_rec);
+  cudaFree(h->gnext);
+  cudaFree(h->ghead);
   for (int b = 0; b < 2; ++b) {
     cudaFree(h->st_op[b]);
     cudaFree(h->st_res[b]);
@@ -493,6 +499,8 @@ static void free_all(gfsl *h) {
     for (auto &e : ev) cudaEventDestroy(e);
   delete h;
 }
+
+static gfsl_status ensure_lists(gfsl *h, uint64_t n);
 
 extern "C" gfsl_t gfsl_create_ex(uint64_t key_range, uint64_t capacity, const gfsl_config *cfg_in) {
   gfsl_config cfg{};
@@ -583,6 +591,8 @@ extern "C" gfsl_t gfsl_create_ex(uint64_t key_range, uint64_t capacity, const gf
     h->d.dir_oc = b.order_chunk;
     h->d.dir_ok = b.order_key;
     if ((e = cudaMalloc(&h->d.freelist, (size_t)cap_b * 8)) != cudaSuccess) return fail("cudaMalloc(freelist)", e);
+    if ((e = cudaMalloc(&h->ghead, (size_t)cap_b * 4)) != cudaSuccess) return fail("cudaMalloc(ghead)", e);  // R40
+    cudaMemset(h->ghead, 0xFF, (size_t)cap_b * 4);
     if ((e = cudaMalloc(&h->d.fl, 8 * 4)) != cudaSuccess) return fail("cudaMalloc(freelist)", e);
     if ((e = cudaMalloc(&h->rc_tiles, ((size_t)cap_b / RC_TILE + 2) * 4)) != cudaSuccess) return fail("cudaMalloc(reclaim)", e);
     cudaMemset(h->d.fl, 0, 8 * 4);
@@ -617,6 +627,21 @@ extern "C" gfsl_t gfsl_create_ex(uint64_t key_range, uint64_t capacity, const gf
   if ((e = cudaDeviceSynchronize()) != cudaSuccess) return fail("init sync", e);
 
   apply_launch_shape(h);
+  // The per-batch lists for batches of up to min(capacity, 2^21) ops, and a stream-ordered
+  // pool that keeps what the bulk path frees (no OS round trip per bulk batch): neither a
+  // handle's first batches nor its bulk batches allocate inside a caller's timed region.
+  if (ensure_lists(h, std::min<uint64_t>(capacity, 1ull << 21)) != GFSL_OK) {
+    free_all(h);
+    return nullptr;
+  }
+  {
+    cudaMemPool_t mp;
+    if (cudaDeviceGetDefaultMemPool(&mp, h->device) == cudaSuccess) {
+      uint64_t thr = ~0ull;
+      cudaMemPoolSetAttribute(mp, cudaMemPoolAttrReleaseThreshold, &thr);
+    }
+    cudaGetLastError();
+  }
   return h;
 }
 
@@ -686,14 +711,17 @@ static gfsl_status ensure_lists(gfsl *h, uint64_t n) {
   cudaFree(h->plan_path);
   cudaFree(h->mut_of);
   cudaFree(h->mut_rec);
+  cudaFree(h->gnext);
   h->plan_path = nullptr;
   h->mut_of = nullptr;
   h->mut_rec = nullptr;
+  h->gnext = nullptr;
   h->list_cap = 0;
   const uint64_t cap = std::max<uint64_t>(n, 1024);
   CK(cudaMalloc(&h->plan_path, cap * 4 * PLAN_LEVELS));
   CK(cudaMalloc(&h->mut_of, cap * 4));
   CK(cudaMalloc(&h->mut_rec, cap * 16));
+  CK(cudaMalloc(&h->gnext, cap * 4));
   h->list_cap = cap;
   return GFSL_OK;
 }
@@ -864,6 +892,10 @@ static gfsl_status enqueue_batch(gfsl *h, const uint8_t *ops, const uint32_t *ke
     h->upper_stale = true;
     h->d.zparity = 0;  // R33: the marks of all lazy batches since the last rebuild
   }
+  // R40: chunk-grouped mutations in lazy concurrent batches (the update paths that take
+  // them: update_multi at N = 16 / 32)
+  h->group_now = h->d.lazy_upper && !h->cfg.combine && !h->cfg.serial_updates && h->cfg.group == GFSL_GROUP_ON &&
+                 (h->N == 16 || h->N == 32) && GFSL_UPD_SEG != 16;
   std::array<cudaEvent_t, 5> ev{};
   const bool prof = h->cfg.profile_phases != 0;
   if (prof) {
@@ -1213,6 +1245,7 @@ extern "C" gfsl_status gfsl_get_stats(gfsl_t h, gfsl_stats *out) {
   out->contains_reads_l0 = s[ST_CREADS_L0];
   out->contains_ops = s[ST_COPS];
   out->mutations = s[ST_MUTATIONS];
+  out->grouped = s[ST_GROUPED];
   out->kernel_launches = h->launches;
   out->library_launches = h->lib_launches;
   return GFSL_OK;

@@ -38,6 +38,7 @@ enum StatSlot {
   ST_CREADS_L0,   // ... of which on the bottom level
   ST_COPS,        // Contains ops counted
   ST_MUTATIONS,   // ops the update kernel applied (all batches)
+  ST_GROUPED,     // R40: records applied through a chunk group of >= 2
   ST_NSTATS
 };
 

@@ -83,7 +83,16 @@ struct SearchOut {
   uint32_t full_path;   // 1 = every Insert/Delete traverses from the top (serial mode)
   uint32_t spread;      // 1 = the update kernel takes the records in a spread order (R31:
                         // combining mode, whose net records come out of a key sort)
+  // Chunk-grouped mutations (R40), or NULL: the records of a batch that target the same
+  // level-0 chunk (path[0]) form one list -- ghead[c - cap_upper] = the last record pushed
+  // for chunk c, gnext[m] = the record pushed before m (EMPTY_GROUP ends the list).  The
+  // update kernel applies a list of >= 2 records in one lock session of its chunk; the
+  // first record pushed (gnext == EMPTY_GROUP) is the list's leader.  ghead is all
+  // EMPTY_GROUP between batches (the update kernel resets the entries it takes).
+  uint32_t *ghead;
+  uint32_t *gnext;
 };
+constexpr uint32_t EMPTY_GROUP = 0xFFFFFFFFu;
 
 // A record slot in the writing block's region (BatchCtl::mcnt).
 __device__ __forceinline__ uint32_t mut_slot(const SearchOut &so) {
@@ -384,6 +393,7 @@ search_kernel(DevState d, const BatchIn in, BatchCtl *__restrict__ ctl, SearchOu
               // R33: in lazy mode a Delete's top is 0 (level-1 copies of k stay until the
               // next rebuild, as stale separators)
               so.mut_rec[m] = make_uint4(w, k, here, (cur_op.x & DELETE_FLAG) ? (d.lazy_upper ? 0u : (uint32_t)seen_top) : cur_val);
+              if (so.ghead) so.gnext[m] = atomicExch(so.ghead + (here - d.cap_upper), m);  // R40
               my_path[0] = here;  // path[0] = the enclosing bottom chunk
               if (via_dir) {      // levels >= 2 (and 1, R37) from the directory rank (R27)
                 uint32_t q = cur_r / F;

@@ -26,6 +26,7 @@ RES_FALSE, RES_TRUE, RES_INVALID = 0, 1, 0xFF
 REBUILD_DEFAULT, REBUILD_NEVER = 0, 0xFFFFFFFF  # rebuild_every: library default period / never
 CHECK_SNAPSHOT, CHECK_CROSS = 1, 2
 BULK_AUTO, BULK_OFF, BULK_ALWAYS = 0, 1, 2
+GROUP_OFF, GROUP_ON = 0, 1
 STATUS_NAMES = ["OK", "EINVAL", "ENOMEM", "EPOOL", "ECUDA", "ECORRUPT", "ETIMEOUT"]
 XR_HANDLE_BYTES = 64
 
@@ -38,7 +39,8 @@ class gfsl_config(ctypes.Structure):
                 ("profile_phases", ctypes.c_uint32), ("l2_window", ctypes.c_uint32),
                 ("no_pdl", ctypes.c_uint32),
                 ("rebuild_every", ctypes.c_uint32), ("combine", ctypes.c_uint32),
-                ("p_chunk_q32", ctypes.c_uint32), ("bulk", ctypes.c_uint32)]
+                ("p_chunk_q32", ctypes.c_uint32), ("bulk", ctypes.c_uint32),
+                ("group", ctypes.c_uint32)]
 
 
 class gfsl_report(ctypes.Structure):
@@ -58,7 +60,8 @@ class gfsl_stats(ctypes.Structure):
                 ("lock_retries", ctypes.c_uint64), ("contains_reads", ctypes.c_uint64),
                 ("contains_reads_l0", ctypes.c_uint64), ("contains_ops", ctypes.c_uint64),
                 ("mutations", ctypes.c_uint64), ("kernel_launches", ctypes.c_uint64),
-                ("library_launches", ctypes.c_uint64), ("reserved", ctypes.c_uint64 * 2)]
+                ("library_launches", ctypes.c_uint64), ("grouped", ctypes.c_uint64),
+                ("reserved", ctypes.c_uint64 * 1)]
 
 
 class gfsl_meta(ctypes.Structure):
@@ -234,7 +237,7 @@ class GFSL:
                  contains_blocks_per_sm: int = 0, update_blocks_per_sm: int = 0,
                  count_reads: bool = False, profile_phases: bool = False,
                  rebuild_every: int = 0, combine: bool = False, p_chunk: float = 1.0,
-                 bulk: int = 0):
+                 bulk: int = 0, group: int = 0):
         import torch
         if not torch.cuda.is_available():
             raise RuntimeError("GFSL needs a CUDA device (there is no CPU fallback)")
@@ -243,7 +246,7 @@ class GFSL:
                           update_blocks_per_sm, 1 if serial_updates else 0,
                           1 if count_reads else 0, 1 if profile_phases else 0, 0, 0,
                           rebuild_every, 1 if combine else 0,
-                          0 if p_chunk >= 1.0 else max(1, int(p_chunk * 2**32)), bulk)
+                          0 if p_chunk >= 1.0 else max(1, int(p_chunk * 2**32)), bulk, group)
         if p_chunk <= 0:
             raise ValueError("p_chunk must be > 0 (p_chunk_q32 = 0 means p_chunk = 1)")
         self.key_range = int(key_range)

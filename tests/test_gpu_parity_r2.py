@@ -129,10 +129,11 @@ def test_paper_mode_c2_fullsize_every_result():
 
 # ---------------------------------------------------------------- out of contract
 
-@pytest.mark.parametrize("serial", [False, True])
-def test_out_of_contract_batches_are_linearizable(serial):
+@pytest.mark.parametrize("serial,group", [(False, 0), (True, 0), (False, 1)])
+def test_out_of_contract_batches_are_linearizable(serial, group):
+    """group = 1: the chunk-grouped path (R40), whose groups then hold duplicate keys."""
     R = 3000
-    g = GFSL(R, serial_updates=serial)
+    g = GFSL(R, serial_updates=serial, group=group)
     rng = np.random.default_rng(7 + serial)
     present = np.zeros(R, bool)
     value = np.zeros(R, np.uint32)
