@@ -61,7 +61,10 @@ struct gfsl {
   gfsl_config cfg{};
   uint64_t key_range = 0;
   DevState d{};
-  BatchCtl *ctl = nullptr;
+  BatchCtl *ctl = nullptr;        // the current batch's control block (one of ctl_buf)
+  BatchCtl *ctl_buf[2] = {nullptr, nullptr};  // alternating by batch; the update kernel of a
+  bool ctl_clean[2] = {true, true};           // batch zeroes the other one
+  int ctl_cur = 0;
   uint32_t *plan_path = nullptr, *mut_of = nullptr;
   uint4 *mut_rec = nullptr;
   uint32_t *gnext = nullptr;  // R40: [list_cap] group links of the records
@@ -320,7 +323,9 @@ static void launch_update(gfsl *h, const BatchIn &in, cudaStream_t s, cudaEvent_
   const uint64_t need = std::max<uint64_t>((uint64_t)h->sms, (in.n + per_block - 1) / per_block);
   lc.gridDim = dim3(h->cfg.serial_updates ? 1 : (unsigned)std::min<uint64_t>((uint64_t)h->update_grid, need));
   const int serial = h->cfg.serial_updates ? 1 : 0;
-  cudaLaunchKernelEx(&lc, update_kernel<N>, h->d, in, h->ctl, update_in(h), serial);
+  BatchCtl *next = h->ctl_buf[h->ctl_cur ^ 1];
+  cudaLaunchKernelEx(&lc, update_kernel<N>, h->d, in, h->ctl, update_in(h), serial, next);
+  h->ctl_clean[h->ctl_cur ^ 1] = true;
   h->launches += 1;  // update
   lc.blockDim = dim3(256);
   if (h->cfg.combine) {  // R26: keys deleted and re-inserted in this batch get their new value
@@ -446,7 +451,7 @@ static void free_all(gfsl *h) {
   cudaFree(h->d.counter);
   cudaFree(h->d.bump);
   cudaFree(h->d.stats);
-  cudaFree(h->ctl);
+  cudaFree(h->ctl_buf[0]);
   cudaFree(h->plan_path);
   cudaFree(h->mut_of);
   cudaFree(h->mut_rec);
@@ -563,15 +568,19 @@ extern "C" gfsl_t gfsl_create_ex(uint64_t key_range, uint64_t capacity, const gf
   if ((e = cudaMalloc(&h->d.counter, 32 * 4)) != cudaSuccess) return fail("cudaMalloc", e);
   if ((e = cudaMalloc(&h->d.bump, 2 * 4)) != cudaSuccess) return fail("cudaMalloc", e);
   if ((e = cudaMalloc(&h->d.stats, ST_NSTATS * 8)) != cudaSuccess) return fail("cudaMalloc", e);
-  if ((e = cudaMalloc(&h->ctl, sizeof(BatchCtl))) != cudaSuccess) return fail("cudaMalloc", e);
+  if ((e = cudaMalloc(&h->ctl_buf[0], 2 * sizeof(BatchCtl))) != cudaSuccess) return fail("cudaMalloc", e);
+  cudaMemset(h->ctl_buf[0], 0, 2 * sizeof(BatchCtl));
+  h->ctl_buf[1] = h->ctl_buf[0] + 1;
+  h->ctl = h->ctl_buf[0];
   h->d.ctl = h->ctl;
   if ((e = cudaHostAlloc(&h->h_error, 4, cudaHostAllocMapped)) != cudaSuccess) return fail("cudaHostAlloc", e);
   *h->h_error = 0;
   if ((e = cudaHostGetDevicePointer(&h->d.error, h->h_error, 0)) != cudaSuccess) return fail("cudaHostGetDevicePointer", e);
   if ((e = cudaEventCreateWithFlags(&h->last, cudaEventDisableTiming)) != cudaSuccess) return fail("cudaEventCreate", e);
-  if ((e = cudaHostAlloc(&h->h_bump, 8, cudaHostAllocDefault)) != cudaSuccess) return fail("cudaHostAlloc", e);
+  if ((e = cudaHostAlloc(&h->h_bump, 8, cudaHostAllocMapped)) != cudaSuccess) return fail("cudaHostAlloc", e);
   h->h_bump[0] = 1;
   h->h_bump[1] = N - 1;
+  if ((e = cudaHostGetDevicePointer(&h->d.bump_host, h->h_bump, 0)) != cudaSuccess) return fail("cudaHostGetDevicePointer", e);
   setup_l2_window(h);
   {
     RebuildBufs &b = h->rb;
@@ -902,7 +911,14 @@ static gfsl_status enqueue_batch(gfsl *h, const uint8_t *ops, const uint32_t *ke
     for (auto &e : ev) CK(cudaEventCreate(&e));
     CK(cudaEventRecord(ev[0], s));
   }
-  CK(cudaMemsetAsync(h->ctl, 0, offsetof(BatchCtl, uq) + (size_t)std::min(h->update_grid, BatchCtl::UQ_MAX) * 32, s));
+  {
+    const int cur = h->ctl_cur;
+    h->ctl = h->ctl_buf[cur];
+    h->d.ctl = h->ctl;
+    // normally zeroed by the previous batch's update kernel; after a failed batch, here
+    if (!h->ctl_clean[cur]) CK(cudaMemsetAsync(h->ctl, 0, sizeof(BatchCtl), s));
+    h->ctl_clean[cur] = false;
+  }
   if (prof) CK(cudaEventRecord(ev[1], s));
   BatchIn in{ops, keys, vals, res, (uint32_t)n, h->key_range, n_dev, nullptr, nullptr};
   {
@@ -940,8 +956,8 @@ static gfsl_status enqueue_batch(gfsl *h, const uint8_t *ops, const uint32_t *ke
     CK(cudaEventRecord(ev[4], s));
     h->phase_ev.push_back(ev);
   }
-  CK(cudaMemcpyAsync(h->h_bump, h->d.bump, 8, cudaMemcpyDeviceToHost, s));
   CK(cudaEventRecord(h->last, s));
+  h->ctl_cur ^= 1;
   h->batches++;
   h->ops += h->n_policy;
   h->live_ub = std::min(h->capacity, h->live_ub + n);
@@ -967,7 +983,9 @@ static gfsl_status enqueue_bulk(gfsl *h, const uint8_t *ops, const uint32_t *key
                                 uint8_t *res, uint64_t n, cudaStream_t s) {
   CK(cudaStreamWaitEvent(s, h->last, 0));
   CK(cudaEventSynchronize(h->last));  // the bump counters after the previous batch
-  const uint32_t used_b = std::min(h->h_bump[0], h->d.cap_bottom);
+  uint32_t hb[2];
+  CK(cudaMemcpy(hb, h->d.bump, 8, cudaMemcpyDeviceToHost));
+  const uint32_t used_b = std::min(hb[0], h->d.cap_bottom);
   const uint64_t M = n + (uint64_t)used_b * (N - 2);
   const int bits = sort_bits_for(h->key_range);
   uint32_t *sk0, *sk1, *hd, *gs, *fi, *fd, *ck;

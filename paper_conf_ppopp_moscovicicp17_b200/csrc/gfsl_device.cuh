@@ -98,6 +98,8 @@ struct DevState {
   const uint32_t *dir_oc;
   const uint32_t *dir_ok;  // R38: the sorted min keys of the last rebuild (order_key)
   uint32_t l0_entry;
+  uint32_t *bump_host;  // mapped pinned host copy of bump[0..1], written by the search kernel
+                        // at its start (the counters after the previous batch; host heuristics)
 };
 
 // isKeyRaised's draw (R28): a counter-based hash of (raised key, level of the split), the

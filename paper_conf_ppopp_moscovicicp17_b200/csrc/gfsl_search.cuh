@@ -148,7 +148,13 @@ search_kernel(DevState d, const BatchIn in, BatchCtl *__restrict__ ctl, SearchOu
       s_n1 = d.dir_hdr[6];
       // R27: Contains enter at level 1 through the directory when there are levels above
       s_dir_shift = (h >= 2 && d.dir_hdr[1]) ? d.dir_hdr[0] : 32u;
-      if (blockIdx.x == 0) ctl->snap_height = h;
+      if (blockIdx.x == 0) {
+        ctl->snap_height = h;
+        if (d.bump_host) {  // (zero-copy: no D2H copy node per batch)
+          d.bump_host[0] = d.bump[0];
+          d.bump_host[1] = d.bump[1];
+        }
+      }
     }
     if (lane < PLAN_LEVELS) s_dir_base[lane] = d.dir_hdr[32 + lane];
   }

@@ -1,4 +1,4 @@
-"""Per-warp timeline of the dual-op update kernel (needs a library built with
+"""Per-warp timeline of the update kernel (update_multi / update_dual) (needs a library built with
 -DGFSL_DEBUG_TIMING in place of libgfsl.so).  python tools/upd_timeline.py [config]"""
 import ctypes, os, sys
 sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
@@ -20,6 +20,7 @@ buf = (ctypes.c_ulonglong * n)()
 buf0 = (ctypes.c_ulonglong * n)()
 for b in range(4):
     if b == 3:
+        torch.empty(256 << 20, dtype=torch.uint8, device=dev).zero_()  # bench.py's L2 flush
         torch.cuda.synchronize()
         lib.gfsl_debug_times(ctypes.c_void_p(g.h), buf0, ctypes.c_uint64(n))
     g.batch(*make_inputs(w, b, dev)[:3])
@@ -37,6 +38,12 @@ ser = a[:, 7]
 print(f"{cfg}: warps={len(a)} iterations={it.sum():.0f} kernel span={en.max():.1f} us")
 print("outcomes done/defer/cont/full:", oc.astype(int).tolist())
 print("start pct 0/50/90/100:", np.percentile(st, [0, 50, 90, 100]).round(1))
+fo = a[:, 8]
+if (fo > 0).any():
+    print("first-op pct 0/50/90/100:", np.percentile((fo[fo > 0] - t0) / 1e3, [0, 50, 90, 100]).round(1),
+          f"(warps with an op: {(fo > 0).sum()})")
+    busy = en[fo > 0]
+    print("end of warps with ops pct 50/90/99/100:", np.percentile(busy, [50, 90, 99, 100]).round(1))
 print("end   pct 0/50/90/99/100:", np.percentile(en, [0, 50, 90, 99, 100]).round(1))
 print("iterations/warp pct 0/50/100:", np.percentile(it, [0, 50, 100]))
 dur = (en - st) * 1e3 * 1.965
