@@ -70,14 +70,17 @@ def test_paper_mode_concurrent_churn_small_range(N):
     R = 600
     g = GFSL(R, chunk_entries=N, rebuild_every=REBUILD_NEVER)   # p_chunk = 1 (default)
     o = OracleMap(R)
+    top = 0
     for op, key, val in batches(R, 300, 40, (50, 50, 0), SEED_BASE + 201 + N):
         run_batch(g, o, op, key, val)
-        _, d = check_all(g, o)
+        rep, d = check_all(g, o)
+        top = max(top, rep.height)
     assert d.cross_checked                    # no rebuild ran: V6 / V11 were checked
     st = g.stats()
     assert st["splits"] > 0 and st["merges"] > 0
-    rep, _, _ = g.validate()
-    assert rep.height >= 1                    # keys were raised (Alg 4.5 l.15-22)
+    # keys were raised (Alg 4.5 l.15-22) at some point; under 50/50 churn the concurrent
+    # top-down Deletes (Alg 4.11 l.13-20) may strip every raised key again by the end
+    assert top >= 1
 
 
 @pytest.mark.parametrize("N", [16, 32])
