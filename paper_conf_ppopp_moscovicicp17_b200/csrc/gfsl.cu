@@ -53,6 +53,14 @@ void gfsl_internal_set_error(const std::string &s) { set_last_error(s); }  // gf
     }                                                                                 \
   } while (0)
 
+// Batches of up to this many ops take the small-batch kernel (GFSL_SMALL_BATCH in the
+// environment at gfsl_create overrides; 0 = never).
+// Measured: no gain at C1 (the time is the lock-session chain, not the kernel
+// boundary), +3% at C2-5050 with a 128K threshold -- off by default.
+#ifndef GFSL_SMALL_BATCH_DEFAULT
+#define GFSL_SMALL_BATCH_DEFAULT 0
+#endif
+
 struct gfsl {
   int device = 0;
   int sms = 148;
@@ -65,6 +73,8 @@ struct gfsl {
   BatchCtl *ctl_buf[2] = {nullptr, nullptr};  // alternating by batch; the update kernel of a
   bool ctl_clean[2] = {true, true};           // batch zeroes the other one
   int ctl_cur = 0;
+  uint32_t small_max = 0;  // batches of <= this many ops take the small-batch kernel (0: never)
+  uint32_t small_grid = 0; // its cooperative grid (blocks that are co-resident)
   uint32_t *plan_path = nullptr, *mut_of = nullptr;
   uint4 *mut_rec = nullptr;
   uint32_t *gnext = nullptr;  // R40: [list_cap] group links of the records
@@ -308,8 +318,37 @@ static void launch_rebuild(gfsl *h, cudaStream_t s) {
   cudaLaunchKernelEx(&lc, reclaim_write_kernel<N>, h->d, b, (const uint32_t *)h->rc_tiles);
 }
 
+// The small-batch kernel (search, grid barrier, update in one cooperative launch) for the
+// default team shapes; false if this (N, team) has none.
+template <int N, int TEAM>
+static void launch_small_t(gfsl *h, const BatchIn &in, cudaStream_t s) {
+  cudaLaunchConfig_t lc{};
+  cudaLaunchAttribute attr[1];
+  attr[0].id = cudaLaunchAttributeCooperative;
+  attr[0].val.cooperative = 1;
+  lc.attrs = attr;
+  lc.numAttrs = 1;
+  lc.stream = s;
+  lc.blockDim = dim3(256);
+  lc.gridDim = dim3(h->small_grid);
+  cudaLaunchKernelEx(&lc, small_batch_kernel<N, TEAM>, h->d, in, h->ctl, search_out(h), h->ctl_buf[h->ctl_cur ^ 1]);
+  h->launches += 1;
+}
+static bool launch_small(gfsl *h, const BatchIn &in, cudaStream_t s) {
+  if (h->N == 16 && h->team == 2) launch_small_t<16, 2>(h, in, s);
+  else if (h->N == 32 && h->team == 4) launch_small_t<32, 4>(h, in, s);
+  else return false;
+  return true;
+}
+template <int N, int TEAM>
+static int occ_small() {
+  int b = 0;
+  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, small_batch_kernel<N, TEAM>, 256, 0);
+  return b;
+}
+
 template <int N>
-static void launch_update(gfsl *h, const BatchIn &in, cudaStream_t s, cudaEvent_t after_update) {
+static void launch_update(gfsl *h, const BatchIn &in, cudaStream_t s, cudaEvent_t after_update, bool fused = false) {
   cudaLaunchConfig_t lc{};
   cudaLaunchAttribute attr[1];
   set_pdl(h, attr[0]);
@@ -324,9 +363,15 @@ static void launch_update(gfsl *h, const BatchIn &in, cudaStream_t s, cudaEvent_
   lc.gridDim = dim3(h->cfg.serial_updates ? 1 : (unsigned)std::min<uint64_t>((uint64_t)h->update_grid, need));
   const int serial = h->cfg.serial_updates ? 1 : 0;
   BatchCtl *next = h->ctl_buf[h->ctl_cur ^ 1];
-  cudaLaunchKernelEx(&lc, update_kernel<N>, h->d, in, h->ctl, update_in(h), serial, next);
+  if (!fused) {  // (the small-batch kernel ran the update phase already)
+    // eight mutations per warp for large batches, four below GFSL_UPD_SEG_SMALL_MAX ops
+    if (N == 16 && in.n < GFSL_UPD_SEG_SMALL_MAX)
+      cudaLaunchKernelEx(&lc, update_kernel<N, GFSL_UPD_SEG_SMALL>, h->d, in, h->ctl, update_in(h), serial, next);
+    else
+      cudaLaunchKernelEx(&lc, update_kernel<N>, h->d, in, h->ctl, update_in(h), serial, next);
+    h->launches += 1;  // update
+  }
   h->ctl_clean[h->ctl_cur ^ 1] = true;
-  h->launches += 1;  // update
   lc.blockDim = dim3(256);
   if (h->cfg.combine) {  // R26: keys deleted and re-inserted in this batch get their new value
     lc.gridDim = dim3(h->sms * 2);
@@ -436,6 +481,12 @@ static void setup_l2_window(gfsl *h) {
 }
 
 static void apply_launch_shape(gfsl *h) {
+  {
+    int bs = 0;
+    if (h->N == 16 && h->team == 2) bs = occ_small<16, 2>();
+    else if (h->N == 32 && h->team == 4) bs = occ_small<32, 4>();
+    h->small_grid = (uint32_t)(h->sms * std::min(bs, 4));
+  }
   int bc = contains_occupancy(h->N, h->team);
   if (h->cfg.contains_blocks_per_sm) bc = std::min<int>(bc, h->cfg.contains_blocks_per_sm);
   int bu = update_occupancy(h->N);
@@ -537,6 +588,8 @@ extern "C" gfsl_t gfsl_create_ex(uint64_t key_range, uint64_t capacity, const gf
     h->l0_entry = (e && *e && *e != '0') ? 0u : 1u;
     const char *ko = getenv("GFSL_KEY_ORDER");
     h->key_order = ko && *ko ? atoi(ko) : -1;
+    const char *sb = getenv("GFSL_SMALL_BATCH");  // ops; 0 = never (default GFSL_SMALL_BATCH_DEFAULT)
+    h->small_max = sb && *sb ? (uint32_t)atoi(sb) : (uint32_t)GFSL_SMALL_BATCH_DEFAULT;
   }
   auto fail = [&](const char *what, cudaError_t e) -> gfsl_t {
     set_last_error(std::string(what) + ": " + cudaGetErrorString(e));
@@ -904,7 +957,7 @@ static gfsl_status enqueue_batch(gfsl *h, const uint8_t *ops, const uint32_t *ke
   // R40: chunk-grouped mutations in lazy concurrent batches (the update paths that take
   // them: update_multi at N = 16 / 32)
   h->group_now = h->d.lazy_upper && !h->cfg.combine && !h->cfg.serial_updates && h->cfg.group == GFSL_GROUP_ON &&
-                 (h->N == 16 || h->N == 32) && GFSL_UPD_SEG != 16;
+                 (h->N == 16 || h->N == 32) && GFSL_UPD_SEG != 16 && GFSL_UPD_SEG_SMALL != 16;
   std::array<cudaEvent_t, 5> ev{};
   const bool prof = h->cfg.profile_phases != 0;
   if (prof) {
@@ -930,7 +983,10 @@ static gfsl_status enqueue_batch(gfsl *h, const uint8_t *ops, const uint32_t *ke
       if (ks != GFSL_OK) return ks;
     }
   }
-  bool ok = dispatch_contains(h, in, s);
+  // small batches: search + barrier + update in one cooperative kernel
+  const bool fused = !h->cfg.serial_updates && !h->cfg.combine && !h->cfg.count_reads && !h->ko_now && !n_dev &&
+                     h->small_grid && n <= h->small_max && launch_small(h, in, s);
+  bool ok = fused || dispatch_contains(h, in, s);
   if (!ok) {
     set_last_error("no contains kernel for this (N, team)");
     return GFSL_EINVAL;
@@ -941,10 +997,10 @@ static gfsl_status enqueue_batch(gfsl *h, const uint8_t *ops, const uint32_t *ke
   }
   if (prof) CK(cudaEventRecord(ev[2], s));
   switch (h->N) {
-    case 32: launch_update<32>(h, in, s, prof ? ev[3] : nullptr); break;
-    case 16: launch_update<16>(h, in, s, prof ? ev[3] : nullptr); break;
-    case 12: launch_update<12>(h, in, s, prof ? ev[3] : nullptr); break;
-    case 6: launch_update<6>(h, in, s, prof ? ev[3] : nullptr); break;
+    case 32: launch_update<32>(h, in, s, prof ? ev[3] : nullptr, fused); break;
+    case 16: launch_update<16>(h, in, s, prof ? ev[3] : nullptr, fused); break;
+    case 12: launch_update<12>(h, in, s, prof ? ev[3] : nullptr, fused); break;
+    case 6: launch_update<6>(h, in, s, prof ? ev[3] : nullptr, fused); break;
   }
   cudaError_t e = cudaGetLastError();
   if (e != cudaSuccess) {

@@ -114,9 +114,11 @@ constexpr uint32_t CW_NOTMUT = 0x20000000u;  // Contains or invalid: not part of
 #define GFSL_SEARCH_MIN_BLOCKS 4
 #endif
 
+// The search phase of a batch: the body of search_kernel, and the first half of the
+// small-batch kernel (gfsl_update.cuh).
 template <int N, int TEAM, bool COUNT = false>
-__global__ void __launch_bounds__(256, GFSL_SEARCH_MIN_BLOCKS)
-search_kernel(DevState d, const BatchIn in, BatchCtl *__restrict__ ctl, SearchOut so) {
+__device__ __forceinline__ void search_body(const DevState &d, const BatchIn &in, BatchCtl *__restrict__ ctl,
+                                            const SearchOut &so) {
   constexpr int EPL = N / TEAM;
   static_assert(EPL * TEAM == N, "TEAM must divide N");
   constexpr int TPW = 32 / TEAM;                    // teams per warp
@@ -311,8 +313,9 @@ search_kernel(DevState d, const BatchIn in, BatchCtl *__restrict__ ctl, SearchOu
     ChunkSlice<EPL> s;
     ld_slice_nc<EPL>(d.pool + (size_t)cur * N + t * EPL, s, level == 0 ? pol_l0 : pol_up);  // idle teams re-read `cur`
     if (pf_dir) {
-      if ((nxt.op == 0 || (dir_upd && nxt.op <= 2)) && (uint64_t)nxt.key < in.key_range)
+      if ((nxt.op == 0 || (dir_upd && nxt.op <= 2)) && (uint64_t)nxt.key < in.key_range) {
         nxt_dir = ld_dir(nxt.key + 1u);
+      }
       pf_dir = false;
     }
     if (COUNT && active) {
@@ -448,6 +451,12 @@ search_kernel(DevState d, const BatchIn in, BatchCtl *__restrict__ ctl, SearchOu
     stat_add(d, ST_CREADS_L0, reads_l0);
     stat_add(d, ST_COPS, nops);
   }
+}
+
+template <int N, int TEAM, bool COUNT = false>
+__global__ void __launch_bounds__(256, GFSL_SEARCH_MIN_BLOCKS)
+search_kernel(const __grid_constant__ DevState d, const BatchIn in, BatchCtl *__restrict__ ctl, SearchOut so) {
+  search_body<N, TEAM, COUNT>(d, in, ctl, so);
 }
 
 // The update kernel's view of the region-numbered records: slot s in [0, total) ->

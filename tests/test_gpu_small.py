@@ -1,0 +1,88 @@
+"""GPU parity of the small-batch kernel: batches of up to GFSL_SMALL_BATCH ops (environment
+at gfsl_create; 0 = never, the default) run the search phase, a grid-wide barrier (the S1
+phase boundary, R1) and the update phase in ONE cooperative launch instead of a
+search and an update kernel.
+Every result vs Oracle-A and the same batches through the two-kernel path, the invariants
+after every batch, and the launch counts that show which path ran."""
+import numpy as np
+import pytest
+import torch
+
+from oracle.oracle_a import OracleMap
+from paper_conf_ppopp_moscovicicp17_b200.gfsl import GFSL
+from tests.test_gpu_parity_r2 import check_all, to_dev
+
+pytestmark = pytest.mark.gpu
+
+
+def _handles(R, N, monkeypatch):
+    monkeypatch.setenv("GFSL_SMALL_BATCH", "0")
+    two = GFSL(R, chunk_entries=N)
+    monkeypatch.setenv("GFSL_SMALL_BATCH", "16384")
+    one = GFSL(R, chunk_entries=N)
+    return one, two
+
+
+@pytest.mark.parametrize("N", [16, 32])
+def test_small_batch_kernel_matches_oracle_and_two_kernel_path(N, monkeypatch):
+    R = 10_000
+    one, two = _handles(R, N, monkeypatch)
+    o = OracleMap(R)
+    rng = np.random.default_rng(800 + N)
+    fused = 0
+    for b, n in enumerate([0, 1, 7, 100, 3000, 6250, 6250, 16384, 16385, 40000, 6250, 2]):
+        # <= 1 mutation per key (R1): mutating keys drawn without replacement
+        m = min(n // 5, R // 2)
+        mk = rng.choice(R, m, replace=False).astype(np.uint32)
+        ck = rng.integers(0, R, n - m).astype(np.uint32)
+        key = np.concatenate([mk, ck])
+        op = np.concatenate([rng.choice([1, 2], m), np.zeros(n - m, np.int64)]).astype(np.uint8)
+        perm = rng.permutation(n)
+        key, op = key[perm], op[perm]
+        val = rng.integers(0, 2**32, n, dtype=np.uint64).astype(np.uint32)
+        l0, l1 = one.stats()["kernel_launches"], two.stats()["kernel_launches"]
+        r1 = one.batch(*to_dev(op, key, val)).cpu().numpy()
+        r2 = two.batch(*to_dev(op, key, val)).cpu().numpy()
+        e = o.batch(op, key, val)
+        assert np.array_equal(r1, e), f"batch {b} (n={n}): fused path differs from the oracle"
+        assert np.array_equal(r2, e), f"batch {b} (n={n}): two-kernel path differs from the oracle"
+        d1 = one.stats()["kernel_launches"] - l0
+        d2 = two.stats()["kernel_launches"] - l1
+        if n == 0:
+            assert d1 == d2 == 0                                        # nothing enqueued
+        elif n <= 16384:
+            assert d1 == d2 - 1, f"batch {b}: {d1} vs {d2} launches"   # search + update -> one kernel
+            fused += 1
+        else:
+            assert d1 == d2
+        check_all(one, o)
+        rep, ks, vs = two.validate()
+        ok, ov = o.export()
+        assert rep.violations == 0 and np.array_equal(ks, ok) and np.array_equal(vs, ov)
+    assert fused >= 8
+    one.close()
+    two.close()
+
+
+def test_small_batch_kernel_churn_with_rebuilds(monkeypatch):
+    """C1's shape (R = 10K, 6250-op batches of [10,10,80]) for 40 batches: splits, merges,
+    the rebuild policy (R29) between fused batches."""
+    from paper_conf_ppopp_moscovicicp17_b200.workload import SEED_BASE, Workload
+    R = 10_000
+    monkeypatch.setenv("GFSL_SMALL_BATCH", "16384")
+    g = GFSL(R)
+    o = OracleMap(R)
+    k0 = np.random.default_rng(3).permutation(R)[:R // 2].astype(np.uint32)
+    o.batch(np.ones(k0.size, np.uint8), k0, k0 + 1)
+    g.batch(*to_dev(np.ones(k0.size, np.uint8), k0, k0 + 1))
+    w = Workload(R, 6250, mix=(10, 10, 80), seed=SEED_BASE + 9)
+    for b in range(40):
+        op, key, val, _ = w.make_batch(b)
+        op, key, val = op.numpy(), key.numpy().astype(np.uint32), val.numpy().astype(np.uint32)
+        r = g.batch(*to_dev(op, key, val)).cpu().numpy()
+        assert np.array_equal(r, o.batch(op, key, val)), f"batch {b}"
+        if b % 5 == 4:
+            check_all(g, o, cross=False)
+    st = g.stats()
+    assert st["splits"] > 0
+    g.close()
