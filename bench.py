@@ -685,6 +685,17 @@ def run_extras(args, S, g, local_g, inputs, W, steps, PROF, st0, st_t, flush, de
             r["traffic_GBps"] = round(t / (ms / 1e3) / 1e9, 1)
         if rand and bound == "hbm":
             r["frac_of_random_access_peak"] = round(ach / rand["R_rand_hbm_GBps"], 4)
+            if kernel == "search":
+                # what R_rand bounds: fully random C_b-byte gathers, i.e. the level-0 chunk
+                # reads of uniform keys; the index reads (sorted min keys, directory) are
+                # 32-B sectors with locality (row-buffer hits), so the kernel's whole DRAM
+                # traffic (ncu) can exceed R_rand while its chunk gathers stay below it
+                g_rate = n_search * reads_l0 / (ms / 1e3)
+                r_rate = rand["R_rand_hbm_GBps"] * 1e9 / Cb
+                r["random_gathers"] = {
+                    "level0_gathers_per_s": round(g_rate / 1e9, 3), "ceiling_gathers_per_s": round(r_rate / 1e9, 3),
+                    "unit": "G gathers/s", "frac": round(g_rate / r_rate, 4),
+                    "note": "level-0 chunk gathers of the search kernel vs gfsl_ubench's random C_b-byte gather rate"}
         return r
 
     roof_c = roof(s_bytes, c_ms, "search", bytes_note)

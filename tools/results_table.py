@@ -29,14 +29,20 @@ def row(d):
     w = c["workload"]
     p = d.get("phase_ms_per_step", {})
     srch = p.get("search", 0.0)
-    r = (d.get("roofline_kernels") or {}).get("search") or d.get("roofline", {})
+    r = (d.get("roofline_kernels") or {}).get("search") or d.get("roofline") or {}
     e2e = d.get("e2e") or {}
     cpu = d.get("cpu_baseline") or {}
-    v = f"**{d['value']:.0f}**" if w in ("C2", "C5") else f"{d['value']:.0f}"
+    runs = d.get("runs") or {}
+    ci = runs.get("ci95_half_width")
+    v = f"{d['value']:.0f}" + (f" ± {ci:.0f}" if ci is not None else "")
+    v = f"**{v}**" if w in ("C2", "C5") else v
+    roof = f"{r.get('bound', '-')} {r.get('frac', 0):.2f}" if r else "-"
+    rg = (r.get("random_gathers") or {}).get("frac")
+    if rg is not None:
+        roof += f" (gathers {rg:.2f} of R_rand)"
     return (f"| {DESC.get(w, w)} | {c.get('chunk_entries', '')} | {v} | {e2e.get('value', 0):.0f} | "
             f"{srch:.3f} / {p.get('update', 0):.3f} / {p.get('upkeep_rebuild', 0):.3f} | "
-            f"{d.get('chunk_reads_per_contains', 0):.1f} ({d.get('chunk_reads_l0_per_contains', 0):.1f}) | "
-            f"{r.get('frac', 0):.2f} / {r.get('frac_of_random_access_peak', 0):.2f} | {cpu.get('value', 0):.1f} |")
+            f"{d.get('chunk_reads_per_contains', 0):.2f} | {roof} | {cpu.get('value', 0):.1f} |")
 
 
 def main():
