@@ -219,7 +219,8 @@ static void fill_window(gfsl *h, cudaLaunchAttribute &a) {
   a.id = cudaLaunchAttributeAccessPolicyWindow;
   // l2_window = 2: the level-1 directory only (R27; 8 B x its buckets); else the upper pool
   const bool dir = h->cfg.l2_window == 2;
-  const size_t used = dir ? (size_t)h->d.dir_cap : (size_t)std::min(h->h_bump[1] + 64u, h->d.cap_upper) * h->N * 8;
+  const size_t used = dir ? (size_t)h->d.dir_cap * 32 / 28
+                          : (size_t)std::min(h->h_bump[1] + 64u, h->d.cap_upper) * h->N * 8;
   const size_t bytes = std::min(used, h->window_max);
   a.val.accessPolicyWindow.base_ptr = dir ? (void *)h->d.dir : (void *)h->d.pool;
   a.val.accessPolicyWindow.num_bytes = bytes;
@@ -665,8 +666,9 @@ extern "C" gfsl_t gfsl_create_ex(uint64_t key_range, uint64_t capacity, const gf
     h->d.dir_cap = dcap;
 #ifdef GFSL_DIR_U32
     if ((e = cudaMalloc(&h->d.dir, (size_t)dcap * 4)) != cudaSuccess) return fail("cudaMalloc(dir)", e);
-#else
-    if ((e = cudaMalloc(&h->d.dir, (size_t)dcap)) != cudaSuccess) return fail("cudaMalloc(dir)", e);
+#else  // room for either layout (R27b split, R27c sector; the rebuild chooses)
+    if ((e = cudaMalloc(&h->d.dir, std::max<size_t>(dcap, ((size_t)dcap / DIR_SEC_BUCKETS + 2) * 32))) != cudaSuccess)
+      return fail("cudaMalloc(dir)", e);
 #endif
     if ((e = cudaMalloc(&h->d.dir_base, (size_t)dcap / 32 * 4)) != cudaSuccess) return fail("cudaMalloc(dir)", e);
     if ((e = cudaMalloc(&h->d.dir_hdr, 64 * 4)) != cudaSuccess) return fail("cudaMalloc(dir)", e);

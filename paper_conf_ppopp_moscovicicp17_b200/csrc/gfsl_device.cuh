@@ -44,6 +44,18 @@ enum StatSlot {
 
 struct BatchCtl;
 
+// R27c: directory layout, chosen by each rebuild (dir_hdr[8]).  Sector layout: groups of
+// DIR_SEC_BUCKETS = 28 buckets in one 32-B sector -- a 32-bit base (the group's first
+// rank) then one byte per bucket -- so the two reads of a lookup hit one sector (one L2
+// request); split layout (R27b): a byte array and a base array (32 buckets per base, two
+// requests).  The sector layout is taken up to GFSL_DIR_SECTOR_MAX buckets (default: any
+// size; measured C2 +1.5%, C3 +5%, C4-16 +14%, C5 -4% / +4% on two boxes);
+// GFSL_DIR_SECTOR_MAX=0 restores R27b.
+#ifndef GFSL_DIR_SECTOR_MAX
+#define GFSL_DIR_SECTOR_MAX 0xFFFFFFFFu
+#endif
+constexpr uint32_t DIR_SEC_BUCKETS = 28;
+
 // Device view of one handle.
 struct DevState {
   uint64_t *pool;        // (cap_upper + cap_bottom) * N entries

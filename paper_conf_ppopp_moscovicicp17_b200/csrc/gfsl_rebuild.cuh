@@ -299,14 +299,22 @@ __global__ void __launch_bounds__(256) rebuild_pack_kernel(const __grid_constant
     int shift = 0;
     while (((uint64_t)d.key_max >> shift) + 1 > target) ++shift;
     const uint32_t buckets = (uint32_t)((uint64_t)d.key_max >> shift) + 1;
+    const bool sector = buckets <= GFSL_DIR_SECTOR_MAX;  // R27c
     for (uint32_t q = blockIdx.x * blockDim.x + threadIdx.x; q < buckets; q += gridDim.x * blockDim.x) {
       const uint32_t r = rb_rank_le(b, q << shift);
 #ifdef GFSL_DIR_U32
       ((uint32_t *)d.dir)[q] = r;
 #else
-      const uint32_t base = (q & 31u) ? rb_rank_le(b, (q & ~31u) << shift) : r;
-      d.dir[q] = (uint8_t)min(255u, r - base);
-      if ((q & 31u) == 0) d.dir_base[q >> 5] = base;
+      if (sector) {
+        const uint32_t g = q / DIR_SEC_BUCKETS, j = q - g * DIR_SEC_BUCKETS;
+        const uint32_t base = j ? rb_rank_le(b, (g * DIR_SEC_BUCKETS) << shift) : r;
+        d.dir[(size_t)g * 32 + 4 + j] = (uint8_t)min(255u, r - base);
+        if (j == 0) *(uint32_t *)(d.dir + (size_t)g * 32) = base;
+      } else {
+        const uint32_t base = (q & 31u) ? rb_rank_le(b, (q & ~31u) << shift) : r;
+        d.dir[q] = (uint8_t)min(255u, r - base);
+        if ((q & 31u) == 0) d.dir_base[q >> 5] = base;
+      }
 #endif
     }
     if (blockIdx.x == 0 && threadIdx.x < 32) {
@@ -323,6 +331,7 @@ __global__ void __launch_bounds__(256) rebuild_pack_kernel(const __grid_constant
         d.dir_hdr[5] = b.n1[4];  // R38: level 0 in rank order (chunk cap_upper + rank)
         d.dir_hdr[6] = n1;       // R38: min keys in order_key
         d.dir_hdr[7] = d.cap_upper;
+        d.dir_hdr[8] = sector ? 1u : 0u;  // R27c: directory layout
       }
     }
   }

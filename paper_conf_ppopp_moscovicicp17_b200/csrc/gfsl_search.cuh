@@ -105,6 +105,12 @@ constexpr uint32_t CW_P0 = 0x80000000u;      // k was present in the snapshot
 constexpr uint32_t CW_DEL = 0x40000000u;     // Delete (else Insert)
 constexpr uint32_t CW_NOTMUT = 0x20000000u;  // Contains or invalid: not part of any chain
 
+// Keys of the sorted-min-key window a coarse directory (C5) reads: 8 (two 16-B reads; 12 and 16
+// measured slower at C5: every read is a request, and the kernel is request-bound)
+#ifndef GFSL_OK_WIN
+#define GFSL_OK_WIN 8
+#endif
+
 #ifndef GFSL_SEARCH_MIN_BLOCKS
 // 4 blocks per SM (<= 64 registers, no spill): with level 0 entered directly (R37/R38) a
 // traversal is ~1-2 dependent gathers, latency-bound (ncu at C5: 0.45 eligible warps per
@@ -128,7 +134,7 @@ __device__ __forceinline__ void search_body(const DevState &d, const BatchIn &in
   constexpr int LOCK_LANE = LOCK_E / EPL, LOCK_J = LOCK_E % EPL;
   constexpr uint32_t FULL = 0xFFFFFFFFu;
 
-  __shared__ uint32_t s_start, s_height, s_dir_shift, s_head0, s_l0_ok, s_korder, s_n1;
+  __shared__ uint32_t s_start, s_height, s_dir_shift, s_head0, s_l0_ok, s_korder, s_n1, s_dsec;
   __shared__ uint32_t s_dir_base[PLAN_LEVELS];  // base of each rebuilt level (R27)
   // the path of the team's current op (written by its lane 0 only), copied out compactly
   // at the end if the op mutates (about 1 op in 10)
@@ -148,6 +154,7 @@ __device__ __forceinline__ void search_body(const DevState &d, const BatchIn &in
       s_l0_ok = d.dir_hdr[4];
       s_korder = d.dir_hdr[5];
       s_n1 = d.dir_hdr[6];
+      s_dsec = d.dir_hdr[8];
       // R27: Contains enter at level 1 through the directory when there are levels above
       s_dir_shift = (h >= 2 && d.dir_hdr[1]) ? d.dir_hdr[0] : 32u;
       if (blockIdx.x == 0) {
@@ -181,6 +188,7 @@ __device__ __forceinline__ void search_body(const DevState &d, const BatchIn &in
   // R37: enter at level 0, in the chunk of level-1 entry r's down pointer (the rebuild's
   // rank order); the levels above are skipped (their path entries come from r, as R27's)
   const bool korder = s_korder != 0;   // R38: level 0 in rank order
+  const bool dsec = s_dsec != 0;       // R27c: sector layout of the directory
   const uint32_t n1 = s_n1;
   const bool l0_entry = d.l0_entry != 0 && (s_l0_ok != 0 || korder);
   const bool fine_dir = s_l0_ok != 0;  // >= 1 directory bucket per level-1 key
@@ -257,6 +265,13 @@ __device__ __forceinline__ void search_body(const DevState &d, const BatchIn &in
     return make_uint2(__ldg((const uint32_t *)d.dir + q), 0u);
 #else
     uint32_t base, byte;
+    if (dsec) {  // R27c: base and byte in one 32-B sector
+      const uint32_t g = q / DIR_SEC_BUCKETS;
+      const uint8_t *sec = d.dir + (size_t)g * 32;
+      asm volatile("ld.global.nc.L2::cache_hint.u32 %0, [%1], %2;" : "=r"(base) : "l"(sec), "l"(pol_up));
+      asm volatile("ld.global.nc.L2::cache_hint.u8 %0, [%1], %2;" : "=r"(byte) : "l"(sec + 4 + (q - g * DIR_SEC_BUCKETS)), "l"(pol_up));
+      return make_uint2(base, byte);
+    }
     asm volatile("ld.global.nc.L2::cache_hint.u32 %0, [%1], %2;" : "=r"(base) : "l"(d.dir_base + (q >> 5)), "l"(pol_up));
     asm volatile("ld.global.nc.L2::cache_hint.u8 %0, [%1], %2;" : "=r"(byte) : "l"(d.dir + q), "l"(pol_up));
     return make_uint2(base, byte);
@@ -279,17 +294,18 @@ __device__ __forceinline__ void search_body(const DevState &d, const BatchIn &in
         for (int i = 0; i < 8; ++i) rho += (g + i < n1 && o[i] <= key) ? 1u : 0u;
         return d.cap_upper + rho;  // the chunk of rank rho (rho = g + 8: laterally onward)
       }
+      constexpr int OKQ = GFSL_OK_WIN / 4;  // 16-B reads of the window
       const uint32_t s0 = r & ~3u;
-      uint32_t o[12];
+      uint32_t o[4 * OKQ];
 #pragma unroll
-      for (int q = 0; q < 3; ++q)
+      for (int q = 0; q < OKQ; ++q)
         asm volatile("ld.global.nc.L2::cache_hint.v4.u32 {%0,%1,%2,%3}, [%4], %5;"
                      : "=r"(o[4 * q]), "=r"(o[4 * q + 1]), "=r"(o[4 * q + 2]), "=r"(o[4 * q + 3])
                      : "l"(d.dir_ok + s0 + 4 * q), "l"(pol_up));
       uint32_t rho = s0;
 #pragma unroll
-      for (int i = 0; i < 12; ++i) rho += (s0 + i < n1 && o[i] <= key) ? 1u : 0u;
-      return d.cap_upper + rho;  // the chunk of rank rho (rho = s0 + 12: laterally onward)
+      for (int i = 0; i < 4 * OKQ; ++i) rho += (s0 + i < n1 && o[i] <= key) ? 1u : 0u;
+      return d.cap_upper + rho;  // the chunk of rank rho (rho = s0 + GFSL_OK_WIN: laterally onward)
     }
     if (!r) return head0;
     uint32_t c;
