@@ -366,10 +366,14 @@ static void launch_update(gfsl *h, const BatchIn &in, cudaStream_t s, cudaEvent_
   BatchCtl *next = h->ctl_buf[h->ctl_cur ^ 1];
   if (!fused) {  // (the small-batch kernel ran the update phase already)
     // eight mutations per warp for large batches, four below GFSL_UPD_SEG_SMALL_MAX ops
-    if (N == 16 && in.n < GFSL_UPD_SEG_SMALL_MAX)
-      cudaLaunchKernelEx(&lc, update_kernel<N, GFSL_UPD_SEG_SMALL>, h->d, in, h->ctl, update_in(h), serial, next);
+    // (R40: the grouped path is its own instantiation, so the default one carries none of it)
+    const bool small = N == 16 && in.n < GFSL_UPD_SEG_SMALL_MAX;
+    if (h->group_now)
+      cudaLaunchKernelEx(&lc, small ? update_kernel<N, GFSL_UPD_SEG_SMALL, true> : update_kernel<N, GFSL_UPD_SEG, true>,
+                         h->d, in, h->ctl, update_in(h), serial, next);
     else
-      cudaLaunchKernelEx(&lc, update_kernel<N>, h->d, in, h->ctl, update_in(h), serial, next);
+      cudaLaunchKernelEx(&lc, small ? update_kernel<N, GFSL_UPD_SEG_SMALL, false> : update_kernel<N, GFSL_UPD_SEG, false>,
+                         h->d, in, h->ctl, update_in(h), serial, next);
     h->launches += 1;  // update
   }
   h->ctl_clean[h->ctl_cur ^ 1] = true;
@@ -987,6 +991,7 @@ static gfsl_status enqueue_batch(gfsl *h, const uint8_t *ops, const uint32_t *ke
   }
   // small batches: search + barrier + update in one cooperative kernel
   const bool fused = !h->cfg.serial_updates && !h->cfg.combine && !h->cfg.count_reads && !h->ko_now && !n_dev &&
+                     !h->group_now &&
                      h->small_grid && n <= h->small_max && launch_small(h, in, s);
   bool ok = fused || dispatch_contains(h, in, s);
   if (!ok) {
