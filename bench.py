@@ -59,6 +59,12 @@ CONFIGS = {
     "C4-32": (100_000_000, 100_000_000, 50_000_000, 10, (0, 0, 100), "uniform", 32),
     "C4-16": (100_000_000, 100_000_000, 50_000_000, 10, (0, 0, 100), "uniform", 16),
     "C5": (1_000_000_000, 500_000_000, 125_000_000, 8, (10, 10, 80), "uniform", 16),
+    # one shard of C5 strong-scaled over G = 2 / 4 / 8 GPUs (R/G keys, its 1/G slice of
+    # every global batch, uniform in the shard's local key space), on one GPU: the local
+    # work of each rank of `--gpus G --config C5` without the exchange
+    "C5-S2": (500_000_000, 250_000_000, 62_500_000, 8, (10, 10, 80), "uniform", 16),
+    "C5-S4": (250_000_000, 125_000_000, 31_250_000, 8, (10, 10, 80), "uniform", 16),
+    "C5-S8": (125_000_000, 62_500_000, 15_625_000, 8, (10, 10, 80), "uniform", 16),
     # NEXT-4: the paper's other workloads (Fig 5.3 mixes, Fig 5.4b/c single-op runs)
     "M1-1-98": (1_000_000, 500_000, 625_000, 16, (1, 1, 98), "uniform", 16),
     "M5-5-90": (1_000_000, 500_000, 625_000, 16, (5, 5, 90), "uniform", 16),

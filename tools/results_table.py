@@ -21,6 +21,9 @@ DESC = {
     "INS-1M": "Insert-only, R ops from empty (INS-1M, Fig 5.4b)",
     "DEL-1M": "Delete-only, R ops from full (DEL-1M, Fig 5.4c)",
     "C5": "**C5** R=1B, 500M live keys, 125M-op batches (8 timed), one GPU",
+    "C5-S2": "C5-S2: one shard of C5 at 2 GPUs (R=500M, 250M keys, 62.5M-op batches), its local work",
+    "C5-S4": "C5-S4: one shard of C5 at 4 GPUs (R=250M, 125M keys, 31.25M-op batches), its local work",
+    "C5-S8": "C5-S8: one shard of C5 at 8 GPUs (R=125M, 62.5M keys, 15.6M-op batches), its local work",
 }
 
 
