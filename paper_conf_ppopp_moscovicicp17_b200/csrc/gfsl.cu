@@ -57,6 +57,12 @@ void gfsl_internal_set_error(const std::string &s) { set_last_error(s); }  // gf
 // environment at gfsl_create overrides; 0 = never).
 // Measured: no gain at C1 (the time is the lock-session chain, not the kernel
 // boundary), +3% at C2-5050 with a 128K threshold -- off by default.
+#ifndef GFSL_NO_DERIVE_PATH
+#define GFSL_DERIVE_PATH 1  // R41 (ablation: -DGFSL_NO_DERIVE_PATH)
+#else
+#define GFSL_DERIVE_PATH 0
+#endif
+
 #ifndef GFSL_SMALL_BATCH_DEFAULT
 #define GFSL_SMALL_BATCH_DEFAULT 0
 #endif
@@ -80,6 +86,8 @@ struct gfsl {
   uint32_t *gnext = nullptr;  // R40: [list_cap] group links of the records
   uint32_t *ghead = nullptr;  // R40: [cap_bottom] per level-0 chunk, EMPTY_GROUP between batches
   bool group_now = false;     // R40: this batch's records are grouped by chunk
+  bool derive_now = false;    // R41: this batch's directory-entered records write no path
+  bool derive_ok = true;      // R41 allowed (GFSL_DERIVE_PATH=0 in the environment at create: no)
   uint64_t list_cap = 0;
   uint32_t *h_error = nullptr;  // mapped host memory, device alias in d.error
   cudaEvent_t last = nullptr;
@@ -188,7 +196,7 @@ static SearchOut search_out(gfsl *h) {
                      0u};
   return SearchOut{h->mut_rec, h->plan_path, h->cfg.serial_updates ? h->mut_of : nullptr,
                    h->ctl->mcnt, h->region_cap, nullptr, nullptr, full, h->spread_now ? 1u : 0u,
-                   h->group_now ? h->ghead : nullptr, h->group_now ? h->gnext : nullptr};
+                   h->group_now ? h->ghead : nullptr, h->group_now ? h->gnext : nullptr, h->derive_now ? 1u : 0u};
 }
 // What the update kernel reads: the same records, or the net mutations of combining mode.
 static SearchOut update_in(gfsl *h) {
@@ -593,6 +601,8 @@ extern "C" gfsl_t gfsl_create_ex(uint64_t key_range, uint64_t capacity, const gf
     h->l0_entry = (e && *e && *e != '0') ? 0u : 1u;
     const char *ko = getenv("GFSL_KEY_ORDER");
     h->key_order = ko && *ko ? atoi(ko) : -1;
+    const char *dp = getenv("GFSL_DERIVE_PATH");
+    h->derive_ok = !(dp && *dp == '0');
     const char *sb = getenv("GFSL_SMALL_BATCH");  // ops; 0 = never (default GFSL_SMALL_BATCH_DEFAULT)
     h->small_max = sb && *sb ? (uint32_t)atoi(sb) : (uint32_t)GFSL_SMALL_BATCH_DEFAULT;
   }
@@ -964,6 +974,9 @@ static gfsl_status enqueue_batch(gfsl *h, const uint8_t *ops, const uint32_t *ke
   // them: update_multi at N = 16 / 32)
   h->group_now = h->d.lazy_upper && !h->cfg.combine && !h->cfg.serial_updates && h->cfg.group == GFSL_GROUP_ON &&
                  (h->N == 16 || h->N == 32) && GFSL_UPD_SEG != 16 && GFSL_UPD_SEG_SMALL != 16;
+  // R41: the update paths that derive a record's path (update_multi at N = 16 / 32)
+  h->derive_now = GFSL_DERIVE_PATH && h->derive_ok && h->d.lazy_upper && !h->cfg.combine && !h->cfg.serial_updates &&
+                  (h->N == 16 || h->N == 32) && GFSL_UPD_SEG != 16 && GFSL_UPD_SEG_SMALL != 16;
   std::array<cudaEvent_t, 5> ev{};
   const bool prof = h->cfg.profile_phases != 0;
   if (prof) {

@@ -91,8 +91,44 @@ struct SearchOut {
   // EMPTY_GROUP between batches (the update kernel resets the entries it takes).
   uint32_t *ghead;
   uint32_t *gnext;
+  // R41: 1 = a mutation whose traversal entered level 0 through the directory (R37) does
+  // not write its path: levels >= 1 are the closed form of its key's directory rank, which
+  // the update kernel recomputes in the rare cases that need them (record flag
+  // PATH_DERIVED; lazy batches, update paths that support it)
+  uint32_t derive_path;
 };
 constexpr uint32_t EMPTY_GROUP = 0xFFFFFFFFu;
+constexpr uint32_t PATH_DERIVED = 0x40000000u;  // on a record's op word (R41)
+
+// R41: the directory rank of an internal key (R27b / R27c layouts): the rank the search
+// kernel entered level 0 with.  The directory is read-only from the search kernel to the
+// next rebuild.
+__device__ __forceinline__ uint32_t dir_rank_of(const DevState &d, uint32_t key) {
+  const uint32_t q = key >> d.dir_hdr[0];
+#ifdef GFSL_DIR_U32
+  return ((const uint32_t *)d.dir)[q];
+#else
+  if (d.dir_hdr[8]) {
+    const uint32_t g = q / DIR_SEC_BUCKETS;
+    const uint8_t *sec = d.dir + (size_t)g * 32;
+    return *(const uint32_t *)sec + sec[4 + (q - g * DIR_SEC_BUCKETS)];
+  }
+  return d.dir_base[q >> 5] + d.dir[q];
+#endif
+}
+// R41: lane l's path entry of such a record (lanes above the snapshot height: head[l]),
+// the chunk the search kernel would have recorded: path[0] = the record's bottom chunk,
+// path[l] = the chunk of rebuilt level l that holds rank r / F^l (R27, R37).
+template <int N>
+__device__ __forceinline__ uint32_t derived_path_lane(const DevState &d, uint32_t k, uint32_t c0, int lane,
+                                                      bool path_lane, uint32_t head_l) {
+  if (!path_lane) return head_l;
+  if (lane == 0) return c0;
+  constexpr uint32_t F = N - 4;  // keys per rebuilt upper chunk (RebuildBufs::fill)
+  uint32_t q = dir_rank_of(d, k);
+  for (int l = 0; l < lane; ++l) q /= F;
+  return q ? d.dir_hdr[32 + lane] + q - 1u : (uint32_t)(lane == 1 ? 0 : lane - 1);
+}
 
 // A record slot in the writing block's region (BatchCtl::mcnt).
 __device__ __forceinline__ uint32_t mut_slot(const SearchOut &so) {
@@ -413,12 +449,15 @@ __device__ __forceinline__ void search_body(const DevState &d, const BatchIn &in
             res[opi] = mut ? 1 : 0;
             if (mut) {
               m = mut_slot(so);
-              // {op index | DELETE_FLAG, key, path[0], top (Delete) | value (Insert)}
-              const uint32_t w = opi | (cur_op.x & DELETE_FLAG);
+              // R41: entered at level 0 through the directory -> the path is derivable
+              const bool derive = so.derive_path && via_l0;
+              // {op index | DELETE_FLAG | PATH_DERIVED, key, path[0], top (Delete) | value (Insert)}
+              const uint32_t w = opi | (cur_op.x & DELETE_FLAG) | (derive ? PATH_DERIVED : 0u);
               // R33: in lazy mode a Delete's top is 0 (level-1 copies of k stay until the
               // next rebuild, as stale separators)
               so.mut_rec[m] = make_uint4(w, k, here, (cur_op.x & DELETE_FLAG) ? (d.lazy_upper ? 0u : (uint32_t)seen_top) : cur_val);
               if (so.ghead) so.gnext[m] = atomicExch(so.ghead + (here - d.cap_upper), m);  // R40
+              if (!derive) {
               my_path[0] = here;  // path[0] = the enclosing bottom chunk
               if (via_dir) {      // levels >= 2 (and 1, R37) from the directory rank (R27)
                 uint32_t q = cur_r / F;
@@ -433,6 +472,7 @@ __device__ __forceinline__ void search_body(const DevState &d, const BatchIn &in
               uint4 *dst = reinterpret_cast<uint4 *>(so.plan_path + (size_t)m * PLAN_LEVELS);
 #pragma unroll
               for (int q = 0; q < PLAN_LEVELS / 4; ++q) dst[q] = src[q];
+              }
             }
           }
           if (so.mut_of) so.mut_of[opi] = m;

@@ -86,3 +86,37 @@ def test_small_batch_kernel_churn_with_rebuilds(monkeypatch):
     st = g.stats()
     assert st["splits"] > 0
     g.close()
+
+
+@pytest.mark.parametrize("N", [16, 32])
+def test_derived_paths_match_recorded_paths(N, monkeypatch):
+    """R41: in lazy batches a directory-entered mutation writes no path and the update
+    kernel recomputes its levels >= 1 from the key's directory rank when a general-path op
+    (split, merge, a Delete whose key moved) needs them.  Heavy 50/50 churn with rebuilds
+    between batches, derived vs recorded paths: the same results (vs Oracle-A) and valid
+    structures after every batch."""
+    R = 20_000
+    monkeypatch.setenv("GFSL_DERIVE_PATH", "0")
+    rec = GFSL(R, chunk_entries=N, rebuild_every=2)
+    monkeypatch.delenv("GFSL_DERIVE_PATH")
+    der = GFSL(R, chunk_entries=N, rebuild_every=2)
+    o = OracleMap(R)
+    rng = np.random.default_rng(900 + N)
+    k0 = rng.permutation(R)[:R // 2].astype(np.uint32)
+    for g in (rec, der):
+        g.batch(*to_dev(np.ones(k0.size, np.uint8), k0, k0 + 3))
+    o.batch(np.ones(k0.size, np.uint8), k0, k0 + 3)
+    for b in range(30):
+        key = rng.choice(R, 6000, replace=False).astype(np.uint32)
+        op = rng.choice([0, 1, 2], key.size, p=[0.2, 0.4, 0.4]).astype(np.uint8)
+        val = rng.integers(0, 2**32, key.size, dtype=np.uint64).astype(np.uint32)
+        e = o.batch(op, key, val)
+        for g in (rec, der):
+            r = g.batch(*to_dev(op, key, val)).cpu().numpy()
+            assert np.array_equal(r, e), f"batch {b}"
+        check_all(der, o, cross=False)
+        assert rec.check().violations == 0
+    st = der.stats()
+    assert st["splits"] > 0 and st["merges"] > 0
+    rec.close()
+    der.close()
