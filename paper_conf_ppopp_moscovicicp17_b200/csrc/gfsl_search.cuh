@@ -147,6 +147,12 @@ constexpr uint32_t CW_NOTMUT = 0x20000000u;  // Contains or invalid: not part of
 #define GFSL_OK_WIN 8
 #endif
 
+// 1 = teams whose ops are done keep re-reading their last chunk while the warp runs (the
+// round-1 code, an ablation): 0 skips those loads
+#ifndef GFSL_IDLE_LOADS
+#define GFSL_IDLE_LOADS 0
+#endif
+
 #ifndef GFSL_SEARCH_MIN_BLOCKS
 // 4 blocks per SM (<= 64 registers, no spill): with level 0 entered directly (R37/R38) a
 // traversal is ~1-2 dependent gathers, latency-bound (ncu at C5: 0.45 eligible warps per
@@ -363,7 +369,12 @@ __device__ __forceinline__ void search_body(const DevState &d, const BatchIn &in
 
   while (__any_sync(FULL, active)) {
     ChunkSlice<EPL> s;
-    ld_slice_nc<EPL>(d.pool + (size_t)cur * N + t * EPL, s, level == 0 ? pol_l0 : pol_up);  // idle teams re-read `cur`
+    if (!GFSL_IDLE_LOADS && !active) {  // a team whose ops are done issues no request
+#pragma unroll
+      for (int j = 0; j < EPL; ++j) s.k[j] = s.v[j] = KEY_EMPTY;
+    } else {
+      ld_slice_nc<EPL>(d.pool + (size_t)cur * N + t * EPL, s, level == 0 ? pol_l0 : pol_up);
+    }
     if (pf_dir) {
       if ((nxt.op == 0 || (dir_upd && nxt.op <= 2)) && (uint64_t)nxt.key < in.key_range) {
         nxt_dir = ld_dir(nxt.key + 1u);

@@ -46,3 +46,15 @@ def test_range_sharded_cpu_baseline_runs():
     assert r["threads"] == 4 and r["mops"] > 0 and r["batches"] >= 1
     r1 = bench.oracle_sample("C1", 3, 1, budget_s=5.0, threads=1)
     assert r1["threads"] == 1 and r1["mops"] > 0
+
+
+def test_c5_shard_configs_are_the_strong_scaled_slices():
+    """C5-S<G> is what one rank of `--gpus G --config C5` holds and runs: R/G keys in its
+    local key space, its share of the prefill, a 1/G slice of every global batch, the same
+    mix, distribution and chunk size."""
+    import bench
+    R, pre, B, nb, mix, dist, N = bench.CONFIGS["C5"]
+    for G in (2, 4, 8):
+        r, p, b, n, m, di, c = bench.CONFIGS[f"C5-S{G}"]
+        assert (r, p, b) == (R // G, pre // G, B // G)
+        assert (n, m, di, c) == (nb, mix, dist, N)
