@@ -646,12 +646,20 @@ def run_extras(args, S, g, local_g, inputs, W, steps, PROF, st0, st_t, flush, de
     rand = None
     if not args.no_ubench and rank == 0:
         from paper_conf_ppopp_moscovicicp17_b200.gfsl import ubench
-        r_hbm, t_hbm = ubench(Cb, 16 << 30)
+        # the gathers span the config's level-0 footprint (a power of two >= it, 512 MiB ..
+        # 16 GiB): TLB reach and DRAM locality depend on it, and a ceiling measured over 16
+        # GiB was exceeded by C4-16's chunk gathers over 1.3 GB (round 2)
+        ub_bytes = 512 << 20
+        while ub_bytes < l0_bytes and ub_bytes < (16 << 30):
+            ub_bytes <<= 1
+        r_hbm, t_hbm = ubench(Cb, ub_bytes)
         r_l2, t_l2 = ubench(Cb, 32 << 20)
         rand = {"block_bytes": Cb, "R_rand_hbm_GBps": round(r_hbm, 1), "R_rand_l2_GBps": round(r_l2, 1),
                 "chase_latency_hbm_ns": round(t_hbm, 1), "chase_latency_l2_ns": round(t_l2, 1),
-                "how": "gfsl_ubench: random aligned chunk-size gathers over 16 GiB (32 MiB for L2), the "
-                       "search kernel's team shape, 4/8/16 gathers in flight per team (best kept)"}
+                "buffer_MiB": ub_bytes >> 20,
+                "how": "gfsl_ubench: random aligned chunk-size gathers over a buffer the size of the config's "
+                       "level 0 (rounded up to a power of two; 32 MiB for L2), the search kernel's team "
+                       "shape, 4/8/16 gathers in flight per team (best kept)"}
     # R37/R38: a traversal entered at level 0 reads no upper level; its index lookup is one
     # 32-B sector of the sorted min keys (4 B per level-0 chunk), compulsory from DRAM for
     # the part of that array the L2 cannot hold beside the 16-MiB directory
