@@ -87,6 +87,7 @@ struct gfsl {
   uint32_t *ghead = nullptr;  // R40: [cap_bottom] per level-0 chunk, EMPTY_GROUP between batches
   bool group_now = false;     // R40: this batch's records are grouped by chunk
   bool derive_now = false;    // R41: this batch's directory-entered records write no path
+  bool idle_skip = false;     // this batch's search kernel: finished teams issue no loads
   bool derive_ok = true;      // R41 allowed (GFSL_DERIVE_PATH=0 in the environment at create: no)
   uint64_t list_cap = 0;
   uint32_t *h_error = nullptr;  // mapped host memory, device alias in d.error
@@ -249,6 +250,8 @@ static void launch_contains(gfsl *h, const BatchIn &in, cudaStream_t s) {
   set_pdl(h, attr[lc.numAttrs++]);
   if (h->cfg.count_reads)
     cudaLaunchKernelEx(&lc, search_kernel<N, TEAM, true>, h->d, in, h->ctl, search_out(h));
+  else if (h->idle_skip)  // level 0 beyond the L2: finished teams issue no loads
+    cudaLaunchKernelEx(&lc, search_kernel<N, TEAM, false, true>, h->d, in, h->ctl, search_out(h));
   else
     cudaLaunchKernelEx(&lc, search_kernel<N, TEAM, false>, h->d, in, h->ctl, search_out(h));
   h->launches += 1;
@@ -951,10 +954,11 @@ static gfsl_status enqueue_batch(gfsl *h, const uint8_t *ops, const uint32_t *ke
     const double l0 = (double)h->h_bump[0] * h->N * 8, up = (double)h->h_bump[1] * h->N * 8;
 #ifdef GFSL_L0_EVICT_FIRST_ALWAYS
     h->d.l0_evict_first = 1u;
-    (void)l0; (void)up; (void)l2;
+    (void)up;
 #else
     h->d.l0_evict_first = (l0 > l2 && up <= l2) ? 0u : 1u;
 #endif
+    h->idle_skip = l0 > l2;
   }
   // R37: enter level 0 straight from the directory (Contains, and the Insert/Delete of lazy
   // batches); GFSL_NO_L0_ENTRY (environment, read at gfsl_create) keeps R27's level-1 entry

@@ -147,12 +147,6 @@ constexpr uint32_t CW_NOTMUT = 0x20000000u;  // Contains or invalid: not part of
 #define GFSL_OK_WIN 8
 #endif
 
-// 1 = teams whose ops are done keep re-reading their last chunk while the warp runs (the
-// round-1 code, an ablation): 0 skips those loads
-#ifndef GFSL_IDLE_LOADS
-#define GFSL_IDLE_LOADS 0
-#endif
-
 #ifndef GFSL_SEARCH_MIN_BLOCKS
 // 4 blocks per SM (<= 64 registers, no spill): with level 0 entered directly (R37/R38) a
 // traversal is ~1-2 dependent gathers, latency-bound (ncu at C5: 0.45 eligible warps per
@@ -164,7 +158,7 @@ constexpr uint32_t CW_NOTMUT = 0x20000000u;  // Contains or invalid: not part of
 
 // The search phase of a batch: the body of search_kernel, and the first half of the
 // small-batch kernel (gfsl_update.cuh).
-template <int N, int TEAM, bool COUNT = false>
+template <int N, int TEAM, bool COUNT = false, bool IDLE_SKIP = false>
 __device__ __forceinline__ void search_body(const DevState &d, const BatchIn &in, BatchCtl *__restrict__ ctl,
                                             const SearchOut &so) {
   constexpr int EPL = N / TEAM;
@@ -369,7 +363,7 @@ __device__ __forceinline__ void search_body(const DevState &d, const BatchIn &in
 
   while (__any_sync(FULL, active)) {
     ChunkSlice<EPL> s;
-    if (!GFSL_IDLE_LOADS && !active) {  // a team whose ops are done issues no request
+    if (IDLE_SKIP && !active) {  // a team whose ops are done issues no request
 #pragma unroll
       for (int j = 0; j < EPL; ++j) s.k[j] = s.v[j] = KEY_EMPTY;
     } else {
@@ -520,10 +514,13 @@ __device__ __forceinline__ void search_body(const DevState &d, const BatchIn &in
   }
 }
 
-template <int N, int TEAM, bool COUNT = false>
+// IDLE_SKIP: a team whose ops are done issues no chunk load while its warp finishes (the
+// host takes it when level 0 exceeds the L2: C5 with R41 9.8 vs 13.4-14.6 ms per batch;
+// where level 0 is L2-resident the re-reads are cheap and the skip's branch is not: C3 -4%)
+template <int N, int TEAM, bool COUNT = false, bool IDLE_SKIP = false>
 __global__ void __launch_bounds__(256, GFSL_SEARCH_MIN_BLOCKS)
 search_kernel(const __grid_constant__ DevState d, const BatchIn in, BatchCtl *__restrict__ ctl, SearchOut so) {
-  search_body<N, TEAM, COUNT>(d, in, ctl, so);
+  search_body<N, TEAM, COUNT, IDLE_SKIP>(d, in, ctl, so);
 }
 
 // The update kernel's view of the region-numbered records: slot s in [0, total) ->
