@@ -801,7 +801,7 @@ static gfsl_status ensure_lists(gfsl *h, uint64_t n) {
   const uint64_t cap = std::max<uint64_t>(n, 1024);
   CK(cudaMalloc(&h->plan_path, cap * 4 * PLAN_LEVELS));
   CK(cudaMalloc(&h->mut_of, cap * 4));
-  CK(cudaMalloc(&h->mut_rec, cap * 16));
+  CK(cudaMalloc(&h->mut_rec, cap * 16 * REC_STRIDE));
   CK(cudaMalloc(&h->gnext, cap * 4));
   h->list_cap = cap;
   return GFSL_OK;
@@ -837,7 +837,7 @@ static gfsl_status ensure_combine(gfsl *h, uint64_t n) {
       CK(cudaMalloc(&h->ck[b], cap * 4));
       CK(cudaMalloc(&h->cw[b], cap * 4));
     }
-    CK(cudaMalloc(&h->net_rec, cap * 16));
+    CK(cudaMalloc(&h->net_rec, cap * 16 * REC_STRIDE));
     CK(cudaMalloc(&h->net_path, cap * 4 * PLAN_LEVELS));
     CK(cudaMalloc(&h->vw, cap * 8));
     h->comb_cap = cap;

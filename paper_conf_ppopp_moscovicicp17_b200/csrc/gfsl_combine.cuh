@@ -66,9 +66,9 @@ combine_kernel(const BatchIn in, BatchCtl *__restrict__ ctl, const uint32_t *__r
     if (p0 != fin) {  // net Insert (absent -> present) or net Delete (present -> absent)
       const uint32_t m = cand.mut_of[i];  // the last op's snapshot answer mutates: recorded
       q = mut_slot(net);
-      uint4 rec = cand.mut_rec[m];
+      uint4 rec = *rec_at(cand.mut_rec, m);
       if (fin) rec.w = v_new;
-      net.mut_rec[q] = rec;
+      rec_store(net.mut_rec, q, rec);
       const uint4 *src = reinterpret_cast<const uint4 *>(cand.plan_path + (size_t)m * PLAN_LEVELS);
       uint4 *dst = reinterpret_cast<uint4 *>(net.plan_path + (size_t)q * PLAN_LEVELS);
 #pragma unroll

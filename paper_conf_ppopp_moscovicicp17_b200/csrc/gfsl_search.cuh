@@ -130,10 +130,36 @@ __device__ __forceinline__ uint32_t derived_path_lane(const DevState &d, uint32_
   return q ? d.dir_hdr[32 + lane] + q - 1u : (uint32_t)(lane == 1 ? 0 : lane - 1);
 }
 
+// Mutation records occupy REC_STRIDE x 16 B: 1 = packed 16-B records (default); 2 = one
+// full 32-B sector per record, written with one 32-B store, so that no record is a
+// partial-sector write (measured: within 0.6% of 1 at C2-C5, profiles/r02/ab_record_stride.txt).
+#ifndef GFSL_REC_STRIDE
+#define GFSL_REC_STRIDE 1
+#endif
+constexpr uint32_t REC_STRIDE = GFSL_REC_STRIDE;
+__device__ __forceinline__ uint4 *rec_at(uint4 *base, uint32_t m) { return base + (size_t)m * REC_STRIDE; }
+__device__ __forceinline__ const uint4 *rec_at(const uint4 *base, uint32_t m) { return base + (size_t)m * REC_STRIDE; }
+__device__ __forceinline__ void rec_store(uint4 *base, uint32_t m, uint4 r) {
+  if (REC_STRIDE == 2) {
+    asm volatile("st.global.v8.u32 [%0], {%1,%2,%3,%4,%5,%5,%5,%5};" ::"l"(base + (size_t)m * 2), "r"(r.x), "r"(r.y),
+                 "r"(r.z), "r"(r.w), "r"(0u)
+                 : "memory");
+  } else {
+    base[m] = r;
+  }
+}
+
 // A record slot in the writing block's region (BatchCtl::mcnt).
+// Warp-aggregated: the converged lanes that append take consecutive slots with one atomic.
 __device__ __forceinline__ uint32_t mut_slot(const SearchOut &so) {
   const uint32_t rg = blockIdx.x % BatchCtl::MUT_REGIONS;
-  return rg * so.region_cap + atomicAdd(so.mut_count + rg, 1u);
+  const uint32_t am = __activemask();
+  const int lane = threadIdx.x & 31;
+  const int leader = __ffs(am) - 1;
+  uint32_t base = 0;
+  if (lane == leader) base = atomicAdd(so.mut_count + rg * BatchCtl::CNT_STRIDE, (uint32_t)__popc(am));
+  base = __shfl_sync(am, base, leader);
+  return rg * so.region_cap + base + (uint32_t)__popc(am & ((1u << lane) - 1u));
 }
 
 // Combining-mode payload flags (R26); the op index is < 2^29.
@@ -460,7 +486,7 @@ __device__ __forceinline__ void search_body(const DevState &d, const BatchIn &in
               const uint32_t w = opi | (cur_op.x & DELETE_FLAG) | (derive ? PATH_DERIVED : 0u);
               // R33: in lazy mode a Delete's top is 0 (level-1 copies of k stay until the
               // next rebuild, as stale separators)
-              so.mut_rec[m] = make_uint4(w, k, here, (cur_op.x & DELETE_FLAG) ? (d.lazy_upper ? 0u : (uint32_t)seen_top) : cur_val);
+              rec_store(so.mut_rec, m, make_uint4(w, k, here, (cur_op.x & DELETE_FLAG) ? (d.lazy_upper ? 0u : (uint32_t)seen_top) : cur_val));
               if (so.ghead) so.gnext[m] = atomicExch(so.ghead + (here - d.cap_upper), m);  // R40
               if (!derive) {
               my_path[0] = here;  // path[0] = the enclosing bottom chunk
@@ -555,7 +581,7 @@ struct MutMap {
 __device__ __forceinline__ void mutmap_build(const uint32_t *cnt, uint32_t *s_excl) {
   if (threadIdx.x < 32) {
     const int lane = threadIdx.x;
-    const uint32_t v = cnt[lane];
+    const uint32_t v = cnt[lane * BatchCtl::CNT_STRIDE];
     uint32_t incl = v;
 #pragma unroll
     for (int o = 1; o < 32; o <<= 1) {

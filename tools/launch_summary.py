@@ -22,13 +22,16 @@ def main():
             float(r[vi].replace(",", "")) / 1e3) for r in rows]
     steps, cur = [], None
     for name, t in seq:
-        if "FillFunctor" in name and t > 20:  # the L2 flush before a timed step
+        # the L2 flush before a timed step: torch's 256-MiB zero_ (FillFunctor in older
+        # torch, a vectorized elementwise kernel in newer), ~70 us
+        if (("FillFunctor" in name) or name.startswith("native::vectorized_elementwise")) and t > 20:
             if cur:
                 steps.append(cur)
             cur = []
             continue
         if cur is not None:
-            if "search_kernel" in name and name.endswith(", 1>"):  # counting replay: after the steps
+            targs = name[name.find("<") + 1:name.rfind(">")].split(",") if "<" in name else []
+            if "search_kernel" in name and len(targs) >= 3 and targs[2].strip() == "1":  # counting replay
                 steps.append(cur)
                 cur = None
                 continue
