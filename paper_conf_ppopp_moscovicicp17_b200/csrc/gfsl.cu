@@ -540,7 +540,6 @@ static void free_all(gfsl *h) {
   cudaFree(h->rb.word_prefix);
   cudaFree(h->rb.block_sum);
   cudaFree(h->rb.order_key);
-  cudaFree(h->rb.order_key16);
   cudaFree(h->rb.order_chunk);
   cudaFree(h->rb.n1);
   cudaFree(h->rb.levels);
@@ -664,7 +663,6 @@ extern "C" gfsl_t gfsl_create_ex(uint64_t key_range, uint64_t capacity, const gf
     if ((e = cudaMalloc(&b.block_sum, (size_t)b.blocks * 4)) != cudaSuccess) return fail("cudaMalloc(rebuild)", e);
     if ((e = cudaMalloc(&b.order_key, ((size_t)cap_b + 16) * 4)) != cudaSuccess) return fail("cudaMalloc(rebuild)", e);  // + the search kernel's look-ahead (R38)
     if ((e = cudaMalloc(&b.order_chunk, (size_t)cap_b * 4)) != cudaSuccess) return fail("cudaMalloc(rebuild)", e);
-    if ((e = cudaMalloc(&b.order_key16, ((size_t)cap_b + 64) * 2)) != cudaSuccess) return fail("cudaMalloc(rebuild)", e);
     if ((e = cudaMalloc(&b.n1, 32)) != cudaSuccess) return fail("cudaMalloc(rebuild)", e);
     if ((e = cudaMalloc(&b.levels, sizeof(RbLevels))) != cudaSuccess) return fail("cudaMalloc(rebuild)", e);
     cudaMemset(b.bitmap, 0, (size_t)b.words * 4);
@@ -672,7 +670,6 @@ extern "C" gfsl_t gfsl_create_ex(uint64_t key_range, uint64_t capacity, const gf
     h->d.dirty = b.n1 + 2;
     h->d.dir_oc = b.order_chunk;
     h->d.dir_ok = b.order_key;
-    h->d.dir_ok16 = b.order_key16;
     if ((e = cudaMalloc(&h->d.freelist, (size_t)cap_b * 8)) != cudaSuccess) return fail("cudaMalloc(freelist)", e);
     if ((e = cudaMalloc(&h->ghead, (size_t)cap_b * 4)) != cudaSuccess) return fail("cudaMalloc(ghead)", e);  // R40
     cudaMemset(h->ghead, 0xFF, (size_t)cap_b * 4);
@@ -683,11 +680,6 @@ extern "C" gfsl_t gfsl_create_ex(uint64_t key_range, uint64_t capacity, const gf
     // 2^GFSL_DIR_CAP_LOG2: one byte per bucket plus one 32-bit base per 32 buckets
     uint32_t dcap = 1024;
     while (dcap < (1u << GFSL_DIR_CAP_LOG2) && (uint64_t)dcap < key_range + 1) dcap <<= 1;
-    {  // tests: a smaller directory (GFSL_DIR_CAP buckets, a power of two >= 1024) forces
-       // the coarse-directory paths (R38b) on small structures
-      const char *dc = getenv("GFSL_DIR_CAP");
-      if (dc && *dc) dcap = std::min<uint32_t>(dcap, std::max<uint32_t>(1024u, (uint32_t)atoi(dc)));
-    }
     h->d.dir_cap = dcap;
 #ifdef GFSL_DIR_U32
     if ((e = cudaMalloc(&h->d.dir, (size_t)dcap * 4)) != cudaSuccess) return fail("cudaMalloc(dir)", e);

@@ -55,9 +55,6 @@ struct BatchCtl;
 #define GFSL_DIR_SECTOR_MAX 0xFFFFFFFFu
 #endif
 constexpr uint32_t DIR_SEC_BUCKETS = 28;
-// R38b: 16-bit sorted min keys: FAR flag, and the largest gap a non-FAR entry follows
-constexpr uint32_t OK16_FAR = 0x8000u;
-constexpr uint32_t OK16_SPAN = 1u << 14;
 
 // Device view of one handle.
 struct DevState {
@@ -112,7 +109,6 @@ struct DevState {
   // level 0 directly.  l0_entry = 1: the search kernel does so (concurrent modes).
   const uint32_t *dir_oc;
   const uint32_t *dir_ok;  // R38: the sorted min keys of the last rebuild (order_key)
-  const uint16_t *dir_ok16;  // R38b: their 16-bit copy (low 15 bits + FAR)
   uint32_t l0_entry;
   uint32_t *bump_host;  // mapped pinned host copy of bump[0..1], written by the search kernel
                         // at its start (the counters after the previous batch; host heuristics)

@@ -33,7 +33,6 @@ struct RebuildBufs {
   uint32_t *block_sum;    // [blocks]     popcount of each block, then its exclusive prefix
   uint32_t *order_key;    // [cap_bottom] min keys in key order
   uint32_t *order_chunk;  // [cap_bottom] their chunks
-  uint16_t *order_key16;  // [cap_bottom + 32] R38b: low 15 bits of order_key, bit 15 = FAR
   uint32_t *n1;           // [8]          marked chunks; old upper bump; dirty; active;
                           //              relocated (R38)
   void *levels;           // RbLevels computed once per rebuild (scan_top kernel)
@@ -287,18 +286,6 @@ __global__ void __launch_bounds__(256) rebuild_pack_kernel(const __grid_constant
   __shared__ RbLevels L;
   if (threadIdx.x == 0) L = *(const RbLevels *)b.levels;
   __syncthreads();
-  // R38b: the 16-bit copy of the sorted min keys the search kernel reads: the low 15 bits,
-  // and FAR (bit 15) when the key is >= 2^14 above its predecessor (or is the first);
-  // entries past n1 are FAR
-  for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < n1 + 32; i += gridDim.x * blockDim.x) {
-    uint16_t v = (uint16_t)OK16_FAR;
-    if (i < n1) {
-      const uint32_t k = b.order_key[i];
-      const bool far = i == 0 ? k >= OK16_SPAN : k - b.order_key[i - 1] >= OK16_SPAN;
-      v = (uint16_t)((k & 0x7FFFu) | (far ? OK16_FAR : 0u));
-    }
-    b.order_key16[i] = v;
-  }
   {
     // R27: bucket q = keys [q << shift, (q+1) << shift); r(q) = rank(q << shift), the
     // number of marked min keys (= level-1 entries >= 1) <= q << shift, so level-1 entry

@@ -169,10 +169,6 @@ constexpr uint32_t CW_NOTMUT = 0x20000000u;  // Contains or invalid: not part of
 
 // Keys of the sorted-min-key window a coarse directory (C5) reads: 8 (two 16-B reads; 12 and 16
 // measured slower at C5: every read is a request, and the kernel is request-bound)
-// R38b: a coarse directory reads the 16-bit copy of the sorted min keys (0: the 32-bit keys)
-#ifndef GFSL_OK16
-#define GFSL_OK16 1
-#endif
 #ifndef GFSL_OK_WIN
 #define GFSL_OK_WIN 8
 #endif
@@ -360,34 +356,6 @@ __device__ __forceinline__ void search_body(const DevState &d, const BatchIn &in
         for (int i = 0; i < 8; ++i) rho += (g + i < n1 && o[i] <= key) ? 1u : 0u;
         return d.cap_upper + rho;  // the chunk of rank rho (rho = g + 8: laterally onward)
       }
-#if GFSL_OK16
-      // R38b: the 16-bit copy (half the bytes: C5's 200-MB array becomes 100 MB, which the
-      // L2 can mostly hold): 16 entries from r rounded down to 8, two 16-B reads.  The
-      // entries below r are <= key (the directory's rank); from r on, count the prefix
-      // judged <= key by a 15-bit difference -- exact while an entry is within 2^14 of its
-      // predecessor (FAR otherwise: stop, i.e. at worst a rank too small and a lateral step)
-      {
-        const uint32_t s0 = r & ~7u;
-        uint32_t o[8];
-#pragma unroll
-        for (int q = 0; q < 2; ++q)
-          asm volatile("ld.global.nc.L2::cache_hint.v4.u32 {%0,%1,%2,%3}, [%4], %5;"
-                       : "=r"(o[4 * q]), "=r"(o[4 * q + 1]), "=r"(o[4 * q + 2]), "=r"(o[4 * q + 3])
-                       : "l"(d.dir_ok16 + s0 + 8 * q), "l"(pol_up));
-        uint32_t rho = r;
-        bool go = true;
-#pragma unroll
-        for (int i = 0; i < 16; ++i) {
-          const uint32_t e = (o[i >> 1] >> (16 * (i & 1))) & 0xFFFFu;
-          const uint32_t idx = s0 + (uint32_t)i;
-          if (idx >= r) {
-            go = go && idx < n1 && !(e & OK16_FAR) && ((key - e) & 0x7FFFu) < OK16_SPAN;
-            rho += go ? 1u : 0u;
-          }
-        }
-        return d.cap_upper + rho;  // (rho = s0 + 16: laterally onward)
-      }
-#endif
       constexpr int OKQ = GFSL_OK_WIN / 4;  // 16-B reads of the window
       const uint32_t s0 = r & ~3u;
       uint32_t o[4 * OKQ];
