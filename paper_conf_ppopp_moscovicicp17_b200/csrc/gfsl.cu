@@ -680,6 +680,11 @@ extern "C" gfsl_t gfsl_create_ex(uint64_t key_range, uint64_t capacity, const gf
     // 2^GFSL_DIR_CAP_LOG2: one byte per bucket plus one 32-bit base per 32 buckets
     uint32_t dcap = 1024;
     while (dcap < (1u << GFSL_DIR_CAP_LOG2) && (uint64_t)dcap < key_range + 1) dcap <<= 1;
+    {  // tests: a smaller directory (GFSL_DIR_CAP buckets, a power of two >= 1024) forces
+       // the coarse-directory path (C5's 8-key min-key window) on small structures
+      const char *dc = getenv("GFSL_DIR_CAP");
+      if (dc && *dc) dcap = std::min<uint32_t>(dcap, std::max<uint32_t>(1024u, (uint32_t)atoi(dc)));
+    }
     h->d.dir_cap = dcap;
 #ifdef GFSL_DIR_U32
     if ((e = cudaMalloc(&h->d.dir, (size_t)dcap * 4)) != cudaSuccess) return fail("cudaMalloc(dir)", e);

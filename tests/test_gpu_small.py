@@ -120,3 +120,51 @@ def test_derived_paths_match_recorded_paths(N, monkeypatch):
     assert st["splits"] > 0 and st["merges"] > 0
     rec.close()
     der.close()
+
+
+@pytest.mark.parametrize("layout", ["dense", "clusters", "sparse"])
+def test_coarse_directory_16bit_window(layout, monkeypatch):
+    """With a coarse directory (C5's regime: more level-0 chunks than directory buckets,
+    forced here by a 1024-bucket directory) the search kernel refines the directory's rank
+    from an 8-key window of the sorted min keys (R38, R27c) and continues laterally when
+    the key's chunk lies beyond it.  Dense keys, tight clusters far apart, and sparse keys:
+    every result vs Oracle-A, with the directory rebuilt after every batch."""
+    monkeypatch.setenv("GFSL_DIR_CAP", "1024")
+    rng = np.random.default_rng({"dense": 1, "clusters": 2, "sparse": 3}[layout])
+    if layout == "dense":
+        R = 200_000
+        keys = rng.permutation(R)[: R // 2]
+    elif layout == "clusters":
+        R = 1 << 30
+        starts = rng.choice(R // (1 << 20), 60, replace=False) * (1 << 20)
+        keys = np.unique(np.concatenate([s + rng.choice(3000, 1500, replace=False) for s in starts]))
+    else:
+        R = 1 << 31
+        keys = np.unique(rng.integers(0, R, 60_000))
+    keys = rng.permutation(keys).astype(np.uint32)
+    g = GFSL(R, capacity=len(keys) * 2, rebuild_every=1)
+    o = OracleMap(R)
+    g.batch(*to_dev(np.ones(keys.size, np.uint8), keys, keys ^ 7))
+    o.batch(np.ones(keys.size, np.uint8), keys, keys ^ 7)
+    for b in range(6):
+        # lookups of present keys, their neighbours, and random keys; a few mutations
+        probe = np.concatenate([rng.choice(keys, 20_000), rng.choice(keys, 5_000) + 1,
+                                rng.integers(0, R, 5_000).astype(np.uint32)]).astype(np.uint32)
+        probe = np.minimum(probe, R - 1).astype(np.uint32)
+        mut = rng.choice(keys, 2_000, replace=False)
+        op = np.concatenate([np.zeros(probe.size, np.uint8), np.full(mut.size, 2, np.uint8)])
+        key = np.concatenate([probe, mut]).astype(np.uint32)
+        mutated = np.zeros(key.size, bool)
+        mutated[probe.size:] = True
+        # <= 1 mutation per key: the Contains of a mutated key may repeat (R1)
+        r = g.batch(*to_dev(op, key, None)).cpu().numpy()
+        e = o.batch(op, key, None)
+        assert np.array_equal(r, e), f"{layout} batch {b}: {np.count_nonzero(r != e)} results differ"
+        keys = np.setdiff1d(keys, mut)
+        ins = rng.integers(0, R, 2_000).astype(np.uint32)
+        ins = np.setdiff1d(ins, keys)[:1500]
+        r = g.batch(*to_dev(np.ones(ins.size, np.uint8), ins, ins)).cpu().numpy()
+        assert np.array_equal(r, o.batch(np.ones(ins.size, np.uint8), ins, ins))
+        keys = np.union1d(keys, ins).astype(np.uint32)
+        assert g.check().violations == 0
+    g.close()
