@@ -964,6 +964,7 @@ static gfsl_status enqueue_batch(gfsl *h, const uint8_t *ops, const uint32_t *ke
     h->d.l0_evict_first = (l0 > l2 && up <= l2) ? 0u : 1u;
 #endif
     h->idle_skip = l0 > l2;
+    h->d.upd_prefetch = l0 > l2 ? 0u : 1u;
   }
   // R37: enter level 0 straight from the directory (Contains, and the Insert/Delete of lazy
   // batches); GFSL_NO_L0_ENTRY (environment, read at gfsl_create) keeps R27's level-1 entry

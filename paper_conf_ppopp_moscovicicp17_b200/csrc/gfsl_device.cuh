@@ -110,6 +110,9 @@ struct DevState {
   const uint32_t *dir_oc;
   const uint32_t *dir_ok;  // R38: the sorted min keys of the last rebuild (order_key)
   uint32_t l0_entry;
+  uint32_t upd_prefetch;  // the update kernel prefetches each record's chunk into L2 (host:
+                          // while level 0 fits the L2; beyond it the extra request costs
+                          // more than it saves -- C5 update 2.21 vs 2.55 ms, round 2)
   uint32_t *bump_host;  // mapped pinned host copy of bump[0..1], written by the search kernel
                         // at its start (the counters after the previous batch; host heuristics)
 };
@@ -151,7 +154,11 @@ struct BatchCtl {
   // queue j of Q hands out the mutation slots j, j + Q, j + 2Q, ... in order; one counter
   // per 32-byte sector
   static constexpr int UQ_MAX = 2048;
-  uint32_t uq[UQ_MAX * 8];
+#ifndef GFSL_UQ_STRIDE
+#define GFSL_UQ_STRIDE 8  // words between queue counters (8: one per 32-B sector; 32: per 128-B line)
+#endif
+  static constexpr int UQ_STRIDE = GFSL_UQ_STRIDE;
+  uint32_t uq[UQ_MAX * UQ_STRIDE];
 };
 
 __device__ __forceinline__ uint32_t lo32(uint64_t x) { return (uint32_t)x; }
