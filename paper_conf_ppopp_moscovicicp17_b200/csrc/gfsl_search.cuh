@@ -169,6 +169,11 @@ constexpr uint32_t CW_NOTMUT = 0x20000000u;  // Contains or invalid: not part of
 
 // Keys of the sorted-min-key window a coarse directory (C5) reads: 8 (two 16-B reads; 12 and 16
 // measured slower at C5: every read is a request, and the kernel is request-bound)
+// L2 priority of the coarse directory's min-key window reads: 0 evict_last (as the
+// directory), 1 evict_normal, 2 evict_first
+#ifndef GFSL_OK_POLICY
+#define GFSL_OK_POLICY 0
+#endif
 #ifndef GFSL_OK_WIN
 #define GFSL_OK_WIN 8
 #endif
@@ -319,6 +324,14 @@ __device__ __forceinline__ void search_body(const DevState &d, const BatchIn &in
 #endif
   const uint64_t pol_l0 = (GFSL_SEARCH_HINTS >= 1 && d.l0_evict_first) ? l2_policy_evict_first() : l2_policy_evict_normal();
   const uint64_t pol_up = GFSL_SEARCH_HINTS >= 2 ? l2_policy_evict_last() : l2_policy_evict_normal();
+  // the coarse directory's min-key window (C5: a 200-MB array, larger than the L2)
+#if GFSL_OK_POLICY == 1
+  const uint64_t pol_ok = l2_policy_evict_normal();
+#elif GFSL_OK_POLICY == 2
+  const uint64_t pol_ok = l2_policy_evict_first();
+#else
+  const uint64_t pol_ok = pol_up;
+#endif
   // the op's directory rank (R27b): base of its 32-bucket group + its byte
   auto dir_rank = [&](uint2 e, uint32_t) -> uint32_t { return e.x + e.y; };
   auto ld_dir = [&](uint32_t key) -> uint2 {
@@ -363,7 +376,7 @@ __device__ __forceinline__ void search_body(const DevState &d, const BatchIn &in
       for (int q = 0; q < OKQ; ++q)
         asm volatile("ld.global.nc.L2::cache_hint.v4.u32 {%0,%1,%2,%3}, [%4], %5;"
                      : "=r"(o[4 * q]), "=r"(o[4 * q + 1]), "=r"(o[4 * q + 2]), "=r"(o[4 * q + 3])
-                     : "l"(d.dir_ok + s0 + 4 * q), "l"(pol_up));
+                     : "l"(d.dir_ok + s0 + 4 * q), "l"(pol_ok));
       uint32_t rho = s0;
 #pragma unroll
       for (int i = 0; i < 4 * OKQ; ++i) rho += (s0 + i < n1 && o[i] <= key) ? 1u : 0u;
