@@ -745,10 +745,14 @@ def run_e2e(args, S, inputs, W, steps, world, dev):
     step the rank's slice is copied in, the collective batch runs, the results are copied
     out (one stream); wall clock, max over ranks."""
     host = [tuple(x.cpu().pin_memory() for x in inp) for inp in inputs]
+    # a workload without Inserts reads no value: its caller passes none (values = NULL)
+    no_ins = CONFIGS[args.config][4][0] == 0 if args.config in CONFIGS else False
+    if no_ins:
+        host = [(o, k, None) for o, k, _ in host]
     n_local = host[0][0].numel()
     outs = [torch.empty(n_local, dtype=torch.uint8).pin_memory() for _ in range(steps)]
     reps = 3 if S.R <= 10_000_000 else 1
-    t_pipes = []
+    t_pipes, zc = [], False
     for _rep in range(reps):
         g, local_g = S.create()
         if world == 1:
@@ -763,18 +767,21 @@ def run_e2e(args, S, inputs, W, steps, world, dev):
                     g.batch_host_async(*host[W + j], out=outs[j])
             torch.cuda.synchronize()
             t_pipes.append(time.perf_counter() - t0)
+            zc = local_g.stats().get("zero_copy_batches", 0) > 0
         else:
             bufs = [torch.empty_like(x, device=dev) for x in inputs[0]]
             for b in range(W):
                 for d_, h_ in zip(bufs, host[b]):
-                    d_.copy_(h_, non_blocking=True)
+                    if h_ is not None:
+                        d_.copy_(h_, non_blocking=True)
                 g.batch(*bufs)
             torch.cuda.synchronize()
             barrier(world)
             t0 = time.perf_counter()
             for j in range(steps):
                 for d_, h_ in zip(bufs, host[W + j]):
-                    d_.copy_(h_, non_blocking=True)
+                    if h_ is not None:
+                        d_.copy_(h_, non_blocking=True)
                 r = g.batch(*bufs)
                 outs[j].copy_(r, non_blocking=True)
             torch.cuda.synchronize()
@@ -782,8 +789,15 @@ def run_e2e(args, S, inputs, W, steps, world, dev):
         S.close(g)
     t_pipe = sorted(t_pipes)[len(t_pipes) // 2]
     B = S.B
+    # H2D per step: op (1 B) + key (4 B) copied, and the values: copied (4 B per op), or --
+    # when the library reads them zero-copy from the pinned buffer -- 4 B per Insert
+    n_ins = sum(int((host[W + j][0] == 1).sum()) for j in range(steps)) / max(steps, 1)
+    h2d = B * 5 + (0 if no_ins else (int(round(4 * n_ins * world)) if zc else B * 4))
     return {"value": round(B * steps / t_pipe / 1e6, 3), "unit": "Mops/s",
-            "h2d_bytes_per_step": B * 9, "d2h_bytes_per_step": B,
+            "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": B,
+            "values": ("none (no Inserts in the workload: values = NULL)" if no_ins else
+                       "Insert values read zero-copy from the pinned host buffer by the search kernel"
+                       if zc else "copied"),
             "how": ("gfsl_batch_host_async on a caller stream, K steps back to back from pinned host "
                     "buffers, wall clock from the first call to the last result in host memory"
                     if world == 1 else

@@ -204,7 +204,11 @@ gfsl_status gfsl_batch_host(gfsl_t h, const uint8_t *op_types, const uint32_t *k
  * `stream` (its inputs are host memory); it is ordered after the handle's earlier
  * batches, as every batch is.  The host buffers must stay
  * valid and unmodified until then, and must be pinned (page-locked) for the copies to
- * be asynchronous (pageable buffers still work, with synchronous copies).
+ * be asynchronous (pageable buffers still work, with synchronous copies).  `values` may
+ * be NULL (all values 0; nothing copied) -- only Inserts read a value.  With
+ * GFSL_ZC_VALUES=1 in the environment at gfsl_create and a mapped pinned `values`, the
+ * search kernel reads each Insert's value from it directly instead of the array being
+ * copied (faster only when Inserts are rare).
  */
 gfsl_status gfsl_batch_host_async(gfsl_t h, const uint8_t *op_types, const uint32_t *keys,
                                   const uint32_t *values, uint8_t *results, uint64_t n,
@@ -291,7 +295,8 @@ typedef struct gfsl_stats {
   uint64_t kernel_launches; /* libgfsl kernels enqueued by gfsl_batch calls so far */
   uint64_t library_launches;/* library (CUB radix sort, combining mode) kernels, estimated */
   uint64_t grouped;         /* Insert/Delete ops applied in a chunk group of >= 2 (R40) */
-  uint64_t reserved[1];
+  uint64_t zero_copy_batches; /* host-path batches whose Insert values the kernel read from
+                               the caller's mapped pinned buffer (no copy) */
 } gfsl_stats;
 gfsl_status gfsl_get_stats(gfsl_t h, gfsl_stats *out);
 

@@ -61,7 +61,7 @@ class gfsl_stats(ctypes.Structure):
                 ("contains_reads_l0", ctypes.c_uint64), ("contains_ops", ctypes.c_uint64),
                 ("mutations", ctypes.c_uint64), ("kernel_launches", ctypes.c_uint64),
                 ("library_launches", ctypes.c_uint64), ("grouped", ctypes.c_uint64),
-                ("reserved", ctypes.c_uint64 * 1)]
+                ("zero_copy_batches", ctypes.c_uint64)]
 
 
 class gfsl_meta(ctypes.Structure):

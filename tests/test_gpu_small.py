@@ -168,3 +168,36 @@ def test_coarse_directory_16bit_window(layout, monkeypatch):
         keys = np.union1d(keys, ins).astype(np.uint32)
         assert g.check().violations == 0
     g.close()
+
+
+def test_host_async_zero_copy_values(monkeypatch):
+    """With GFSL_ZC_VALUES=1, gfsl_batch_host_async reads the Insert values from a mapped
+    pinned buffer instead of copying the value array (a pageable buffer is still copied):
+    results and stored values vs Oracle-A, and the library's count of zero-copy batches."""
+    R = 50_000
+    monkeypatch.setenv("GFSL_ZC_VALUES", "1")
+    g = GFSL(R)
+    o = OracleMap(R)
+    rng = np.random.default_rng(77)
+    k0 = rng.permutation(R)[: R // 2].astype(np.uint32)
+    g.batch(*to_dev(np.ones(k0.size, np.uint8), k0, k0 + 5))
+    o.batch(np.ones(k0.size, np.uint8), k0, k0 + 5)
+    outs = []
+    for b in range(8):
+        key = rng.choice(R, 20_000, replace=False).astype(np.uint32)
+        op = rng.choice([0, 1, 2], key.size, p=[0.5, 0.3, 0.2]).astype(np.uint8)
+        val = rng.integers(0, 2**32, key.size, dtype=np.uint64).astype(np.uint32)
+        pinned = b % 2 == 0
+        t = (torch.from_numpy(op), torch.from_numpy(key.view(np.int32)), torch.from_numpy(val.view(np.int32)))
+        if pinned:
+            t = tuple(x.pin_memory() for x in t)
+        outs.append((g.batch_host_async(*t), o.batch(op, key, val), t))
+    torch.cuda.synchronize()
+    for r, e, _ in outs:
+        assert np.array_equal(r.numpy(), e)
+    dk, dv = g.export()
+    ok, ov = o.export()
+    assert np.array_equal(dk.cpu().numpy().view(np.uint32), ok)
+    assert np.array_equal(dv.cpu().numpy().view(np.uint32), ov)
+    assert g.stats()["zero_copy_batches"] == 4
+    g.close()
