@@ -63,6 +63,10 @@ void gfsl_internal_set_error(const std::string &s) { set_last_error(s); }  // gf
 #define GFSL_DERIVE_PATH 0
 #endif
 
+#ifndef GFSL_REBUILD_MUT_RULE
+#define GFSL_REBUILD_MUT_RULE 1  // R29's mutation rule (0: the ops rule alone, round 1)
+#endif
+
 #ifndef GFSL_SMALL_BATCH_DEFAULT
 #define GFSL_SMALL_BATCH_DEFAULT 0
 #endif
@@ -109,6 +113,8 @@ struct gfsl {
   uint64_t capacity = 0;           // max live keys (gfsl_create)
   uint64_t ops_since_rebuild = 0;  // default rebuild policy (R29)
   uint64_t ops_at_rebuild = 0;     // h->ops after the batch of the last rebuild
+  unsigned long long *h_mut = nullptr;  // mapped: cumulative mutations (update kernel)
+  uint64_t muts_at_rebuild = 0;    // *h_mut as known at the last rebuild
   bool upper_stale = false;        // R33: a lazy batch ran since the last rebuild
   bool upkeep_pending = false;     // R33: lazy batches skipped the upkeep sweep
   uint64_t launches = 0, lib_launches = 0;  // our kernels / CUB's (combining sort) enqueued by batches
@@ -424,12 +430,23 @@ static void launch_update(gfsl *h, const BatchIn &in, cudaStream_t s, cudaEvent_
     h->ops_since_rebuild += h->n_policy;
     const uint64_t L = std::min(h->capacity, h->ops_at_rebuild);
     rebuild = 2 * h->ops_since_rebuild >= (uint64_t)(2 * GFSL_REBUILD_DEFAULT_WEAR) * L;
+    // and the structure must have worn: successful mutations since the last rebuild >= L/2
+    // (the device's count, read from mapped memory, a batch or two behind).  Both rules
+    // cross together at the paper's [10,10,80] mix; a Contains-heavy mix rebuilds far less
+    // often (M1-1-98: every ~80 batches instead of 8); a map growing from empty keeps the ops
+    // rule (every op mutates).  Not in serial mode: its rule must stay deterministic (host
+    // counts only), since its pools are compared byte for byte with Oracle-B's
+    if (GFSL_REBUILD_MUT_RULE && rebuild && !h->cfg.serial_updates) {
+      const uint64_t muts = *(volatile unsigned long long *)h->h_mut - h->muts_at_rebuild;
+      rebuild = 2 * muts >= L;
+    }
   } else {
     rebuild = h->cfg.rebuild_every != GFSL_REBUILD_NEVER && (h->batches + 1) % h->cfg.rebuild_every == 0;
   }
   if (rebuild) {
     h->ops_since_rebuild = 0;
     h->ops_at_rebuild = h->ops + h->n_policy;
+    h->muts_at_rebuild = *(volatile unsigned long long *)h->h_mut;
     launch_rebuild<N>(h, s);
   }
 }
@@ -568,6 +585,7 @@ static void free_all(gfsl *h) {
   cudaFree(h->snap_zh);
   if (h->h_error) cudaFreeHost(h->h_error);
   if (h->h_bump) cudaFreeHost(h->h_bump);
+  if (h->h_mut) cudaFreeHost(h->h_mut);
   if (h->last) cudaEventDestroy(h->last);
   for (auto &ev : h->phase_ev)
     for (auto &e : ev) cudaEventDestroy(e);
@@ -656,6 +674,9 @@ extern "C" gfsl_t gfsl_create_ex(uint64_t key_range, uint64_t capacity, const gf
   h->h_bump[0] = 1;
   h->h_bump[1] = N - 1;
   if ((e = cudaHostGetDevicePointer(&h->d.bump_host, h->h_bump, 0)) != cudaSuccess) return fail("cudaHostGetDevicePointer", e);
+  if ((e = cudaHostAlloc(&h->h_mut, 8, cudaHostAllocMapped)) != cudaSuccess) return fail("cudaHostAlloc", e);
+  *h->h_mut = 0;
+  if ((e = cudaHostGetDevicePointer(&h->d.mut_host, h->h_mut, 0)) != cudaSuccess) return fail("cudaHostGetDevicePointer", e);
   setup_l2_window(h);
   {
     RebuildBufs &b = h->rb;
@@ -1147,6 +1168,7 @@ static gfsl_status enqueue_bulk(gfsl *h, const uint8_t *ops, const uint32_t *key
   h->live_ub = std::min(h->capacity, h->live_ub + n);
   h->ops_since_rebuild = 0;
   h->ops_at_rebuild = h->ops;
+  h->muts_at_rebuild = *(volatile unsigned long long *)h->h_mut;
   return GFSL_OK;
 }
 
@@ -1180,6 +1202,7 @@ extern "C" gfsl_status gfsl_rebuild(gfsl_t h, void *stream) {
   CK(cudaEventRecord(h->last, s));
   h->ops_since_rebuild = 0;
   h->ops_at_rebuild = h->ops;
+  h->muts_at_rebuild = *(volatile unsigned long long *)h->h_mut;
   return GFSL_OK;
 }
 

@@ -113,6 +113,8 @@ struct DevState {
   uint32_t upd_prefetch;  // the update kernel prefetches each record's chunk into L2 (host:
                           // while level 0 fits the L2; beyond it the extra request costs
                           // more than it saves -- C5 update 2.21 vs 2.55 ms, round 2)
+  unsigned long long *mut_host;  // mapped pinned host copy of the cumulative mutation count
+                                 // (written by the update kernel; the rebuild policy, R29)
   uint32_t *bump_host;  // mapped pinned host copy of bump[0..1], written by the search kernel
                         // at its start (the counters after the previous batch; host heuristics)
 };
